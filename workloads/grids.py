@@ -320,3 +320,28 @@ def random_spd_pattern(n: int, density: float, seed: int, dup: float = 0.0, uppe
     colptr = np.zeros(n + 1, dtype=np.int64)
     np.cumsum(np.bincount(cc, minlength=n), out=colptr[1:])
     return CSC(n, colptr, rr.astype(np.int32), vv)
+
+
+def manufactured(n: int, Lp: np.ndarray, Li: np.ndarray, perm: np.ndarray, seed: int = 1234):
+    """Manufactured SPD matrix with an exactly known integer factor
+    (SURVEY.md Sec. 8(c) "Manufactured exact factor"): L0 = +1 on the given
+    off-diagonal structure (final labels, struct(L_j) ascending with j first),
+    diagonal 2^p_j with p_j in {1,2,3} drawn from PCG64(seed); A = L0 L0^T,
+    returned as the lower CSC in ORIGINAL labels (A_orig[perm[i], perm[j]] =
+    A[i, j]).  Returns (CSC, L0 values aligned with Li)."""
+    import scipy.sparse as sp
+    rng = np.random.Generator(np.random.PCG64(seed))
+    p = rng.integers(1, 4, n)
+    Lx = np.ones(Li.size)
+    Lx[Lp[:-1]] = 2.0 ** p                       # first entry of each column = diagonal
+    L0 = sp.csc_matrix((Lx, Li, Lp), shape=(n, n))
+    A = (L0 @ L0.T).tocoo()
+    perm = np.asarray(perm, dtype=np.int64)
+    r, c = perm[A.row], perm[A.col]
+    keep = r >= c
+    r, c, v = r[keep], c[keep], A.data[keep]
+    order = np.lexsort((r, c))
+    r, c, v = r[order], c[order], v[order]
+    colptr = np.zeros(n + 1, dtype=np.int64)
+    np.cumsum(np.bincount(c, minlength=n), out=colptr[1:])
+    return CSC(n, colptr, r.astype(np.int32), v), Lx
