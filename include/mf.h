@@ -1,0 +1,148 @@
+/*
+ * mf.h -- C ABI of the B200-native multifrontal sparse SPD Cholesky hot path.
+ *
+ * The problem statement is the paper's [PAPER.md L7, Sec. I]: "For SPD linear
+ * systems, the solution involves a Cholesky factorization of the coefficient
+ * matrix A into LL^T, followed by a forward triangular solve Ly = b and a
+ * backward triangular solve L^T x = y."  The factorization is the supernodal
+ * multifrontal method of [PAPER.md L27, Sec. II-A]: a postorder traversal of the
+ * supernodal elimination tree; per supernode n the frontal matrix F^n is built
+ * from A's entries and the children's update matrices by extend-add, then the
+ * factor-update (F-U) step -- potrf on L1^n (k x k), trsm on L2^n (m x k), and
+ * U^n = U^n - L2^n L2^nT (syrk) [Fig. 1, PAPER.md L33-65] -- produces L and
+ * the update matrix passed to the parent.
+ *
+ * Conventions:
+ *   - Input matrix: 0-based CSC, n columns.  colptr: int64[n+1] (monotone,
+ *     colptr[0] = 0); rowind: int32[colptr[n]] (need not be sorted).  Only
+ *     entries with row >= col are read (LAPACK uplo='L'); upper entries are
+ *     ignored, so a full symmetric CSC works too.  Duplicates are summed in
+ *     input order.  A missing diagonal counts as 0 (=> not SPD).
+ *   - perm: int32[n], perm[k] = original index of the k-th pivot (new -> old,
+ *     as in A(p,p)).  The library composes it with an elimination-tree
+ *     postorder; mf_get_perm() returns the composition ("final perm").
+ *     perm must be non-NULL (this library ships no ordering; callers pass a
+ *     nested-dissection order, see workloads/grids.py).
+ *   - values, b, x: float64 arrays that may be HOST or DEVICE pointers
+ *     (detected with cudaPointerGetAttributes).  They are borrowed for the
+ *     duration of the call only.  x is caller-allocated (n doubles) and must
+ *     not alias b.
+ *   - Ownership: the ctx owns the symbolic plan, the device arena (L panels
+ *     and update matrices) and its CUDA stream usage until mf_destroy().
+ *   - State machine: create -> analyze -> factor -> solve*; factor may repeat
+ *     with new values of the same pattern; analyze resets.  Calls out of order
+ *     return MF_ERR_STATE.
+ *   - Errors: 0 = OK; negative = usage/resource errors (below); positive
+ *     MF_NOT_SPD = a pivot was <= 0 or NaN: info.failed_col holds the ORIGINAL
+ *     index of the first failing pivot in final-perm order, the factor is
+ *     invalid and mf_solve returns MF_ERR_STATE.
+ *   - Thread safety: one ctx per host thread; no global mutable state.
+ */
+#ifndef MF_H
+#define MF_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define MF_OK 0
+#define MF_NOT_SPD 1
+#define MF_ERR_ARG (-1)
+#define MF_ERR_STATE (-2)
+#define MF_ERR_NOMEM (-3)
+#define MF_ERR_CUDA (-4)
+#define MF_ERR_NCCL (-5)
+
+typedef struct mf_ctx mf_ctx;
+
+typedef struct {
+    int32_t amalgamate;       /* 1 = SURVEY Appendix-B relaxed rule (default), 0 = fundamental supernodes */
+    int32_t nrelax[3];        /* default {4, 16, 48}                                              */
+    double zrelax[3];         /* default {0.8, 0.1, 0.05}                                         */
+    int32_t small_front_max;  /* fronts of order <= this use the batched shared-memory kernel      */
+    int32_t panel_w;          /* large-front diagonal block width (multiple of 16, <= 64)          */
+    int32_t device;           /* CUDA device ordinal (-1 = current)                                */
+    int32_t host_only;        /* 1 = symbolic analysis + planning only, no device (mf_factor/mf_solve
+                                 then return MF_ERR_STATE); lets CPU-only hosts inspect the plan   */
+    void *stream;             /* cudaStream_t to run on (NULL = the ctx creates its own)           */
+} mf_options;
+
+typedef struct {
+    int64_t n;
+    int64_t nnzA;             /* entries read (row >= col) */
+    int64_t nnzL;             /* true nnz(L) = sum of column counts */
+    int64_t nnzL_stored;      /* sum over supernodes of k(k+1)/2 + k m */
+    int64_t panel_words;      /* sum over supernodes of ldL * k (device storage of L) */
+    int64_t flops_true;       /* sum cc_j^2 (SURVEY Sec. 8(a) flop accounting) */
+    int64_t flops_exec;       /* sum over fronts of k m^2 + m k(k+1) + k(k+1)(2k+1)/6 */
+    int32_t nfund;            /* fundamental supernodes */
+    int32_t nsuper;           /* supernodes after amalgamation */
+    int32_t nlevels;          /* levels of the bottom-up schedule */
+    int32_t max_front;        /* largest f = k + m */
+    int64_t rows_total;       /* sum over supernodes of f (length of the row lists) */
+    int64_t failed_col;       /* original index of the first failing pivot, or -1 */
+    int64_t workspace_bytes;  /* device bytes held by the ctx */
+    int64_t launches_factor;  /* kernel launches issued by one mf_factor */
+    double t_analyze;         /* seconds (host wall) of the last mf_analyze */
+    double t_factor;          /* seconds (device events) of the last mf_factor */
+    double t_solve;           /* seconds (device events) of the last mf_solve */
+} mf_info;
+
+/* Fill *opt with the defaults. */
+int mf_default_options(mf_options *opt);
+
+/* Create a context.  opt may be NULL (defaults). */
+int mf_create(mf_ctx **ctx, const mf_options *opt);
+
+/* Symbolic analysis + device planning for the pattern (colptr, rowind) under
+ * the order perm.  Host arrays only.  Uploads the
+ * flat plan arrays and allocates the device arena. */
+int mf_analyze(mf_ctx *ctx, int64_t n, const int64_t *colptr, const int32_t *rowind,
+               const int32_t *perm);
+
+/* Numeric factorization A = L L^T (rows a1-a8): values[colptr[n]] aligned with
+ * rowind, host or device.  Runs on the ctx stream and synchronizes it before
+ * returning (the NOT_SPD flag is read back). */
+int mf_factor(mf_ctx *ctx, const double *values);
+
+/* x = A^{-1} b through L y = P b, L^T z = y, x = P^T z.  b, x host or device. */
+int mf_solve(mf_ctx *ctx, const double *b, double *x);
+
+int mf_get_info(const mf_ctx *ctx, mf_info *out);
+
+/* final_perm[n]: perm composed with the postorder (new -> old). */
+int mf_get_perm(const mf_ctx *ctx, int32_t *final_perm);
+
+/* Elimination tree (final labels) and column counts: parent[n] (-1 = root),
+ * colcount[n] (incl. diagonal).  Host buffers. */
+int mf_get_etree(const mf_ctx *ctx, int32_t *parent, int64_t *colcount);
+
+/* Supernode partition after amalgamation (host buffers):
+ * sn_first[nsuper+1], sn_parent[nsuper], sn_rowptr[nsuper+1],
+ * sn_rows[rows_total] (R_s ascending, first k entries = the pivot columns).
+ * fund_first[nfund+1] = fundamental partition (may be NULL). */
+int mf_get_supernodes(const mf_ctx *ctx, int32_t *sn_first, int32_t *sn_parent, int64_t *sn_rowptr,
+                      int32_t *sn_rows, int32_t *fund_first);
+
+/* Copy the L panel of supernode s to host memory: out[f * k], column-major
+ * with leading dimension f (rows R_s, columns cols(s)); the strict upper
+ * triangle of the k x k block is zero.  Requires a successful mf_factor. */
+int mf_export_panel(const mf_ctx *ctx, int32_t s, double *out);
+
+/* Diagonal of L in final-perm order: out[n] (host).  log det A = 2 sum log out[j]. */
+int mf_export_diag(const mf_ctx *ctx, double *out);
+
+/* Copy every panel (supernode order, each f*k as above) to host: out[sum f*k]. */
+int mf_export_L(const mf_ctx *ctx, double *out);
+
+void mf_destroy(mf_ctx *ctx);
+
+const char *mf_strerror(int code);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MF_H */

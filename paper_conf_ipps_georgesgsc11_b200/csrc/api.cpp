@@ -1,0 +1,484 @@
+// api.cpp -- the C ABI (include/mf.h): state machine, device arena, and the
+// level-by-level driver of the factor-update hot path.
+//
+// mf_factor is the postorder traversal of PAPER.md L27 (Sec. II-A) realised as
+// a bottom-up level schedule (children always in a lower level than their
+// parent): per level, the small fronts run in one batched fused launch per size
+// class, the large fronts in the blocked path (assembly; per diagonal block:
+// potrf, trsm, DMMA trailing update; then the DMMA syrk on U^n).  Everything
+// stays resident in HBM; the only host<->device traffic is the optional upload
+// of `values` and the 4-byte NOT_SPD flag.
+#include <algorithm>
+#include <chrono>
+#include <climits>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <vector>
+
+#include "kernels.cuh"
+#include "mf.h"
+#include "mf_plan.h"
+
+using namespace mf;
+
+struct mf_ctx {
+    Options opt;
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    int state = 0;   // 0 created, 1 analyzed, 2 factored (ok), 3 factor failed
+    bool host_only = false;
+    Symbolic S;
+    Plan P;
+    mf_info info{};
+    std::vector<void *> allocs;
+    DevPlan d{};
+    // device copies of schedule arrays
+    int32_t *d_small = nullptr, *d_large = nullptr, *d_asm = nullptr, *d_trsm = nullptr, *d_levels = nullptr;
+    int32_t *d_sn_rows = nullptr;
+    int64_t *d_sn_rowptr = nullptr;
+    GemmProb *d_probs = nullptr;
+    TileTask *d_tiles = nullptr;
+    double *d_values = nullptr;
+    double *d_y = nullptr, *d_bx = nullptr;
+    int *d_failed = nullptr;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    int64_t launches = 0;
+};
+
+namespace {
+
+int cuda_err(cudaError_t e) {
+    if (e == cudaSuccess) return MF_OK;
+    fprintf(stderr, "[libmf] CUDA error: %s\n", cudaGetErrorString(e));
+    return e == cudaErrorMemoryAllocation ? MF_ERR_NOMEM : MF_ERR_CUDA;
+}
+
+#define CK(x)                            \
+    do {                                 \
+        int _r = cuda_err(x);            \
+        if (_r != MF_OK) return _r;      \
+    } while (0)
+
+template <class T>
+int dev_upload(mf_ctx *c, T **dst, const std::vector<T> &src) {
+    size_t bytes = std::max<size_t>(src.size(), 1) * sizeof(T);
+    void *p = nullptr;
+    CK(cudaMalloc(&p, bytes));
+    c->allocs.push_back(p);
+    if (!src.empty()) CK(cudaMemcpy(p, src.data(), src.size() * sizeof(T), cudaMemcpyHostToDevice));
+    *dst = (T *)p;
+    return MF_OK;
+}
+
+int dev_alloc(mf_ctx *c, void **dst, size_t bytes) {
+    void *p = nullptr;
+    CK(cudaMalloc(&p, std::max<size_t>(bytes, 16)));
+    c->allocs.push_back(p);
+    *dst = p;
+    return MF_OK;
+}
+
+void free_device(mf_ctx *c) {
+    for (void *p : c->allocs) cudaFree(p);
+    c->allocs.clear();
+    c->d = DevPlan{};
+}
+
+bool is_device_ptr(const void *p) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+
+void fill_info(mf_ctx *c, int64_t n, int with_device) {
+    const Symbolic &S = c->S;
+    const Plan &P = c->P;
+    mf_info &I = c->info;
+    I = mf_info{};
+    I.n = n;
+    I.nnzA = S.nnzA_read;
+    I.nnzL = S.nnzL;
+    I.nnzL_stored = S.stored_L;
+    I.panel_words = P.L_words - 2;
+    I.flops_true = S.flops;
+    I.flops_exec = S.exec_flops;
+    I.nfund = (int32_t)S.fund_first.size() - 1;
+    I.nsuper = P.nsuper;
+    I.nlevels = P.nlevels;
+    I.max_front = P.max_front;
+    I.rows_total = P.rows_total;
+    I.failed_col = -1;
+    int64_t ws = 0;
+    ws += (P.L_words + P.U_words + P.fv_words + 2 * std::max<int64_t>(n, 1) + S.nnz_in) * 8;
+    ws += (int64_t)P.tiles.size() * sizeof(TileTask) + (int64_t)P.probs.size() * sizeof(GemmProb);
+    ws += (int64_t)(S.bvidx.size() * 16 + S.brow.size() * 16 + P.relmap.size() * 4);
+    I.workspace_bytes = with_device ? ws : 0;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *mf_strerror(int code) {
+    switch (code) {
+        case MF_OK: return "ok";
+        case MF_NOT_SPD: return "matrix is not symmetric positive definite";
+        case MF_ERR_ARG: return "invalid argument";
+        case MF_ERR_STATE: return "call out of order";
+        case MF_ERR_NOMEM: return "out of memory";
+        case MF_ERR_CUDA: return "CUDA error";
+        case MF_ERR_NCCL: return "NCCL error";
+        default: return "unknown error";
+    }
+}
+
+int mf_default_options(mf_options *o) {
+    if (!o) return MF_ERR_ARG;
+    Options d;
+    o->amalgamate = d.amalgamate;
+    for (int i = 0; i < 3; i++) {
+        o->nrelax[i] = d.nrelax[i];
+        o->zrelax[i] = d.zrelax[i];
+    }
+    o->small_front_max = d.small_front_max;
+    o->panel_w = d.panel_w;
+    o->device = -1;
+    o->stream = nullptr;
+    return MF_OK;
+}
+
+int mf_create(mf_ctx **out, const mf_options *o) {
+    if (!out) return MF_ERR_ARG;
+    *out = nullptr;
+    mf_options def;
+    mf_default_options(&def);
+    if (!o) o = &def;
+    if (o->panel_w < 16 || o->panel_w > 64 || (o->panel_w % 16)) return MF_ERR_ARG;
+    if (o->small_front_max < 8 || !small_front_smem_ok(o->small_front_max)) return MF_ERR_ARG;
+    mf_ctx *c = new (std::nothrow) mf_ctx();
+    if (!c) return MF_ERR_NOMEM;
+    c->opt.amalgamate = o->amalgamate;
+    for (int i = 0; i < 3; i++) {
+        c->opt.nrelax[i] = o->nrelax[i];
+        c->opt.zrelax[i] = o->zrelax[i];
+    }
+    c->opt.small_front_max = o->small_front_max;
+    c->opt.panel_w = o->panel_w;
+    c->host_only = o->host_only != 0;
+    c->info.failed_col = -1;
+    if (c->host_only) {   // symbolic analysis + plan only; never touches CUDA
+        *out = c;
+        return MF_OK;
+    }
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+        cudaGetLastError();
+        delete c;
+        fprintf(stderr, "[libmf] no CUDA device: the product path has no CPU fallback\n");
+        return MF_ERR_CUDA;
+    }
+    if (o->device >= 0) {
+        if (cudaSetDevice(o->device) != cudaSuccess) {
+            delete c;
+            return MF_ERR_CUDA;
+        }
+    }
+    cudaGetDevice(&c->device);
+    if (o->stream) {
+        c->stream = (cudaStream_t)o->stream;
+    } else {
+        if (cudaStreamCreateWithFlags(&c->stream, cudaStreamNonBlocking) != cudaSuccess) {
+            delete c;
+            return MF_ERR_CUDA;
+        }
+        c->own_stream = true;
+    }
+    cudaEventCreate(&c->ev0);
+    cudaEventCreate(&c->ev1);
+    c->info.failed_col = -1;
+    *out = c;
+    return MF_OK;
+}
+
+void mf_destroy(mf_ctx *c) {
+    if (!c) return;
+    if (c->host_only) {
+        delete c;
+        return;
+    }
+    cudaSetDevice(c->device);
+    if (c->stream) cudaStreamSynchronize(c->stream);
+    free_device(c);
+    if (c->ev0) cudaEventDestroy(c->ev0);
+    if (c->ev1) cudaEventDestroy(c->ev1);
+    if (c->own_stream) cudaStreamDestroy(c->stream);
+    delete c;
+}
+
+int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowind, const int32_t *perm) {
+    if (!c) return MF_ERR_ARG;
+    auto t0 = std::chrono::steady_clock::now();
+    if (!c->host_only) {
+        CK(cudaSetDevice(c->device));
+        cudaStreamSynchronize(c->stream);
+        free_device(c);
+    }
+    c->state = 0;
+    int st = analyze_symbolic(n, colptr, rowind, perm, c->opt, c->S);
+    if (st) return st;
+    st = build_plan(c->S, c->opt, c->P);
+    if (st) return st;
+    if (c->host_only) {
+        fill_info(c, n, 0);
+        c->info.t_analyze = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+        c->state = 1;
+        return MF_OK;
+    }
+    const Symbolic &S = c->S;
+    const Plan &P = c->P;
+    DevPlan &d = c->d;
+    int r;
+#define UP(dst, vec)                                   \
+    if ((r = dev_upload(c, dst, vec)) != MF_OK) return r;
+    int32_t *sn_first, *sn_k, *sn_f, *sn_ld, *child_ptr, *child_list, *relmap, *blrow, *perm_d;
+    int64_t *L_off, *U_off, *fv_off, *relmap_ptr, *bcolptr, *bvptr, *bvidx;
+    UP(&sn_first, S.sn_first);
+    UP(&sn_k, P.sn_k);
+    UP(&sn_f, P.sn_f);
+    UP(&sn_ld, P.sn_ld);
+    UP(&L_off, P.L_off);
+    UP(&U_off, P.U_off);
+    UP(&fv_off, P.fv_off);
+    UP(&child_ptr, P.child_ptr);
+    UP(&child_list, P.child_list);
+    UP(&relmap_ptr, P.relmap_ptr);
+    UP(&relmap, P.relmap);
+    UP(&bcolptr, S.bcolptr);
+    UP(&blrow, P.blrow);
+    UP(&bvptr, S.bvptr);
+    UP(&bvidx, S.bvidx);
+    UP(&perm_d, S.perm);
+    UP(&c->d_small, P.small_list);
+    UP(&c->d_large, P.large_list);
+    UP(&c->d_asm, P.asm_tasks);
+    UP(&c->d_trsm, P.trsm_tasks);
+    UP(&c->d_levels, P.level_list);
+    UP(&c->d_sn_rows, S.sn_rows);
+    UP(&c->d_sn_rowptr, S.sn_rowptr);
+    UP(&c->d_probs, P.probs);
+    UP(&c->d_tiles, P.tiles);
+#undef UP
+    d.sn_first = sn_first;
+    d.sn_k = sn_k;
+    d.sn_f = sn_f;
+    d.sn_ld = sn_ld;
+    d.L_off = L_off;
+    d.U_off = U_off;
+    d.fv_off = fv_off;
+    d.child_ptr = child_ptr;
+    d.child_list = child_list;
+    d.relmap_ptr = relmap_ptr;
+    d.relmap = relmap;
+    d.bcolptr = bcolptr;
+    d.blrow = blrow;
+    d.bvptr = bvptr;
+    d.bvidx = bvidx;
+    d.perm = perm_d;
+    void *p;
+    if ((r = dev_alloc(c, &p, P.L_words * sizeof(double))) != MF_OK) return r;
+    d.L = (double *)p;
+    if ((r = dev_alloc(c, &p, P.U_words * sizeof(double))) != MF_OK) return r;
+    d.U = (double *)p;
+    if ((r = dev_alloc(c, &p, P.fv_words * sizeof(double))) != MF_OK) return r;
+    d.fv = (double *)p;
+    if ((r = dev_alloc(c, &p, sizeof(int) * 4)) != MF_OK) return r;
+    c->d_failed = (int *)p;
+    d.failed = c->d_failed;
+    if ((r = dev_alloc(c, &p, std::max<int64_t>(S.nnz_in, 1) * sizeof(double))) != MF_OK) return r;
+    c->d_values = (double *)p;
+    if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(n, 1) * sizeof(double))) != MF_OK) return r;
+    c->d_y = (double *)p;
+    if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(n, 1) * sizeof(double))) != MF_OK) return r;
+    c->d_bx = (double *)p;
+    // the L arena starts zeroed once so that never-written padding words are defined
+    CK(cudaMemsetAsync(d.L, 0, P.L_words * sizeof(double), c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+
+    fill_info(c, n, 1);
+    mf_info &I = c->info;
+    I.t_analyze = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
+    c->state = 1;
+    return MF_OK;
+}
+
+int mf_factor(mf_ctx *c, const double *values) {
+    if (!c || !values) return MF_ERR_ARG;
+    if (c->state < 1 || c->host_only) return MF_ERR_STATE;
+    CK(cudaSetDevice(c->device));
+    const Plan &P = c->P;
+    const DevPlan &d = c->d;
+    cudaStream_t st = c->stream;
+    const int64_t nv = (int64_t)c->S.bvidx.size() ? (int64_t)c->S.bvidx.size() : 0;
+    CK(cudaEventRecord(c->ev0, st));
+    const double *vals = values;
+    if (!is_device_ptr(values)) {
+        // bvidx indexes the caller's array; copy the whole array (colptr[n] entries)
+        const int64_t nall = c->S.nnz_in;
+        (void)nv;
+        if (nall > 0) CK(cudaMemcpyAsync(c->d_values, values, nall * sizeof(double), cudaMemcpyHostToDevice, st));
+        vals = c->d_values;
+    }
+    int64_t launches = 0;
+    launch_init_failed(c->d_failed, st);
+    launches++;
+    for (int l = 0; l < P.nlevels; l++) {
+        const LevelPlan &LP = P.levels[l];
+        for (int cls = 0; cls < kSmallClasses; cls++) {
+            const int a = LP.small_class_off[cls], b = LP.small_class_off[cls + 1];
+            if (b > a) {
+                launch_small_fronts(d, c->d_small + a, b - a, P.small_class_fmax[cls], vals, st);
+                launches++;
+            }
+        }
+        if (LP.nlarge == 0) continue;
+        launch_assemble(d, c->d_asm + 2 * LP.asm_off, LP.nasm, vals, st);
+        launches++;
+        for (const auto &W : LP.waves) {
+            launch_potrf_diag(d, c->d_large + LP.large_off, W.nactive, W.j0, P.w, st);
+            launch_trsm_panel(d, c->d_trsm + 2 * W.trsm_off, W.ntrsm, W.j0, P.w, st);
+            launch_update(d, c->d_probs, c->d_tiles + W.tile_off, W.ntile, st);
+            launches += 1 + (W.ntrsm > 0) + (W.ntile > 0);
+        }
+        if (LP.syrk_ntile > 0) {
+            launch_update(d, c->d_probs, c->d_tiles + LP.syrk_tile_off, LP.syrk_ntile, st);
+            launches++;
+        }
+    }
+    CK(cudaGetLastError());
+    int failed = INT_MAX;
+    CK(cudaMemcpyAsync(&failed, c->d_failed, sizeof(int), cudaMemcpyDeviceToHost, st));
+    CK(cudaEventRecord(c->ev1, st));
+    CK(cudaStreamSynchronize(st));
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, c->ev0, c->ev1);
+    c->info.t_factor = ms * 1e-3;
+    c->info.launches_factor = launches;
+    if (failed != INT_MAX) {
+        c->info.failed_col = c->S.perm[failed];
+        c->state = 3;
+        return MF_NOT_SPD;
+    }
+    c->info.failed_col = -1;
+    c->state = 2;
+    return MF_OK;
+}
+
+int mf_solve(mf_ctx *c, const double *b, double *x) {
+    if (!c || !b || !x || b == x) return MF_ERR_ARG;
+    if (c->state != 2 || c->host_only) return MF_ERR_STATE;
+    CK(cudaSetDevice(c->device));
+    const Plan &P = c->P;
+    const DevPlan &d = c->d;
+    cudaStream_t st = c->stream;
+    const int64_t n = c->S.n;
+    CK(cudaEventRecord(c->ev0, st));
+    const bool bdev = is_device_ptr(b), xdev = is_device_ptr(x);
+    const double *bd = b;
+    if (!bdev) {
+        CK(cudaMemcpyAsync(c->d_bx, b, n * sizeof(double), cudaMemcpyHostToDevice, st));
+        bd = c->d_bx;
+    }
+    launch_permute_in(d, bd, c->d_y, n, st);
+    for (int l = 0; l < P.nlevels; l++)
+        launch_fwd_solve(d, c->d_levels + P.level_ptr[l], P.level_ptr[l + 1] - P.level_ptr[l], c->d_y, st);
+    for (int l = P.nlevels - 1; l >= 0; l--)
+        launch_bwd_solve(d, c->d_levels + P.level_ptr[l], P.level_ptr[l + 1] - P.level_ptr[l], c->d_y,
+                         c->d_sn_rows, c->d_sn_rowptr, st);
+    double *xd = xdev ? x : c->d_bx;
+    launch_permute_out(d, c->d_y, xd, n, st);
+    if (!xdev) CK(cudaMemcpyAsync(x, c->d_bx, n * sizeof(double), cudaMemcpyDeviceToHost, st));
+    CK(cudaGetLastError());
+    CK(cudaEventRecord(c->ev1, st));
+    CK(cudaStreamSynchronize(st));
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, c->ev0, c->ev1);
+    c->info.t_solve = ms * 1e-3;
+    return MF_OK;
+}
+
+int mf_get_info(const mf_ctx *c, mf_info *out) {
+    if (!c || !out) return MF_ERR_ARG;
+    *out = c->info;
+    return MF_OK;
+}
+
+int mf_get_perm(const mf_ctx *c, int32_t *out) {
+    if (!c || !out) return MF_ERR_ARG;
+    if (c->state < 1) return MF_ERR_STATE;
+    std::memcpy(out, c->S.perm.data(), c->S.perm.size() * sizeof(int32_t));
+    return MF_OK;
+}
+
+int mf_get_etree(const mf_ctx *c, int32_t *parent, int64_t *cc) {
+    if (!c) return MF_ERR_ARG;
+    if (c->state < 1) return MF_ERR_STATE;
+    if (parent) std::memcpy(parent, c->S.parent.data(), c->S.parent.size() * sizeof(int32_t));
+    if (cc) std::memcpy(cc, c->S.cc.data(), c->S.cc.size() * sizeof(int64_t));
+    return MF_OK;
+}
+
+int mf_get_supernodes(const mf_ctx *c, int32_t *sn_first, int32_t *sn_parent, int64_t *sn_rowptr, int32_t *sn_rows,
+                      int32_t *fund_first) {
+    if (!c) return MF_ERR_ARG;
+    if (c->state < 1) return MF_ERR_STATE;
+    const Symbolic &S = c->S;
+    if (sn_first) std::memcpy(sn_first, S.sn_first.data(), S.sn_first.size() * sizeof(int32_t));
+    if (sn_parent) std::memcpy(sn_parent, S.sn_parent.data(), S.sn_parent.size() * sizeof(int32_t));
+    if (sn_rowptr) std::memcpy(sn_rowptr, S.sn_rowptr.data(), S.sn_rowptr.size() * sizeof(int64_t));
+    if (sn_rows) std::memcpy(sn_rows, S.sn_rows.data(), S.sn_rows.size() * sizeof(int32_t));
+    if (fund_first) std::memcpy(fund_first, S.fund_first.data(), S.fund_first.size() * sizeof(int32_t));
+    return MF_OK;
+}
+
+int mf_export_panel(const mf_ctx *c, int32_t s, double *out) {
+    if (!c || !out) return MF_ERR_ARG;
+    if (c->state != 2) return MF_ERR_STATE;
+    if (s < 0 || s >= c->P.nsuper) return MF_ERR_ARG;
+    CK(cudaSetDevice(c->device));
+    const int f = c->P.sn_f[s], k = c->P.sn_k[s], ld = c->P.sn_ld[s];
+    CK(cudaMemcpy2DAsync(out, f * sizeof(double), c->d.L + c->P.L_off[s], ld * sizeof(double), f * sizeof(double), k,
+                         cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    return MF_OK;
+}
+
+int mf_export_diag(const mf_ctx *c, double *out) {
+    if (!c || !out) return MF_ERR_ARG;
+    if (c->state != 2) return MF_ERR_STATE;
+    CK(cudaSetDevice(c->device));
+    const int64_t n = c->S.n;
+    launch_export_diag(c->d, c->P.nsuper, c->d_bx, c->stream);
+    CK(cudaMemcpyAsync(out, c->d_bx, n * sizeof(double), cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaStreamSynchronize(c->stream));
+    return MF_OK;
+}
+
+int mf_export_L(const mf_ctx *c, double *out) {
+    if (!c || !out) return MF_ERR_ARG;
+    if (c->state != 2) return MF_ERR_STATE;
+    int64_t o = 0;
+    for (int32_t s = 0; s < c->P.nsuper; s++) {
+        int r = mf_export_panel(c, s, out + o);
+        if (r) return r;
+        o += (int64_t)c->P.sn_f[s] * c->P.sn_k[s];
+    }
+    return MF_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,525 @@
+// kernels.cu -- sm_100a kernels of the multifrontal factor-update hot path.
+//
+// What each kernel computes follows PAPER.md L27 (Sec. II-A) and Fig. 1
+// (L33-65): per supernode, F^n = A entries (+) extend-add of the children's
+// U^c, then potrf on L1 (k x k), trsm on L2 (m x k), U^n = U^n - L2 L2^T.
+// The large-front path is the blocked variant of PAPER.md L325 / Fig. 9
+// (w x w potrf kernel, trsm on the panel below it, trailing update), with the
+// syrk on U^n done once with inner dimension k.  All arithmetic is fp64
+// (reading C7).  FP64 tensor-core work uses DMMA (mma.sync m8n8k4 f64): on
+// sm_100a tcgen05 has no f64 kind (probe 1).
+//
+// Determinism: extend-add has no atomics; every destination entry receives
+// 0, then its A value, then the children's contributions in ascending child
+// order (reading C6) -- the same summation order as the oracle.
+#include <climits>
+#include <cstdio>
+
+#include "kernels.cuh"
+
+namespace mf {
+
+// ------------------------------------------------------------------ helpers
+__device__ __forceinline__ double sum_values(const DevPlan &d, const double *__restrict__ values, int64_t e) {
+    const int64_t b = d.bvptr[e], q = d.bvptr[e + 1];
+    double v = values[d.bvidx[b]];
+    for (int64_t t = b + 1; t < q; t++) v += values[d.bvidx[t]];
+    return v;
+}
+
+__device__ __forceinline__ void note_pivot(const DevPlan &d, double djj, int col) {
+    if (!(djj > 0.0)) atomicMin(d.failed, col);   // non-positive or NaN pivot (reading C8)
+}
+
+__global__ void k_init_failed(int *failed) { *failed = INT_MAX; }
+
+// ============================================================ small fronts
+// One CTA per front; the whole f x f front lives in shared memory (column-major,
+// leading dimension f).  Assembly, potrf, trsm and the syrk on U^n are fused:
+// the k pivot columns are eliminated right-looking, which produces L1, L2 and
+// U^n = F22 - L2 L2^T in place.  Writes the L panel and U^n to HBM.
+template <int NT>
+__global__ void __launch_bounds__(NT) k_small_front(DevPlan d, const int32_t *__restrict__ list,
+                                                    const double *__restrict__ values) {
+    extern __shared__ double F[];
+    const int s = list[blockIdx.x];
+    const int k = d.sn_k[s], f = d.sn_f[s], m = f - k, first = d.sn_first[s];
+    const int tid = threadIdx.x;
+    for (int i = tid; i < f * f; i += NT) F[i] = 0.0;
+    __syncthreads();
+    // A entries of the k pivot columns: warp per column, lanes over entries
+    {
+        const int warp = tid >> 5, lane = tid & 31;
+        for (int j = warp; j < k; j += NT / 32) {
+            const int64_t e0 = d.bcolptr[first + j], e1 = d.bcolptr[first + j + 1];
+            for (int64_t e = e0 + lane; e < e1; e += 32) F[d.blrow[e] + j * f] = sum_values(d, values, e);
+        }
+    }
+    __syncthreads();
+    // extend-add of the children's U^c, ascending child order
+    for (int q = d.child_ptr[s]; q < d.child_ptr[s + 1]; q++) {
+        const int c = d.child_list[q];
+        const int mc = d.sn_f[c] - d.sn_k[c];
+        const int32_t *__restrict__ rel = d.relmap + d.relmap_ptr[c];
+        const double *__restrict__ Uc = d.U + d.U_off[c];
+        for (int idx = tid; idx < mc * mc; idx += NT) {
+            const int p = idx % mc, qq = idx / mc;
+            if (p >= qq) F[rel[p] + rel[qq] * f] += Uc[idx];
+        }
+        __syncthreads();
+    }
+    // right-looking elimination of the k pivot columns over the whole front
+    for (int j = 0; j < k; j++) {
+        const double djj = F[j + j * f];
+        const double piv = sqrt(djj);
+        for (int i = j + 1 + tid; i < f; i += NT) F[i + j * f] /= piv;
+        __syncthreads();
+        if (tid == 0) {
+            note_pivot(d, djj, first + j);
+            F[j + j * f] = piv;
+        }
+        const int nr = f - j - 1;
+        for (int idx = tid; idx < nr * nr; idx += NT) {
+            const int i = j + 1 + idx % nr, c = j + 1 + idx / nr;
+            if (i >= c) F[i + c * f] -= F[i + j * f] * F[c + j * f];
+        }
+        __syncthreads();
+    }
+    // write the L panel (upper triangle of L1 = 0) and U^n (lower triangle)
+    double *__restrict__ P = d.L + d.L_off[s];
+    const int ld = d.sn_ld[s];
+    for (int idx = tid; idx < f * k; idx += NT) {
+        const int i = idx % f, j = idx / f;
+        P[i + (int64_t)j * ld] = i >= j ? F[i + j * f] : 0.0;
+    }
+    if (m > 0) {
+        double *__restrict__ Us = d.U + d.U_off[s];
+        for (int idx = tid; idx < m * m; idx += NT) {
+            const int i = idx % m, c = idx / m;
+            if (i >= c) Us[idx] = F[(k + i) + (k + c) * f];
+        }
+    }
+}
+
+int small_front_smem_ok(int fmax) { return (size_t)fmax * fmax * sizeof(double) <= 227 * 1024; }
+
+void launch_small_fronts(const DevPlan &d, const int32_t *list, int count, int fmax, const double *values,
+                         cudaStream_t st) {
+    if (count <= 0) return;
+    const size_t smem = (size_t)fmax * fmax * sizeof(double);
+    if (fmax <= 32) {
+        k_small_front<64><<<count, 64, smem, st>>>(d, list, values);
+    } else if (fmax <= 64) {
+        k_small_front<128><<<count, 128, smem, st>>>(d, list, values);
+    } else {
+        static bool attr = false;
+        if (!attr) {
+            cudaFuncSetAttribute(k_small_front<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+            attr = true;
+        }
+        k_small_front<256><<<count, 256, smem, st>>>(d, list, values);
+    }
+}
+
+// ============================================================ large-front assembly
+// Task = (front s, first local column c0): zero columns [c0, c0+32) of the
+// front, write the A entries, then extend-add every child's U^c columns that
+// map into these columns (child order ascending, barrier between children, so
+// the summation order is fixed).  Columns < k live in the L panel, columns >= k
+// in U^s.
+constexpr int kAsmThreads = 256;
+__global__ void __launch_bounds__(kAsmThreads) k_assemble(DevPlan d, const int32_t *__restrict__ tasks,
+                                                          const double *__restrict__ values) {
+    const int s = tasks[2 * blockIdx.x], c0 = tasks[2 * blockIdx.x + 1];
+    const int k = d.sn_k[s], f = d.sn_f[s], m = f - k, ld = d.sn_ld[s], first = d.sn_first[s];
+    const int c1 = min(c0 + kAsmCols, f);
+    double *__restrict__ P = d.L + d.L_off[s];
+    double *__restrict__ Us = d.U + d.U_off[s];
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    constexpr int NW = kAsmThreads / 32;
+    for (int c = c0 + warp; c < c1; c += NW) {
+        if (c < k) {
+            for (int i = lane; i < f; i += 32) P[i + (int64_t)c * ld] = 0.0;
+        } else {
+            const int cu = c - k;
+            for (int i = cu + lane; i < m; i += 32) Us[i + (int64_t)cu * m] = 0.0;
+        }
+    }
+    __syncthreads();
+    for (int c = c0 + warp; c < min(c1, k); c += NW) {
+        const int64_t e0 = d.bcolptr[first + c], e1 = d.bcolptr[first + c + 1];
+        for (int64_t e = e0 + lane; e < e1; e += 32) P[d.blrow[e] + (int64_t)c * ld] = sum_values(d, values, e);
+    }
+    __syncthreads();
+    __shared__ int qrange[2];
+    for (int q = d.child_ptr[s]; q < d.child_ptr[s + 1]; q++) {
+        const int ch = d.child_list[q];
+        const int mc = d.sn_f[ch] - d.sn_k[ch];
+        const int32_t *__restrict__ rel = d.relmap + d.relmap_ptr[ch];
+        const double *__restrict__ Uc = d.U + d.U_off[ch];
+        if (tid < 2) {   // child columns qa..qb-1 map into [c0, c1): rel is increasing
+            const int target = tid == 0 ? c0 : c1;
+            int lo = 0, hi = mc;
+            while (lo < hi) {
+                const int mid = (lo + hi) >> 1;
+                if (rel[mid] < target) lo = mid + 1; else hi = mid;
+            }
+            qrange[tid] = lo;
+        }
+        __syncthreads();
+        const int qa = qrange[0], qb = qrange[1];
+        for (int qc = qa + warp; qc < qb; qc += NW) {
+            const int dc = rel[qc];
+            const double *__restrict__ ucol = Uc + (int64_t)qc * mc;
+            if (dc < k) {
+                double *__restrict__ pcol = P + (int64_t)dc * ld;
+                for (int p = qc + lane; p < mc; p += 32) pcol[rel[p]] += ucol[p];
+            } else {
+                double *__restrict__ ucol_dst = Us + (int64_t)(dc - k) * m - k;
+                for (int p = qc + lane; p < mc; p += 32) ucol_dst[rel[p]] += ucol[p];
+            }
+        }
+        __syncthreads();
+    }
+}
+
+void launch_assemble(const DevPlan &d, const int32_t *tasks, int64_t count, const double *values, cudaStream_t st) {
+    if (count <= 0) return;
+    k_assemble<<<(unsigned)count, kAsmThreads, 0, st>>>(d, tasks, values);
+}
+
+// ============================================================ diagonal-block potrf
+// The "light-weight GPU kernel ... performing potrf on a w x w matrix" of
+// one CTA per active front factors its diagonal block
+// [j0, j0+we) x [j0, j0+we) in shared memory (right-looking, unblocked).
+constexpr int kWmax = 64;
+constexpr int kPotrfThreads = 256;
+__global__ void __launch_bounds__(kPotrfThreads) k_potrf_diag(DevPlan d, const int32_t *__restrict__ fronts,
+                                                              int j0, int w) {
+    __shared__ double A[kWmax * (kWmax + 1)];
+    constexpr int LDA = kWmax + 1;
+    const int s = fronts[blockIdx.x];
+    const int k = d.sn_k[s], ld = d.sn_ld[s], first = d.sn_first[s];
+    const int we = min(w, k - j0);
+    double *__restrict__ P = d.L + d.L_off[s] + (int64_t)j0 * ld + j0;
+    const int tid = threadIdx.x;
+    for (int idx = tid; idx < we * we; idx += kPotrfThreads) {
+        const int i = idx % we, c = idx / we;
+        A[i + c * LDA] = P[i + (int64_t)c * ld];
+    }
+    __syncthreads();
+    for (int j = 0; j < we; j++) {
+        const double djj = A[j + j * LDA];
+        const double piv = sqrt(djj);
+        for (int i = j + 1 + tid; i < we; i += kPotrfThreads) A[i + j * LDA] /= piv;
+        __syncthreads();
+        if (tid == 0) {
+            note_pivot(d, djj, first + j0 + j);
+            A[j + j * LDA] = piv;
+        }
+        const int nr = we - j - 1;
+        for (int idx = tid; idx < nr * nr; idx += kPotrfThreads) {
+            const int i = j + 1 + idx % nr, c = j + 1 + idx / nr;
+            if (i >= c) A[i + c * LDA] -= A[i + j * LDA] * A[c + j * LDA];
+        }
+        __syncthreads();
+    }
+    for (int idx = tid; idx < we * we; idx += kPotrfThreads) {
+        const int i = idx % we, c = idx / we;
+        if (i >= c) P[i + (int64_t)c * ld] = A[i + c * LDA];
+    }
+}
+
+void launch_potrf_diag(const DevPlan &d, const int32_t *fronts, int count, int j0, int w, cudaStream_t st) {
+    if (count <= 0) return;
+    k_potrf_diag<<<count, kPotrfThreads, 0, st>>>(d, fronts, j0, w);
+}
+
+// ============================================================ panel trsm
+// X L11^T = B for the rows [r0, r0+64) below the diagonal block (these rows
+// span the rest of L1 and all of L2: "we perform trsm on a (m + k - w) x w
+// matrix which spans both L1 and L2").  Substitution order
+// (ascending columns), no explicit inverse: integer-exact on manufactured inputs.
+constexpr int kTrsmThreads = 256;
+__global__ void __launch_bounds__(kTrsmThreads) k_trsm_panel(DevPlan d, const int32_t *__restrict__ tasks,
+                                                             int j0, int w) {
+    extern __shared__ double trsm_sm[];
+    double *Ls = trsm_sm;                          // w x w diagonal block
+    double *X = trsm_sm + kWmax * (kWmax + 1);     // 64 rows x w
+    constexpr int LDL = kWmax + 1, LDX = kTrsmRows + 1;
+    const int s = tasks[2 * blockIdx.x], r0 = tasks[2 * blockIdx.x + 1];
+    const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s];
+    const int we = min(w, k - j0);
+    const int nr = min(kTrsmRows, f - r0);
+    const double *__restrict__ D = d.L + d.L_off[s] + (int64_t)j0 * ld + j0;
+    double *__restrict__ B = d.L + d.L_off[s] + (int64_t)j0 * ld + r0;
+    const int tid = threadIdx.x;
+    for (int idx = tid; idx < we * we; idx += kTrsmThreads) {
+        const int i = idx % we, c = idx / we;
+        Ls[i + c * LDL] = D[i + (int64_t)c * ld];
+    }
+    for (int idx = tid; idx < kTrsmRows * we; idx += kTrsmThreads) {
+        const int i = idx % kTrsmRows, c = idx / kTrsmRows;
+        X[i + c * LDX] = i < nr ? B[i + (int64_t)c * ld] : 0.0;
+    }
+    __syncthreads();
+    const int r = tid % kTrsmRows, g = tid / kTrsmRows;
+    constexpr int NG = kTrsmThreads / kTrsmRows;
+    for (int c = 0; c < we; c++) {
+        if (g == 0) X[r + c * LDX] /= Ls[c + c * LDL];
+        __syncthreads();
+        const double xc = X[r + c * LDX];
+        for (int cc = c + 1 + g; cc < we; cc += NG) X[r + cc * LDX] -= xc * Ls[cc + c * LDL];
+        __syncthreads();
+    }
+    for (int idx = tid; idx < kTrsmRows * we; idx += kTrsmThreads) {
+        const int i = idx % kTrsmRows, c = idx / kTrsmRows;
+        if (i < nr) B[i + (int64_t)c * ld] = X[i + c * LDX];
+    }
+}
+
+void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, cudaStream_t st) {
+    if (count <= 0) return;
+    constexpr size_t smem = (size_t)(kWmax * (kWmax + 1) + (kTrsmRows + 1) * kWmax) * sizeof(double);
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(k_trsm_panel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        attr = true;
+    }
+    k_trsm_panel<<<(unsigned)count, kTrsmThreads, smem, st>>>(d, tasks, j0, w);
+}
+
+// ============================================================ DMMA Schur update
+// C[i][j] -= sum_p A[i][p] A[j][p]  for a 128 x 64 output tile, lower-trapezoid
+// mask (i >= j, i < M, j < N).  FP64 tensor cores via mma.sync.m8n8k4.f64
+// (SASS DMMA.8x8x4), operands staged by 16-byte cp.async (LDGSTS) in a
+// 3-stage ring, 8 warps each owning a 32 x 32 sub-tile (32 fp64 accumulators
+// per thread), two CTAs per SM.
+namespace gemm {
+constexpr int BM = kTileM, BN = kTileN, BK = 16, STAGES = 3, NT = 256;
+constexpr int SA = BM + 4;   // 130 rows needed (odd-row alignment shift) + pad: 132 % 16 == 4 (conflict-free)
+constexpr int SB = BN + 4;   // 66 rows needed + pad: 68 % 16 == 4
+constexpr int CHA = (BM + 2) / 2, CHB = (BN + 2) / 2;   // 16-byte chunks per column (65, 33)
+constexpr int STAGE_WORDS = BK * (SA + SB);
+constexpr size_t SMEM = (size_t)STAGES * STAGE_WORDS * sizeof(double);
+}  // namespace gemm
+
+__device__ __forceinline__ void cp_async16(void *smem, const void *gmem, bool valid) {
+    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    const int n = valid ? 16 : 0;
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(s), "l"(gmem), "r"(n));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
+
+__device__ __forceinline__ void dmma(double &c0, double &c1, double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+                 : "+d"(c0), "+d"(c1)
+                 : "d"(a), "d"(b));
+}
+
+__global__ void __launch_bounds__(gemm::NT, 2) k_update(double *__restrict__ Larena, double *__restrict__ Uarena,
+                                                        const GemmProb *__restrict__ probs,
+                                                        const TileTask *__restrict__ tiles) {
+    using namespace gemm;
+    extern __shared__ __align__(16) double sm[];
+    const TileTask t = tiles[blockIdx.x];
+    const GemmProb g = probs[t.prob];
+    const int ti = t.tij >> 16, tj = t.tij & 0xffff;
+    const int i0 = ti * BM, j0 = tj * BN;
+    const int sh = (int)(g.a_off & 1);   // columns are 16B aligned (even lda); shift odd row starts
+    const double *__restrict__ A = Larena + g.a_off - sh;   // aligned base of row -sh
+    const int lda = g.lda, K = g.K;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int wm = warp & 3, wn = warp >> 2;   // 4 x 2 warps of 32 x 32
+    const int gq = lane >> 2, tq = lane & 3;
+
+    auto load_stage = [&](int stage, int kt) {
+        double *As = sm + stage * STAGE_WORDS;
+        double *Bs = As + BK * SA;
+        const int p0 = kt * BK;
+        for (int c = tid; c < BK * (CHA + CHB); c += NT) {
+            if (c < BK * CHA) {
+                const int p = c / CHA, ch = c - p * CHA;
+                const int row = i0 + 2 * ch;          // aligned row index (relative to -sh)
+                const bool ok = (p0 + p < K) && (row - sh < g.M);
+                cp_async16(As + p * SA + 2 * ch, ok ? A + row + (int64_t)(p0 + p) * lda : A, ok);
+            } else {
+                const int cc = c - BK * CHA;
+                const int p = cc / CHB, ch = cc - p * CHB;
+                const int row = j0 + 2 * ch;
+                const bool ok = (p0 + p < K) && (row - sh < g.N);
+                cp_async16(Bs + p * SB + 2 * ch, ok ? A + row + (int64_t)(p0 + p) * lda : A, ok);
+            }
+        }
+    };
+
+    double acc[4][4][2];
+#pragma unroll
+    for (int a = 0; a < 4; a++)
+#pragma unroll
+        for (int b = 0; b < 4; b++) acc[a][b][0] = acc[a][b][1] = 0.0;
+
+    const int KT = (K + BK - 1) / BK;
+#pragma unroll
+    for (int st = 0; st < STAGES - 1; st++) {
+        if (st < KT) load_stage(st, st);
+        cp_async_commit();
+    }
+    for (int kt = 0; kt < KT; kt++) {
+        cp_async_wait<STAGES - 2>();
+        __syncthreads();
+        {
+            const int nk = kt + STAGES - 1;
+            if (nk < KT) load_stage(nk % STAGES, nk);
+            cp_async_commit();
+        }
+        const double *As = sm + (kt % STAGES) * STAGE_WORDS + sh + wm * 32 + gq;
+        const double *Bs = sm + (kt % STAGES) * STAGE_WORDS + BK * SA + sh + wn * 32 + gq;
+#pragma unroll
+        for (int kk = 0; kk < BK / 4; kk++) {
+            double a[4], b[4];
+#pragma unroll
+            for (int mb = 0; mb < 4; mb++) a[mb] = As[(kk * 4 + tq) * SA + mb * 8];
+#pragma unroll
+            for (int nb = 0; nb < 4; nb++) b[nb] = Bs[(kk * 4 + tq) * SB + nb * 8];
+#pragma unroll
+            for (int mb = 0; mb < 4; mb++)
+#pragma unroll
+                for (int nb = 0; nb < 4; nb++) dmma(acc[mb][nb][0], acc[mb][nb][1], a[mb], b[nb]);
+        }
+    }
+    cp_async_wait<0>();
+    // epilogue: C -= acc on the lower-trapezoid mask
+    double *__restrict__ C = (g.c_in_U ? Uarena : Larena) + g.c_off;
+    const int ldc = g.ldc;
+#pragma unroll
+    for (int mb = 0; mb < 4; mb++) {
+        const int i = i0 + wm * 32 + mb * 8 + gq;
+        if (i >= g.M) continue;
+#pragma unroll
+        for (int nb = 0; nb < 4; nb++) {
+#pragma unroll
+            for (int e = 0; e < 2; e++) {
+                const int j = j0 + wn * 32 + nb * 8 + 2 * tq + e;
+                if (j < g.N && i >= j) C[i + (int64_t)j * ldc] -= acc[mb][nb][e];
+            }
+        }
+    }
+}
+
+void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, cudaStream_t st) {
+    if (ntiles <= 0) return;
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(k_update, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)gemm::SMEM);
+        attr = true;
+    }
+    k_update<<<(unsigned)ntiles, gemm::NT, gemm::SMEM, st>>>(d.L, d.U, probs, tiles);
+}
+
+void launch_init_failed(int *failed, cudaStream_t st) { k_init_failed<<<1, 1, 0, st>>>(failed); }
+
+// diag(L) in final labels (one warp per supernode)
+__global__ void k_export_diag(DevPlan d, int nsuper, double *__restrict__ out) {
+    const int s = blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);
+    if (s >= nsuper) return;
+    const int k = d.sn_k[s], ld = d.sn_ld[s], first = d.sn_first[s];
+    const double *__restrict__ P = d.L + d.L_off[s];
+    for (int j = threadIdx.x & 31; j < k; j += 32) out[first + j] = P[j + (int64_t)j * ld];
+}
+void launch_export_diag(const DevPlan &d, int nsuper, double *out, cudaStream_t st) {
+    if (nsuper > 0) k_export_diag<<<(nsuper + 7) / 8, 256, 0, st>>>(d, nsuper, out);
+}
+
+// ============================================================ triangular solves
+// "a forward triangular solve Ly = b and a backward triangular
+// solve L^T x = y".  Supernodal, level by level; the forward sweep carries
+// per-front update vectors that the parent gathers through the same relative
+// maps as the extend-add (deterministic, no atomics).
+__global__ void k_permute_in(const int32_t *__restrict__ perm, const double *__restrict__ b, double *__restrict__ y,
+                             int64_t n) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        y[i] = b[perm[i]];
+}
+__global__ void k_permute_out(const int32_t *__restrict__ perm, const double *__restrict__ xf, double *__restrict__ x,
+                              int64_t n) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        x[perm[i]] = xf[i];
+}
+void launch_permute_in(const DevPlan &d, const double *b, double *y, int64_t n, cudaStream_t st) {
+    if (n > 0) k_permute_in<<<(unsigned)((n + 255) / 256 < 4096 ? (n + 255) / 256 : 4096), 256, 0, st>>>(d.perm, b, y, n);
+}
+void launch_permute_out(const DevPlan &d, const double *xf, double *x, int64_t n, cudaStream_t st) {
+    if (n > 0) k_permute_out<<<(unsigned)((n + 255) / 256 < 4096 ? (n + 255) / 256 : 4096), 256, 0, st>>>(d.perm, xf, x, n);
+}
+
+constexpr int kSolveThreads = 256;
+__global__ void __launch_bounds__(kSolveThreads) k_fwd_solve(DevPlan d, const int32_t *__restrict__ list,
+                                                             double *__restrict__ y) {
+    const int s = list[blockIdx.x];
+    const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
+    double *__restrict__ v = d.fv + d.fv_off[s];
+    const double *__restrict__ P = d.L + d.L_off[s];
+    const int tid = threadIdx.x;
+    for (int i = tid; i < f; i += kSolveThreads) v[i] = i < k ? y[first + i] : 0.0;
+    __syncthreads();
+    for (int q = d.child_ptr[s]; q < d.child_ptr[s + 1]; q++) {
+        const int c = d.child_list[q];
+        const int kc = d.sn_k[c], mc = d.sn_f[c] - kc;
+        const int32_t *__restrict__ rel = d.relmap + d.relmap_ptr[c];
+        const double *__restrict__ vc = d.fv + d.fv_off[c] + kc;
+        for (int p = tid; p < mc; p += kSolveThreads) v[rel[p]] += vc[p];
+        __syncthreads();
+    }
+    for (int j = 0; j < k; j++) {
+        const double xj = v[j] / P[j + (int64_t)j * ld];
+        if (tid == 0) y[first + j] = xj;
+        const double *__restrict__ col = P + (int64_t)j * ld;
+        for (int i = j + 1 + tid; i < f; i += kSolveThreads) v[i] -= col[i] * xj;
+        __syncthreads();
+    }
+}
+
+__global__ void __launch_bounds__(kSolveThreads) k_bwd_solve(DevPlan d, const int32_t *__restrict__ list,
+                                                             double *__restrict__ y,
+                                                             const int32_t *__restrict__ sn_rows,
+                                                             const int64_t *__restrict__ sn_rowptr) {
+    const int s = list[blockIdx.x];
+    const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
+    double *__restrict__ v = d.fv + d.fv_off[s];
+    const double *__restrict__ P = d.L + d.L_off[s];
+    const int32_t *__restrict__ R = sn_rows + sn_rowptr[s];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    __shared__ double red[kSolveThreads / 32];
+    for (int i = k + tid; i < f; i += kSolveThreads) v[i] = y[R[i]];   // ancestors are final
+    __syncthreads();
+    for (int j = k - 1; j >= 0; j--) {
+        const double *__restrict__ col = P + (int64_t)j * ld;
+        double part = 0.0;
+        for (int i = j + 1 + tid; i < f; i += kSolveThreads) part += col[i] * v[i];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
+        if (lane == 0) red[warp] = part;
+        __syncthreads();
+        if (tid == 0) {
+            double tot = 0.0;
+            for (int w = 0; w < kSolveThreads / 32; w++) tot += red[w];
+            const double xj = (y[first + j] - tot) / col[j];
+            v[j] = xj;
+            y[first + j] = xj;
+        }
+        __syncthreads();
+    }
+}
+
+void launch_fwd_solve(const DevPlan &d, const int32_t *list, int count, double *y, cudaStream_t st) {
+    if (count > 0) k_fwd_solve<<<count, kSolveThreads, 0, st>>>(d, list, y);
+}
+void launch_bwd_solve(const DevPlan &d, const int32_t *list, int count, double *y, const int32_t *sn_rows,
+                      const int64_t *sn_rowptr, cudaStream_t st) {
+    if (count > 0) k_bwd_solve<<<count, kSolveThreads, 0, st>>>(d, list, y, sn_rows, sn_rowptr);
+}
+
+}  // namespace mf

@@ -1,0 +1,44 @@
+// kernels.cuh -- device-side plan view and kernel launchers (internal to libmf).
+#pragma once
+#include <cuda_runtime.h>
+#include <cstdint>
+
+#include "mf_plan.h"
+
+namespace mf {
+
+// Flat device arrays of the plan (uploaded once by mf_analyze).
+struct DevPlan {
+    double *L;            // L arena (panels)
+    double *U;            // U arena (update matrices)
+    double *fv;           // solve: one front vector per supernode
+    const int32_t *sn_first, *sn_k, *sn_f, *sn_ld;
+    const int64_t *L_off, *U_off, *fv_off;
+    const int32_t *child_ptr, *child_list;
+    const int64_t *relmap_ptr;
+    const int32_t *relmap;
+    const int64_t *bcolptr;  // B entries per column (final labels)
+    const int32_t *blrow;    // local row of each B entry in its front
+    const int64_t *bvptr;    // value-index list per B entry
+    const int64_t *bvidx;
+    const int32_t *perm;     // final perm (new -> old)
+    int *failed;             // min failing pivot column (final labels); INT_MAX = none
+};
+
+// launchers (all asynchronous on `st`)
+void launch_init_failed(int *failed, cudaStream_t st);
+void launch_small_fronts(const DevPlan &d, const int32_t *list, int count, int fmax, const double *values,
+                         cudaStream_t st);
+void launch_assemble(const DevPlan &d, const int32_t *tasks, int64_t count, const double *values, cudaStream_t st);
+void launch_potrf_diag(const DevPlan &d, const int32_t *fronts, int count, int j0, int w, cudaStream_t st);
+void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, cudaStream_t st);
+void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, cudaStream_t st);
+void launch_permute_in(const DevPlan &d, const double *b, double *y, int64_t n, cudaStream_t st);
+void launch_permute_out(const DevPlan &d, const double *xf, double *x, int64_t n, cudaStream_t st);
+void launch_fwd_solve(const DevPlan &d, const int32_t *list, int count, double *y, cudaStream_t st);
+void launch_bwd_solve(const DevPlan &d, const int32_t *list, int count, double *y, const int32_t *sn_rows,
+                      const int64_t *sn_rowptr, cudaStream_t st);
+int small_front_smem_ok(int fmax);
+void launch_export_diag(const DevPlan &d, int nsuper, double *out, cudaStream_t st);
+
+}  // namespace mf

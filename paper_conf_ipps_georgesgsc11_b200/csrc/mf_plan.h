@@ -1,0 +1,113 @@
+// mf_plan.h -- host-side symbolic analysis + device plan of the multifrontal
+// factor-update hot path (internal to libmf; the public ABI is include/mf.h).
+//
+// The symbolic layer feeds PAPER.md L27 (Sec. II-A): supernodal elimination
+// tree in postorder, front row lists R_s (front order f = k + m, reading C1),
+// child -> parent extend-add index maps, A-entry -> front maps.  Algorithms
+// (Liu's etree with path compression, row-subtree column counts, supernodal
+// row-list merge) are deliberately different from the oracle's definitions
+// (oracle/symbolic.c) so that bit-exact agreement is a real check.
+#pragma once
+#include <cstdint>
+#include <vector>
+
+namespace mf {
+
+struct Options {
+    int amalgamate = 1;
+    int nrelax[3] = {4, 16, 48};
+    double zrelax[3] = {0.8, 0.1, 0.05};
+    int small_front_max = 128;
+    int panel_w = 64;
+};
+
+// ---------------------------------------------------------------- symbolic
+struct Symbolic {
+    int64_t n = 0;
+    int64_t nnzA_read = 0;
+    int64_t nnz_in = 0;              // colptr[n]: length of the caller's values array
+    std::vector<int32_t> perm;       // final perm (new -> old)
+    std::vector<int32_t> parent;     // elimination tree
+    std::vector<int64_t> cc;         // column counts
+    int64_t nnzL = 0, flops = 0, stored_L = 0, exec_flops = 0;
+    std::vector<int32_t> fund_first;
+    std::vector<int32_t> sn_first, sn_parent;
+    std::vector<int64_t> sn_rowptr;
+    std::vector<int32_t> sn_rows;
+    // unique entries of B = P A P^T (lower incl. diagonal), sorted (col, row);
+    // value of entry e = sum of values[bvidx[bvptr[e] .. bvptr[e+1])] in input order
+    std::vector<int64_t> bcolptr;    // n+1
+    std::vector<int32_t> brow;
+    std::vector<int64_t> bvptr;
+    std::vector<int64_t> bvidx;
+};
+
+// returns 0 or a negative MF_ERR_* code
+int analyze_symbolic(int64_t n, const int64_t *colptr, const int32_t *rowind, const int32_t *perm,
+                     const Options &opt, Symbolic &S);
+
+// ---------------------------------------------------------------- device plan
+// A (lower-trapezoidal) Schur update problem:  C[i][j] -= sum_p A[i][p] * A[j][p]
+// for 0 <= j < N, j <= i < M (only entries with i >= j are written).
+// A: M x K, column-major, leading dim lda, inside the L arena.
+// C: column-major, leading dim ldc, inside the L arena (c_in_U = 0) or the U arena (1).
+struct GemmProb {
+    int64_t a_off;
+    int64_t c_off;
+    int32_t lda, ldc;
+    int32_t M, N, K;
+    int32_t c_in_U;
+};
+static_assert(sizeof(GemmProb) == 40, "GemmProb layout");
+
+struct TileTask {       // one kTileM x kTileN output tile of a GemmProb
+    int32_t prob;
+    int32_t tij;        // (ti << 16) | tj
+};
+
+struct LevelPlan {
+    // small fronts: batched fused kernel, grouped in size classes
+    std::vector<int32_t> small_class_off;   // per class, offset into small_list (nclass+1)
+    // large fronts (sorted by k descending)
+    int64_t large_off = 0, nlarge = 0;       // into large_list
+    int64_t asm_off = 0, nasm = 0;           // assembly tasks (int2: front, c0)
+    struct Wave {
+        int32_t j0;
+        int32_t nactive;                     // prefix of the level's large list
+        int64_t trsm_off, ntrsm;             // (front, row-block) tasks
+        int64_t prob_off, nprob;             // update problems
+        int64_t tile_off, ntile;             // update tiles
+    };
+    std::vector<Wave> waves;
+    int64_t syrk_prob_off = 0, syrk_nprob = 0, syrk_tile_off = 0, syrk_ntile = 0;
+};
+
+struct Plan {
+    int32_t nsuper = 0, nlevels = 0, w = 64, small_max = 128, max_front = 0;
+    int64_t L_words = 0, U_words = 0, rows_total = 0, relmap_total = 0, fv_words = 0;
+    // per supernode (host copies; device mirrors in the ctx)
+    std::vector<int32_t> sn_k, sn_f, sn_ld, sn_level;
+    std::vector<int64_t> L_off, U_off, fv_off;
+    std::vector<int32_t> child_ptr, child_list;      // children ascending
+    std::vector<int64_t> relmap_ptr;                 // per supernode (as a child)
+    std::vector<int32_t> relmap;                     // positions of R_c[k_c:] in R_parent
+    std::vector<int32_t> blrow;                      // local row in the front of each B entry
+    // schedule
+    std::vector<int32_t> level_ptr, level_list;      // all supernodes by level (solve)
+    std::vector<int32_t> small_list, small_class_fmax;
+    std::vector<int32_t> large_list;
+    std::vector<int32_t> asm_tasks;                  // pairs (front, c0)
+    std::vector<int32_t> trsm_tasks;                 // pairs (front, row0)
+    std::vector<GemmProb> probs;
+    std::vector<TileTask> tiles;
+    std::vector<LevelPlan> levels;
+};
+
+constexpr int kTileM = 128, kTileN = 64;
+constexpr int kAsmCols = 32;
+constexpr int kTrsmRows = 64;
+constexpr int kSmallClasses = 3;
+
+int build_plan(const Symbolic &S, const Options &opt, Plan &P);
+
+}  // namespace mf

@@ -1,0 +1,220 @@
+"""ctypes binding of include/mf.h -- argument marshalling only.
+
+Every step of the hot path runs inside libmf.so (CUDA kernels for sm_100a);
+this module converts numpy arrays / torch tensors to raw pointers and return
+codes to exceptions.  It never computes anything itself and has no fallback.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+from ._build import LIB as _LIB_PATH
+
+MF_OK = 0
+MF_NOT_SPD = 1
+MF_ERR_ARG = -1
+MF_ERR_STATE = -2
+MF_ERR_NOMEM = -3
+MF_ERR_CUDA = -4
+MF_ERR_NCCL = -5
+
+# every symbol include/mf.h declares (checked by tests/test_abi.py)
+EXPORTED_SYMBOLS = (
+    "mf_default_options", "mf_create", "mf_analyze", "mf_factor", "mf_solve", "mf_get_info",
+    "mf_get_perm", "mf_get_etree", "mf_get_supernodes", "mf_export_panel", "mf_export_diag", "mf_export_L",
+    "mf_destroy", "mf_strerror",
+)
+
+
+class Options(ctypes.Structure):
+    _fields_ = [
+        ("amalgamate", ctypes.c_int32), ("nrelax", ctypes.c_int32 * 3), ("zrelax", ctypes.c_double * 3),
+        ("small_front_max", ctypes.c_int32), ("panel_w", ctypes.c_int32), ("device", ctypes.c_int32),
+        ("host_only", ctypes.c_int32), ("stream", ctypes.c_void_p),
+    ]
+
+
+class Info(ctypes.Structure):
+    _fields_ = [
+        ("n", ctypes.c_int64), ("nnzA", ctypes.c_int64), ("nnzL", ctypes.c_int64),
+        ("nnzL_stored", ctypes.c_int64), ("panel_words", ctypes.c_int64), ("flops_true", ctypes.c_int64),
+        ("flops_exec", ctypes.c_int64), ("nfund", ctypes.c_int32), ("nsuper", ctypes.c_int32),
+        ("nlevels", ctypes.c_int32), ("max_front", ctypes.c_int32), ("rows_total", ctypes.c_int64),
+        ("failed_col", ctypes.c_int64), ("workspace_bytes", ctypes.c_int64), ("launches_factor", ctypes.c_int64),
+        ("t_analyze", ctypes.c_double), ("t_factor", ctypes.c_double), ("t_solve", ctypes.c_double),
+    ]
+
+    def as_dict(self) -> dict:
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+def lib_path() -> str:
+    return _LIB_PATH
+
+
+def _load():
+    if not os.path.exists(_LIB_PATH):
+        raise ImportError(f"libmf.so not built at {_LIB_PATH}: run `python -c 'import __graft_entry__ as g; g.build()'`"
+                          " (there is no CPU fallback)")
+    L = ctypes.CDLL(_LIB_PATH)
+    vp, i32, i64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64
+    sig = {
+        "mf_default_options": ([ctypes.POINTER(Options)], ctypes.c_int),
+        "mf_create": ([ctypes.POINTER(vp), ctypes.POINTER(Options)], ctypes.c_int),
+        "mf_analyze": ([vp, i64, vp, vp, vp], ctypes.c_int),
+        "mf_factor": ([vp, vp], ctypes.c_int),
+        "mf_solve": ([vp, vp, vp], ctypes.c_int),
+        "mf_get_info": ([vp, ctypes.POINTER(Info)], ctypes.c_int),
+        "mf_get_perm": ([vp, vp], ctypes.c_int),
+        "mf_get_etree": ([vp, vp, vp], ctypes.c_int),
+        "mf_get_supernodes": ([vp, vp, vp, vp, vp, vp], ctypes.c_int),
+        "mf_export_panel": ([vp, i32, vp], ctypes.c_int),
+        "mf_export_diag": ([vp, vp], ctypes.c_int),
+        "mf_export_L": ([vp, vp], ctypes.c_int),
+        "mf_destroy": ([vp], None),
+        "mf_strerror": ([ctypes.c_int], ctypes.c_char_p),
+    }
+    for name, (args, res) in sig.items():
+        fn = getattr(L, name)
+        fn.argtypes = args
+        fn.restype = res
+    return L
+
+
+lib = _load()
+
+
+class MfError(RuntimeError):
+    def __init__(self, code: int, where: str):
+        super().__init__(f"{where}: {lib.mf_strerror(code).decode()} ({code})")
+        self.code = code
+
+
+class MfNotSPD(MfError):
+    def __init__(self, code: int, where: str, failed_col: int):
+        super().__init__(code, where)
+        self.failed_col = failed_col
+
+
+def _ptr(x, dtype) -> int:
+    """Raw pointer of a contiguous numpy array or torch tensor of ``dtype``."""
+    if isinstance(x, np.ndarray):
+        if x.dtype != dtype or not x.flags.c_contiguous:
+            raise TypeError(f"expected contiguous {np.dtype(dtype)} array")
+        return x.ctypes.data
+    if hasattr(x, "data_ptr"):   # torch.Tensor (host or CUDA)
+        import torch
+        tdt = {np.float64: torch.float64, np.int32: torch.int32, np.int64: torch.int64}[np.dtype(dtype).type]
+        if x.dtype != tdt or not x.is_contiguous():
+            raise TypeError(f"expected contiguous {tdt} tensor")
+        return x.data_ptr()
+    raise TypeError(f"unsupported argument type {type(x)}")
+
+
+class Solver:
+    """mf_create / mf_analyze / mf_factor / mf_solve on one context."""
+
+    def __init__(self, amalgamate: bool = True, small_front_max: int | None = None, panel_w: int | None = None,
+                 device: int = -1, stream: int | None = None, host_only: bool = False):
+        o = Options()
+        lib.mf_default_options(ctypes.byref(o))
+        o.amalgamate = int(amalgamate)
+        if small_front_max is not None:
+            o.small_front_max = small_front_max
+        if panel_w is not None:
+            o.panel_w = panel_w
+        o.device = device
+        o.host_only = int(host_only)
+        o.stream = stream
+        h = ctypes.c_void_p()
+        r = lib.mf_create(ctypes.byref(h), ctypes.byref(o))
+        if r != MF_OK:
+            raise MfError(r, "mf_create")
+        self._h = h
+        self.n = None
+
+    def close(self):
+        if getattr(self, "_h", None):
+            lib.mf_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        self.close()
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def _check(self, r, where):
+        if r == MF_NOT_SPD:
+            raise MfNotSPD(r, where, self.info()["failed_col"])
+        if r != MF_OK:
+            raise MfError(r, where)
+
+    def analyze(self, n: int, colptr, rowind, perm):
+        colptr = np.ascontiguousarray(colptr, dtype=np.int64)
+        rowind = np.ascontiguousarray(rowind, dtype=np.int32)
+        perm = np.ascontiguousarray(perm, dtype=np.int32)
+        self._check(lib.mf_analyze(self._h, int(n), colptr.ctypes.data, rowind.ctypes.data, perm.ctypes.data),
+                    "mf_analyze")
+        self.n = int(n)
+        self._info = self.info()
+
+    def factor(self, values):
+        """values: float64 numpy array (host) or torch tensor (host or CUDA)."""
+        self._check(lib.mf_factor(self._h, _ptr(values, np.float64)), "mf_factor")
+
+    def solve(self, b, x=None):
+        if x is None:
+            x = np.empty(self.n, dtype=np.float64)
+        self._check(lib.mf_solve(self._h, _ptr(b, np.float64), _ptr(x, np.float64)), "mf_solve")
+        return x
+
+    def info(self) -> dict:
+        i = Info()
+        self._check(lib.mf_get_info(self._h, ctypes.byref(i)), "mf_get_info")
+        return i.as_dict()
+
+    def perm(self) -> np.ndarray:
+        p = np.empty(self.n, dtype=np.int32)
+        self._check(lib.mf_get_perm(self._h, p.ctypes.data), "mf_get_perm")
+        return p
+
+    def etree(self):
+        par = np.empty(self.n, dtype=np.int32)
+        cc = np.empty(self.n, dtype=np.int64)
+        self._check(lib.mf_get_etree(self._h, par.ctypes.data, cc.ctypes.data), "mf_get_etree")
+        return par, cc
+
+    def supernodes(self) -> dict:
+        inf = self.info()
+        ns, nf = inf["nsuper"], inf["nfund"]
+        first = np.empty(ns + 1, dtype=np.int32)
+        par = np.empty(ns, dtype=np.int32)
+        rp = np.empty(ns + 1, dtype=np.int64)
+        rows = np.empty(inf["rows_total"], dtype=np.int32)
+        fund = np.empty(nf + 1, dtype=np.int32)
+        self._check(lib.mf_get_supernodes(self._h, first.ctypes.data, par.ctypes.data, rp.ctypes.data,
+                                          rows.ctypes.data, fund.ctypes.data), "mf_get_supernodes")
+        return dict(sn_first=first, sn_parent=par, sn_rowptr=rp, sn_rows=rows, fund_first=fund)
+
+    def panel(self, s: int, f: int, k: int) -> np.ndarray:
+        """Panel of supernode s as an f x k array (column-major copy transposed to numpy order)."""
+        out = np.empty(f * k, dtype=np.float64)
+        self._check(lib.mf_export_panel(self._h, int(s), out.ctypes.data), "mf_export_panel")
+        return out.reshape(k, f).T
+
+    def diag(self) -> np.ndarray:
+        out = np.empty(self.n, dtype=np.float64)
+        self._check(lib.mf_export_diag(self._h, out.ctypes.data), "mf_export_diag")
+        return out
+
+    def export_L(self, total_words: int) -> np.ndarray:
+        out = np.empty(total_words, dtype=np.float64)
+        self._check(lib.mf_export_L(self._h, out.ctypes.data), "mf_export_L")
+        return out
