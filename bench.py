@@ -1,0 +1,342 @@
+#!/usr/bin/env python
+"""bench.py -- fp64 multifrontal sparse Cholesky factorization throughput on B200.
+
+Metric (BASELINE.json): "fp64 factorization GFLOP/s and seconds at 1/2/4/8 B200
+(% of FP64 TC peak)".  A step = one mf_factor (the whole hot path: every front's
+assembly/extend-add, potrf, trsm and Schur update) of the N=1 workload, the
+north-star target "3D 27-point stencil 100^3 (n=1M), nested dissection"
+(BASELINE.json configs[4], `--config c5`, the default).  GFLOP/s counts the
+algorithmic flops of the TRUE factor, sum_j cc_j^2.
+
+    python bench.py [--gpus N --steps K --warmup W] [--config c5] [--impl reference]
+
+Multi-GPU (torchrun, one rank per GPU): round 1 runs N independent replicas
+(each rank factors its own copy; weak scaling, no data-path collective) --
+DESIGN.md "Multi-GPU" explains why and what comes next.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from workloads import grids as G  # noqa: E402
+
+PEAK_NOMINAL_FP64 = 37.2e12   # 148 SM x 64 FP64 FMA/clk x 2 x 1.965 GHz
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c5", choices=sorted(G.CONFIGS))
+    ap.add_argument("--impl", default="mf", choices=["mf", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-sample-gflop", type=float, default=170.0,
+                    help="true GFLOP of the oracle sample (one whole subtree)")
+    ap.add_argument("--small-front-max", type=int, default=None)
+    ap.add_argument("--panel-w", type=int, default=None)
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    """nvidia-smi sampling DURING the timed region (B200_PROFILING.md clocks line)."""
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.proc = None
+        self.lines: list[str] = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self) -> dict:
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.15)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sm, smax, reasons, power = [], [], set(), []
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [x.strip() for x in ln.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                smax.append(float(parts[2]))
+                power.append(float(parts[3]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm), "power_w_max": max(power) if power else None}
+
+
+# ------------------------------------------------------------------ helpers
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def measured_dgemm_peak(torch) -> float:
+    """cuBLAS DGEMM 8192^3 burst on this GPU (the fp64 roofline denominator;
+    MEASURED_PEAKS.json has no fp64 figure)."""
+    n = 8192
+    a = torch.randn(n, n, dtype=torch.float64, device="cuda")
+    b = torch.randn(n, n, dtype=torch.float64, device="cuda")
+    for _ in range(2):
+        a @ b
+    torch.cuda.synchronize()
+    best = 1e9
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    for _ in range(5):
+        e0.record()
+        a @ b
+        e1.record()
+        torch.cuda.synchronize()
+        best = min(best, e0.elapsed_time(e1))
+    del a, b
+    torch.cuda.empty_cache()
+    return 2.0 * n ** 3 / (best * 1e-3)
+
+
+def oracle_sample(A, perm, target_gflop: float):
+    """The bounded CPU sample: one whole elimination subtree of the workload
+    (closed under descendants, so the oracle factors it exactly as in the full run)."""
+    import oracle
+    sym = oracle.symbolic(A, perm)
+    ch = sym.children()
+    cc = sym.cc.astype(np.float64)
+    first = sym.sn_first
+    own = np.array([np.sum(cc[first[s]:first[s + 1]] ** 2) for s in range(sym.nsuper)])
+    sub = own.copy()
+    for s in range(sym.nsuper):
+        for q in ch[s]:
+            sub[s] += sub[q]
+    r = int(np.argmin(np.abs(sub - target_gflop * 1e9)))
+    subset, stack = [], [r]
+    while stack:
+        v = stack.pop()
+        subset.append(v)
+        stack.extend(ch[v])
+    return sym, sorted(subset), float(sub[r]), r
+
+
+def run_oracle_steps(A, sym, subset, steps: int):
+    import oracle
+    times = []
+    for _ in range(steps):
+        t0 = time.perf_counter()
+        oracle.factor(A, sym, subset=subset)
+        times.append(time.perf_counter() - t0)
+    return times
+
+
+def cpu_cores() -> int:
+    try:
+        from threadpoolctl import threadpool_info
+        th = [i.get("num_threads", 0) for i in threadpool_info() if i.get("user_api") == "blas"]
+        if th:
+            return int(max(th))
+    except Exception:
+        pass
+    return os.cpu_count() or 1
+
+
+# ------------------------------------------------------------------ reference arm
+def run_reference(args):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return 0
+    c = G.CONFIGS[args.config]
+    A, perm = G.make_config(c["kind"], c["N"])
+    sym, subset, gflop, root = oracle_sample(A, perm, args.cpu_sample_gflop)
+    run_oracle_steps(A, sym, subset, args.warmup)
+    times = run_oracle_steps(A, sym, subset, args.steps)
+    t = float(np.mean(times))
+    value = gflop / t / 1e9
+    sample = (f"oracle.factor of the whole elimination subtree rooted at supernode {root} "
+              f"({len(subset)} fronts, {gflop:.3e} true flops) of {args.config}, incl. B assembly")
+    line = {
+        "impl": "reference", "metric": "fp64 factorization GFLOP/s", "value": value, "unit": "GFLOP/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": c["desc"] + f" [{args.config}], CPU oracle sample", "n": A.n},
+        "cpu_baseline": {"value": value, "unit": "GFLOP/s", "cores": cpu_cores(), "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "gpu_launches": 0,
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ product arm
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    rank, world, local = dist_env()
+    import torch
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    torch.cuda.set_device(local)
+    import paper_conf_ipps_georgesgsc11_b200 as mf
+
+    c = G.CONFIGS[args.config]
+    A, perm = G.make_config(c["kind"], c["N"])
+    stream = torch.cuda.Stream()
+    S = mf.Solver(device=local, stream=stream.cuda_stream, small_front_max=args.small_front_max,
+                  panel_w=args.panel_w)
+    S.analyze(A.n, A.colptr, A.rowind, perm)
+    info = S.info()
+    flops = float(info["flops_true"])
+    vals_d = torch.from_numpy(A.values).cuda()
+    torch.cuda.synchronize()
+
+    def barrier():
+        if world > 1:
+            torch.distributed.barrier()
+
+    for _ in range(max(args.warmup, 3)):
+        S.factor(vals_d)
+    barrier()
+    torch.cuda.synchronize()
+    sampler = ClockSampler(local)
+    sampler.start()
+    time.sleep(0.3)
+    S.set_profiling(True)
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    barrier()
+    torch.cuda.synchronize()
+    e0.record(stream)
+    for _ in range(args.steps):
+        S.factor(vals_d)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    barrier()
+    clocks = sampler.stop()
+    ms = e0.elapsed_time(e1) / args.steps
+    stats = S.kernel_stats()
+    S.set_profiling(False)
+    info = S.info()
+    if world > 1:
+        t = torch.tensor([ms], device="cuda", dtype=torch.float64)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ms = float(t.item())
+    value = world * flops / (ms * 1e-3) / 1e9
+
+    # ---- end to end through the C ABI with HOST buffers (pinned), factor + solve
+    vals_h = torch.from_numpy(A.values).pin_memory()
+    b_h = torch.from_numpy(G.rhs(A.n, 0)).pin_memory()
+    x_h = torch.empty(A.n, dtype=torch.float64).pin_memory()
+    S.factor(vals_h)
+    S.solve(b_h, x_h)
+    barrier()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        S.factor(vals_h)
+        S.solve(b_h, x_h)
+    t_e2e = (time.perf_counter() - t0) / args.steps
+    if world > 1:
+        t = torch.tensor([t_e2e], device="cuda", dtype=torch.float64)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        t_e2e = float(t.item())
+    t_solve = S.info()["t_solve"]
+
+    # ---- roofline of the dominant kernel (by event time inside the timed region)
+    dom = max(stats, key=lambda s: s["ms"])
+    peak_meas = measured_dgemm_peak(torch)
+    traffic = None
+    try:
+        prof = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
+        traffic = prof.get(dom["name"])
+    except (OSError, ValueError):
+        pass
+    if dom["name"] == "dmma_schur_update":
+        achieved = dom["flops"] / (dom["ms"] * 1e-3) / 1e12
+        roof = {"kernel": dom["name"], "bound": "tensor", "achieved": achieved, "peak": peak_meas / 1e12,
+                "unit": "TFLOP/s", "frac": achieved / (peak_meas / 1e12), "traffic": traffic,
+                "peak_source": "cuBLAS DGEMM 8192^3 burst measured in this run (fp64 DMMA path)",
+                "frac_of_nominal_37.2": achieved / (PEAK_NOMINAL_FP64 / 1e12),
+                "launches": dom["launches"] // max(args.steps, 1), "share_of_step": dom["ms"] / (ms * args.steps)}
+    else:
+        hbm = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"] \
+            if os.path.exists(os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6650.0
+        achieved = dom["bytes"] / (dom["ms"] * 1e-3) / 1e9
+        roof = {"kernel": dom["name"], "bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                "frac": achieved / hbm, "traffic": traffic,
+                "launches": dom["launches"] // max(args.steps, 1), "share_of_step": dom["ms"] / (ms * args.steps)}
+
+    line = {
+        "metric": "fp64 factorization GFLOP/s", "value": value, "unit": "GFLOP/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "seconds_per_factorization": ms * 1e-3,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "pct_of_fp64_peak": {"nominal_37.2TF": value / (world * PEAK_NOMINAL_FP64 / 1e9),
+                             "measured_dgemm": value / (world * peak_meas / 1e9)},
+        "config": {"workload": c["desc"] + f" [{args.config}]", "n": A.n, "nnz_lower": A.nnz,
+                   "flops_true": flops, "flops_exec": float(info["flops_exec"]), "nsuper": info["nsuper"],
+                   "max_front": info["max_front"], "parallelism": f"replicas{world}" if world > 1 else "1 GPU",
+                   "l2": "no flush: working set (L = %.1f GB) >> 126 MB L2" % (info["panel_words"] * 8 / 1e9)},
+        "clocks": clocks,
+        "e2e": {"value": flops * world / t_e2e / 1e9, "unit": "GFLOP/s",
+                "what": "mf_factor(host pinned values) + mf_solve(host b -> host x), host wall",
+                "seconds": t_e2e, "solve_seconds": t_solve,
+                "h2d_bytes_per_step": int(A.nnz * 8 + A.n * 8), "d2h_bytes_per_step": int(A.n * 8 + 4)},
+        "gpu_launches": int(info["launches_factor"]) * args.steps,
+        "roofline": roof,
+        "kernels": [{k: (round(v, 4) if isinstance(v, float) else v) for k, v in s.items()} for s in stats],
+    }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        sym, subset, gflop, root = oracle_sample(A, perm, args.cpu_sample_gflop)
+        times = run_oracle_steps(A, sym, subset, 1)
+        line["cpu_baseline"] = {
+            "value": gflop / times[0] / 1e9, "unit": "GFLOP/s", "cores": cpu_cores(), "kind": "oracle",
+            "sample": (f"oracle.factor of the whole elimination subtree rooted at supernode {root} "
+                       f"({len(subset)} fronts, {gflop:.3e} true flops) of {args.config}, incl. B assembly"),
+            "seconds": times[0]}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        torch.distributed.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -91,6 +91,19 @@ typedef struct {
     double t_solve;           /* seconds (device events) of the last mf_solve */
 } mf_info;
 
+/* Per-kernel-class statistics of profiled factorizations (mf_set_profiling):
+ * CUDA-event time on the ctx stream around every launch of the class, and the
+ * ALGORITHMIC flops / HBM bytes of those launches. */
+typedef struct {
+    char name[32];
+    int64_t launches;
+    double ms;
+    double flops;
+    double bytes;
+} mf_kernel_stat;
+
+#define MF_KERNEL_CLASSES 5
+
 /* Fill *opt with the defaults. */
 int mf_default_options(mf_options *opt);
 
@@ -137,6 +150,26 @@ int mf_export_diag(const mf_ctx *ctx, double *out);
 
 /* Copy every panel (supernode order, each f*k as above) to host: out[sum f*k]. */
 int mf_export_L(const mf_ctx *ctx, double *out);
+
+/* The static launch program mf_factor replays (one entry per kernel launch, in
+ * order; the leading init launch is not listed).  kind = kernel class index
+ * (order of mf_kernel_stat), count = CTAs (tasks) of the launch. */
+typedef struct {
+    int32_t kind;
+    int32_t level;
+    int64_t count;
+    double flops;
+    double bytes;
+} mf_launch_info;
+
+/* out may be NULL to query *count only. */
+int mf_get_program(const mf_ctx *ctx, mf_launch_info *out, int64_t max, int64_t *count);
+
+/* Enable (1) / disable (0) per-launch CUDA-event timing in mf_factor; resets the stats. */
+int mf_set_profiling(mf_ctx *ctx, int enable);
+
+/* out[MF_KERNEL_CLASSES]: accumulated stats since the last mf_set_profiling; *count = classes written. */
+int mf_get_kernel_stats(const mf_ctx *ctx, mf_kernel_stat *out, int32_t *count);
 
 void mf_destroy(mf_ctx *ctx);
 

@@ -45,6 +45,10 @@ struct mf_ctx {
     int *d_failed = nullptr;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     int64_t launches = 0;
+    bool profiling = false;
+    std::vector<cudaEvent_t> prof_events;
+    mf_kernel_stat kstats[KC_COUNT];
+    int64_t prof_factors = 0;
 };
 
 namespace {
@@ -215,6 +219,7 @@ void mf_destroy(mf_ctx *c) {
     cudaSetDevice(c->device);
     if (c->stream) cudaStreamSynchronize(c->stream);
     free_device(c);
+    for (cudaEvent_t e : c->prof_events) cudaEventDestroy(e);
     if (c->ev0) cudaEventDestroy(c->ev0);
     if (c->ev1) cudaEventDestroy(c->ev1);
     if (c->own_stream) cudaStreamDestroy(c->stream);
@@ -337,28 +342,26 @@ int mf_factor(mf_ctx *c, const double *values) {
     int64_t launches = 0;
     launch_init_failed(c->d_failed, st);
     launches++;
-    for (int l = 0; l < P.nlevels; l++) {
-        const LevelPlan &LP = P.levels[l];
-        for (int cls = 0; cls < kSmallClasses; cls++) {
-            const int a = LP.small_class_off[cls], b = LP.small_class_off[cls + 1];
-            if (b > a) {
-                launch_small_fronts(d, c->d_small + a, b - a, P.small_class_fmax[cls], vals, st);
-                launches++;
-            }
+    const bool prof = c->profiling;
+    if (prof && c->prof_events.size() < 2 * P.program.size()) {
+        for (size_t i = c->prof_events.size(); i < 2 * P.program.size(); i++) {
+            cudaEvent_t e;
+            CK(cudaEventCreate(&e));
+            c->prof_events.push_back(e);
         }
-        if (LP.nlarge == 0) continue;
-        launch_assemble(d, c->d_asm + 2 * LP.asm_off, LP.nasm, vals, st);
+    }
+    for (size_t li = 0; li < P.program.size(); li++) {
+        const Launch &L = P.program[li];
+        if (prof) CK(cudaEventRecord(c->prof_events[2 * li], st));
+        switch (L.kind) {
+            case KC_SMALL: launch_small_fronts(d, c->d_small + L.off, (int)L.count, L.param, vals, st); break;
+            case KC_ASSEMBLE: launch_assemble(d, c->d_asm + 2 * L.off, L.count, vals, st); break;
+            case KC_POTRF: launch_potrf_diag(d, c->d_large + L.off, (int)L.count, L.param, P.w, st); break;
+            case KC_TRSM: launch_trsm_panel(d, c->d_trsm + 2 * L.off, L.count, L.param, P.w, st); break;
+            case KC_UPDATE: launch_update(d, c->d_probs, c->d_tiles + L.off, L.count, st); break;
+        }
+        if (prof) CK(cudaEventRecord(c->prof_events[2 * li + 1], st));
         launches++;
-        for (const auto &W : LP.waves) {
-            launch_potrf_diag(d, c->d_large + LP.large_off, W.nactive, W.j0, P.w, st);
-            launch_trsm_panel(d, c->d_trsm + 2 * W.trsm_off, W.ntrsm, W.j0, P.w, st);
-            launch_update(d, c->d_probs, c->d_tiles + W.tile_off, W.ntile, st);
-            launches += 1 + (W.ntrsm > 0) + (W.ntile > 0);
-        }
-        if (LP.syrk_ntile > 0) {
-            launch_update(d, c->d_probs, c->d_tiles + LP.syrk_tile_off, LP.syrk_ntile, st);
-            launches++;
-        }
     }
     CK(cudaGetLastError());
     int failed = INT_MAX;
@@ -369,6 +372,19 @@ int mf_factor(mf_ctx *c, const double *values) {
     cudaEventElapsedTime(&ms, c->ev0, c->ev1);
     c->info.t_factor = ms * 1e-3;
     c->info.launches_factor = launches;
+    if (prof) {
+        for (size_t li = 0; li < P.program.size(); li++) {
+            const Launch &L = P.program[li];
+            float t = 0.f;
+            cudaEventElapsedTime(&t, c->prof_events[2 * li], c->prof_events[2 * li + 1]);
+            mf_kernel_stat &K = c->kstats[L.kind];
+            K.launches += 1;
+            K.ms += t;
+            K.flops += L.flops;
+            K.bytes += L.bytes;
+        }
+        c->prof_factors++;
+    }
     if (failed != INT_MAX) {
         c->info.failed_col = c->S.perm[failed];
         c->state = 3;
@@ -455,6 +471,38 @@ int mf_export_panel(const mf_ctx *c, int32_t s, double *out) {
     CK(cudaMemcpy2DAsync(out, f * sizeof(double), c->d.L + c->P.L_off[s], ld * sizeof(double), f * sizeof(double), k,
                          cudaMemcpyDeviceToHost, c->stream));
     CK(cudaStreamSynchronize(c->stream));
+    return MF_OK;
+}
+
+static const char *kKernelNames[KC_COUNT] = {"small_front_fused", "assemble_extend_add", "potrf_diag",
+                                             "trsm_panel", "dmma_schur_update"};
+
+int mf_set_profiling(mf_ctx *c, int enable) {
+    if (!c) return MF_ERR_ARG;
+    c->profiling = enable != 0;
+    for (int k = 0; k < KC_COUNT; k++) {
+        c->kstats[k] = mf_kernel_stat{};
+        snprintf(c->kstats[k].name, sizeof(c->kstats[k].name), "%s", kKernelNames[k]);
+    }
+    c->prof_factors = 0;
+    return MF_OK;
+}
+
+int mf_get_program(const mf_ctx *c, mf_launch_info *out, int64_t max, int64_t *count) {
+    if (!c || !count) return MF_ERR_ARG;
+    if (c->state < 1) return MF_ERR_STATE;
+    const auto &prog = c->P.program;
+    *count = (int64_t)prog.size();
+    if (out)
+        for (int64_t i = 0; i < std::min<int64_t>(max, (int64_t)prog.size()); i++)
+            out[i] = mf_launch_info{prog[i].kind, prog[i].level, prog[i].count, prog[i].flops, prog[i].bytes};
+    return MF_OK;
+}
+
+int mf_get_kernel_stats(const mf_ctx *c, mf_kernel_stat *out, int32_t *count) {
+    if (!c || !out || !count) return MF_ERR_ARG;
+    for (int k = 0; k < KC_COUNT; k++) out[k] = c->kstats[k];
+    *count = KC_COUNT;
     return MF_OK;
 }
 

@@ -193,40 +193,45 @@ void launch_assemble(const DevPlan &d, const int32_t *tasks, int64_t count, cons
 // one CTA per active front factors its diagonal block
 // [j0, j0+we) x [j0, j0+we) in shared memory (right-looking, unblocked).
 constexpr int kWmax = 64;
-constexpr int kPotrfThreads = 256;
+constexpr int kPotrfThreads = 256;   // 4 threads per row of the 64 x 64 block
 __global__ void __launch_bounds__(kPotrfThreads) k_potrf_diag(DevPlan d, const int32_t *__restrict__ fronts,
                                                               int j0, int w) {
-    __shared__ double A[kWmax * (kWmax + 1)];
-    constexpr int LDA = kWmax + 1;
+    constexpr int LDA = kWmax + 1;        // row-major, odd stride: conflict-free row-per-thread access
+    __shared__ double A[kWmax * LDA];
+    __shared__ double sh_inv;
     const int s = fronts[blockIdx.x];
     const int k = d.sn_k[s], ld = d.sn_ld[s], first = d.sn_first[s];
     const int we = min(w, k - j0);
     double *__restrict__ P = d.L + d.L_off[s] + (int64_t)j0 * ld + j0;
-    const int tid = threadIdx.x;
-    for (int idx = tid; idx < we * we; idx += kPotrfThreads) {
-        const int i = idx % we, c = idx / we;
-        A[i + c * LDA] = P[i + (int64_t)c * ld];
+    const int tid = threadIdx.x, i = tid >> 2, h = tid & 3;
+    for (int c = tid >> 6; c < we; c += kPotrfThreads / 64) {
+        const int r = tid & 63;
+        if (r < we) A[r * LDA + c] = P[r + (int64_t)c * ld];
     }
     __syncthreads();
     for (int j = 0; j < we; j++) {
-        const double djj = A[j + j * LDA];
-        const double piv = sqrt(djj);
-        for (int i = j + 1 + tid; i < we; i += kPotrfThreads) A[i + j * LDA] /= piv;
-        __syncthreads();
-        if (tid == 0) {
+        // phase 1: the thread that last updated A[j][j] takes the pivot
+        if (i == j && h == 0) {
+            const double djj = A[j * LDA + j];
+            const double piv = sqrt(djj);
             note_pivot(d, djj, first + j0 + j);
-            A[j + j * LDA] = piv;
-        }
-        const int nr = we - j - 1;
-        for (int idx = tid; idx < nr * nr; idx += kPotrfThreads) {
-            const int i = j + 1 + idx % nr, c = j + 1 + idx / nr;
-            if (i >= c) A[i + c * LDA] -= A[i + j * LDA] * A[c + j * LDA];
+            A[j * LDA + j] = piv;
+            sh_inv = 1.0 / piv;
         }
         __syncthreads();
+        // phase 2: scale column j
+        if (h == 0 && i > j && i < we) A[i * LDA + j] *= sh_inv;
+        __syncthreads();
+        // phase 3: rank-1 update of row i, columns (j, i]; A[c][j] is final for c <= i
+        if (i > j && i < we) {
+            const double l = A[i * LDA + j];
+            for (int c = j + 1 + h; c <= i; c += 4) A[i * LDA + c] -= l * A[c * LDA + j];
+        }
     }
-    for (int idx = tid; idx < we * we; idx += kPotrfThreads) {
-        const int i = idx % we, c = idx / we;
-        if (i >= c) P[i + (int64_t)c * ld] = A[i + c * LDA];
+    __syncthreads();
+    for (int c = tid >> 6; c < we; c += kPotrfThreads / 64) {
+        const int r = tid & 63;
+        if (r < we && r >= c) P[r + (int64_t)c * ld] = A[r * LDA + c];
     }
 }
 
@@ -240,53 +245,50 @@ void launch_potrf_diag(const DevPlan &d, const int32_t *fronts, int count, int j
 // span the rest of L1 and all of L2: "we perform trsm on a (m + k - w) x w
 // matrix which spans both L1 and L2").  Substitution order
 // (ascending columns), no explicit inverse: integer-exact on manufactured inputs.
-constexpr int kTrsmThreads = 256;
-__global__ void __launch_bounds__(kTrsmThreads) k_trsm_panel(DevPlan d, const int32_t *__restrict__ tasks,
-                                                             int j0, int w) {
-    extern __shared__ double trsm_sm[];
-    double *Ls = trsm_sm;                          // w x w diagonal block
-    double *X = trsm_sm + kWmax * (kWmax + 1);     // 64 rows x w
-    constexpr int LDL = kWmax + 1, LDX = kTrsmRows + 1;
+constexpr int kTrsmThreads = kTrsmRows;   // one thread per row
+__global__ void __launch_bounds__(kTrsmThreads, 2) k_trsm_panel(DevPlan d, const int32_t *__restrict__ tasks,
+                                                                int j0, int w) {
+    __shared__ __align__(16) double Ls[kWmax * kWmax];   // column-major L11 (padded with identity)
+    __shared__ double inv[kWmax];
     const int s = tasks[2 * blockIdx.x], r0 = tasks[2 * blockIdx.x + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s];
     const int we = min(w, k - j0);
-    const int nr = min(kTrsmRows, f - r0);
     const double *__restrict__ D = d.L + d.L_off[s] + (int64_t)j0 * ld + j0;
     double *__restrict__ B = d.L + d.L_off[s] + (int64_t)j0 * ld + r0;
     const int tid = threadIdx.x;
-    for (int idx = tid; idx < we * we; idx += kTrsmThreads) {
-        const int i = idx % we, c = idx / we;
-        Ls[i + c * LDL] = D[i + (int64_t)c * ld];
-    }
-    for (int idx = tid; idx < kTrsmRows * we; idx += kTrsmThreads) {
-        const int i = idx % kTrsmRows, c = idx / kTrsmRows;
-        X[i + c * LDX] = i < nr ? B[i + (int64_t)c * ld] : 0.0;
+    for (int idx = tid; idx < kWmax * kWmax; idx += kTrsmThreads) {
+        const int i = idx & (kWmax - 1), c = idx / kWmax;
+        double v = (i == c) ? 1.0 : 0.0;
+        if (i < we && c < we && i >= c) v = D[i + (int64_t)c * ld];
+        Ls[idx] = v;
     }
     __syncthreads();
-    const int r = tid % kTrsmRows, g = tid / kTrsmRows;
-    constexpr int NG = kTrsmThreads / kTrsmRows;
-    for (int c = 0; c < we; c++) {
-        if (g == 0) X[r + c * LDX] /= Ls[c + c * LDL];
-        __syncthreads();
-        const double xc = X[r + c * LDX];
-        for (int cc = c + 1 + g; cc < we; cc += NG) X[r + cc * LDX] -= xc * Ls[cc + c * LDL];
-        __syncthreads();
+    if (tid < kWmax) inv[tid] = 1.0 / Ls[tid * kWmax + tid];
+    const bool row_ok = tid < f - r0;
+    double x[kWmax];
+#pragma unroll
+    for (int c = 0; c < kWmax; c++) x[c] = (row_ok && c < we) ? B[tid + (int64_t)c * ld] : 0.0;
+    __syncthreads();
+    // x L11^T = b by substitution, ascending columns (no explicit inverse of L11):
+    // x_c = (b_c - sum_{p<c} x_p L_cp) / L_cc, the sum accumulated in ascending p
+#pragma unroll
+    for (int c = 0; c < kWmax; c++) {
+        const double *Lr = Ls + c;                 // row c of L11: Ls[c + p * kWmax]
+        double acc = x[c];
+#pragma unroll
+        for (int p = 0; p < c; p++) acc -= x[p] * Lr[p * kWmax];
+        x[c] = acc * inv[c];
     }
-    for (int idx = tid; idx < kTrsmRows * we; idx += kTrsmThreads) {
-        const int i = idx % kTrsmRows, c = idx / kTrsmRows;
-        if (i < nr) B[i + (int64_t)c * ld] = X[i + c * LDX];
+    if (row_ok) {
+#pragma unroll
+        for (int c = 0; c < kWmax; c++)
+            if (c < we) B[tid + (int64_t)c * ld] = x[c];
     }
 }
 
 void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, cudaStream_t st) {
     if (count <= 0) return;
-    constexpr size_t smem = (size_t)(kWmax * (kWmax + 1) + (kTrsmRows + 1) * kWmax) * sizeof(double);
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(k_trsm_panel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        attr = true;
-    }
-    k_trsm_panel<<<(unsigned)count, kTrsmThreads, smem, st>>>(d, tasks, j0, w);
+    k_trsm_panel<<<(unsigned)count, kTrsmThreads, 0, st>>>(d, tasks, j0, w);
 }
 
 // ============================================================ DMMA Schur update
@@ -355,11 +357,22 @@ __global__ void __launch_bounds__(gemm::NT, 2) k_update(double *__restrict__ Lar
         }
     };
 
+    // accumulators start from C (loaded while the first stages are in flight);
+    // the DMMA then accumulates C - A B^T directly, so the epilogue is a store
+    double *__restrict__ C = (g.c_in_U ? Uarena : Larena) + g.c_off;
+    const int ldc = g.ldc;
     double acc[4][4][2];
 #pragma unroll
-    for (int a = 0; a < 4; a++)
+    for (int mb = 0; mb < 4; mb++) {
+        const int i = i0 + wm * 32 + mb * 8 + gq;
 #pragma unroll
-        for (int b = 0; b < 4; b++) acc[a][b][0] = acc[a][b][1] = 0.0;
+        for (int nb = 0; nb < 4; nb++)
+#pragma unroll
+            for (int e = 0; e < 2; e++) {
+                const int j = j0 + wn * 32 + nb * 8 + 2 * tq + e;
+                acc[mb][nb][e] = (i < g.M && j < g.N) ? C[i + (int64_t)j * ldc] : 0.0;
+            }
+    }
 
     const int KT = (K + BK - 1) / BK;
 #pragma unroll
@@ -381,7 +394,7 @@ __global__ void __launch_bounds__(gemm::NT, 2) k_update(double *__restrict__ Lar
         for (int kk = 0; kk < BK / 4; kk++) {
             double a[4], b[4];
 #pragma unroll
-            for (int mb = 0; mb < 4; mb++) a[mb] = As[(kk * 4 + tq) * SA + mb * 8];
+            for (int mb = 0; mb < 4; mb++) a[mb] = -As[(kk * 4 + tq) * SA + mb * 8];
 #pragma unroll
             for (int nb = 0; nb < 4; nb++) b[nb] = Bs[(kk * 4 + tq) * SB + nb * 8];
 #pragma unroll
@@ -391,9 +404,7 @@ __global__ void __launch_bounds__(gemm::NT, 2) k_update(double *__restrict__ Lar
         }
     }
     cp_async_wait<0>();
-    // epilogue: C -= acc on the lower-trapezoid mask
-    double *__restrict__ C = (g.c_in_U ? Uarena : Larena) + g.c_off;
-    const int ldc = g.ldc;
+    // epilogue: store on the lower-trapezoid mask
 #pragma unroll
     for (int mb = 0; mb < 4; mb++) {
         const int i = i0 + wm * 32 + mb * 8 + gq;
@@ -403,7 +414,7 @@ __global__ void __launch_bounds__(gemm::NT, 2) k_update(double *__restrict__ Lar
 #pragma unroll
             for (int e = 0; e < 2; e++) {
                 const int j = j0 + wn * 32 + nb * 8 + 2 * tq + e;
-                if (j < g.N && i >= j) C[i + (int64_t)j * ldc] -= acc[mb][nb][e];
+                if (j < g.N && i >= j) C[i + (int64_t)j * ldc] = acc[mb][nb][e];
             }
         }
     }

@@ -65,21 +65,24 @@ struct TileTask {       // one kTileM x kTileN output tile of a GemmProb
     int32_t tij;        // (ti << 16) | tj
 };
 
-struct LevelPlan {
-    // small fronts: batched fused kernel, grouped in size classes
-    std::vector<int32_t> small_class_off;   // per class, offset into small_list (nclass+1)
-    // large fronts (sorted by k descending)
-    int64_t large_off = 0, nlarge = 0;       // into large_list
-    int64_t asm_off = 0, nasm = 0;           // assembly tasks (int2: front, c0)
-    struct Wave {
-        int32_t j0;
-        int32_t nactive;                     // prefix of the level's large list
-        int64_t trsm_off, ntrsm;             // (front, row-block) tasks
-        int64_t prob_off, nprob;             // update problems
-        int64_t tile_off, ntile;             // update tiles
-    };
-    std::vector<Wave> waves;
-    int64_t syrk_prob_off = 0, syrk_nprob = 0, syrk_tile_off = 0, syrk_ntile = 0;
+// The factorization is a static launch program built once per pattern
+// (mf_analyze) and replayed by every mf_factor.
+enum KernelClass : int32_t {
+    KC_SMALL = 0,     // batched fused small-front kernel (assembly + potrf + trsm + syrk in SMEM)
+    KC_ASSEMBLE = 1,  // large-front assembly (A scatter + extend-add)
+    KC_POTRF = 2,     // w x w diagonal-block potrf
+    KC_TRSM = 3,      // panel trsm below the diagonal block
+    KC_UPDATE = 4,    // DMMA Schur update (panel trailing update and the syrk on U^n)
+    KC_COUNT = 5
+};
+
+struct Launch {
+    int32_t kind;       // KernelClass
+    int32_t param;      // KC_SMALL: class fmax; KC_POTRF/KC_TRSM: j0
+    int64_t off, count; // offset/count into the kind's task array
+    double flops;       // algorithmic flops of this launch
+    double bytes;       // algorithmic HBM bytes of this launch
+    int32_t level;
 };
 
 struct Plan {
@@ -100,12 +103,12 @@ struct Plan {
     std::vector<int32_t> trsm_tasks;                 // pairs (front, row0)
     std::vector<GemmProb> probs;
     std::vector<TileTask> tiles;
-    std::vector<LevelPlan> levels;
+    std::vector<Launch> program;
 };
 
 constexpr int kTileM = 128, kTileN = 64;
 constexpr int kAsmCols = 32;
-constexpr int kTrsmRows = 64;
+constexpr int kTrsmRows = 128;
 constexpr int kSmallClasses = 3;
 
 int build_plan(const Symbolic &S, const Options &opt, Plan &P);

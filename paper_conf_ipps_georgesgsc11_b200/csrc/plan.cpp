@@ -15,6 +15,7 @@
 //   * its update matrix U^s: m_s x m_s column-major (lower triangle used) in the
 //     U arena, written by the F-U of s and read by the extend-add of its parent.
 #include <algorithm>
+#include <functional>
 #include <numeric>
 
 #include "mf.h"
@@ -125,77 +126,133 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     // small-front classes: f <= small_max/4, <= small_max/2, <= small_max
     P.small_class_fmax = {std::max(8, P.small_max / 4), std::max(16, P.small_max / 2), P.small_max};
     const int w = P.w;
-    P.levels.resize(nlev);
+    // algorithmic bytes of assembling front s: its A entries (value + index), the
+    // children's U^c lower triangles and relative maps (read once)
+    auto asm_bytes = [&](int32_t s) {
+        double b = 0;
+        const int64_t e0 = S.bcolptr[S.sn_first[s]], e1 = S.bcolptr[S.sn_first[s + 1]];
+        b += (double)(e1 - e0) * (8 + 4);
+        for (int32_t q = P.child_ptr[s]; q < P.child_ptr[s + 1]; q++) {
+            const double mc = P.sn_f[P.child_list[q]] - P.sn_k[P.child_list[q]];
+            b += 8.0 * mc * (mc + 1) / 2 + 4.0 * mc;
+        }
+        return b;
+    };
+    auto panel_words = [&](int32_t s) {
+        const double k = P.sn_k[s], m = P.sn_f[s] - P.sn_k[s];
+        return k * (k + 1) / 2 + k * m;
+    };
+    auto upd_flops = [](double M, double N, double K) { return 2.0 * K * (N * (N + 1) / 2 + (M - N) * N); };
+    auto upd_bytes = [](double M, double N, double K) { return 8.0 * (M * K + 2 * (N * (N + 1) / 2 + (M - N) * N)); };
     for (int32_t l = 0; l < nlev; l++) {
-        LevelPlan &LP = P.levels[l];
         std::vector<int32_t> fronts(P.level_list.begin() + P.level_ptr[l], P.level_list.begin() + P.level_ptr[l + 1]);
-        LP.small_class_off.assign(kSmallClasses + 1, 0);
-        LP.small_class_off[0] = (int32_t)P.small_list.size();
         for (int cls = 0; cls < kSmallClasses; cls++) {
-            int lo = cls == 0 ? 0 : P.small_class_fmax[cls - 1];
+            const int lo = cls == 0 ? 0 : P.small_class_fmax[cls - 1];
+            Launch L{KC_SMALL, P.small_class_fmax[cls], (int64_t)P.small_list.size(), 0, 0.0, 0.0, l};
             for (int32_t s : fronts)
-                if (P.sn_f[s] > lo && P.sn_f[s] <= P.small_class_fmax[cls]) P.small_list.push_back(s);
-            LP.small_class_off[cls + 1] = (int32_t)P.small_list.size();
+                if (P.sn_f[s] > lo && P.sn_f[s] <= P.small_class_fmax[cls]) {
+                    P.small_list.push_back(s);
+                    const double k = P.sn_k[s], m = P.sn_f[s] - P.sn_k[s];
+                    L.flops += k * m * m + m * k * (k + 1) + k * (k + 1) * (2 * k + 1) / 6;
+                    L.bytes += asm_bytes(s) + 8.0 * (panel_words(s) + m * (m + 1) / 2);
+                }
+            L.count = (int64_t)P.small_list.size() - L.off;
+            if (L.count) P.program.push_back(L);
         }
         std::vector<int32_t> large;
         for (int32_t s : fronts)
             if (P.sn_f[s] > P.small_max) large.push_back(s);
+        if (large.empty()) continue;
         std::stable_sort(large.begin(), large.end(), [&](int32_t a, int32_t b) { return P.sn_k[a] > P.sn_k[b]; });
-        LP.large_off = (int64_t)P.large_list.size();
-        LP.nlarge = (int64_t)large.size();
+        const int64_t large_off = (int64_t)P.large_list.size();
         P.large_list.insert(P.large_list.end(), large.begin(), large.end());
-        // assembly tasks
-        LP.asm_off = (int64_t)P.asm_tasks.size() / 2;
-        for (int32_t s : large)
-            for (int32_t c0 = 0; c0 < P.sn_f[s]; c0 += kAsmCols) {
-                P.asm_tasks.push_back(s);
-                P.asm_tasks.push_back(c0);
-            }
-        LP.nasm = (int64_t)P.asm_tasks.size() / 2 - LP.asm_off;
-        // waves over diagonal blocks of width w
-        int32_t kmax = large.empty() ? 0 : P.sn_k[large[0]];
-        for (int32_t j0 = 0; j0 < kmax; j0 += w) {
-            LevelPlan::Wave W;
-            W.j0 = j0;
-            W.nactive = 0;
-            while (W.nactive < (int32_t)large.size() && P.sn_k[large[W.nactive]] > j0) W.nactive++;
-            W.trsm_off = (int64_t)P.trsm_tasks.size() / 2;
-            W.prob_off = (int64_t)P.probs.size();
-            W.tile_off = (int64_t)P.tiles.size();
-            for (int32_t a = 0; a < W.nactive; a++) {
-                int32_t s = large[a];
-                int32_t k = P.sn_k[s], f = P.sn_f[s], ld = P.sn_ld[s];
-                int32_t we = std::min(w, k - j0);
-                for (int32_t r0 = j0 + we; r0 < f; r0 += kTrsmRows) {
-                    P.trsm_tasks.push_back(s);
-                    P.trsm_tasks.push_back(r0);
+        // assembly
+        {
+            Launch L{KC_ASSEMBLE, 0, (int64_t)P.asm_tasks.size() / 2, 0, 0.0, 0.0, l};
+            for (int32_t s : large) {
+                for (int32_t c0 = 0; c0 < P.sn_f[s]; c0 += kAsmCols) {
+                    P.asm_tasks.push_back(s);
+                    P.asm_tasks.push_back(c0);
                 }
-                int32_t M = f - j0 - we, N = k - j0 - we;
-                if (N > 0 && M > 0) {
-                    GemmProb g;
-                    g.a_off = P.L_off[s] + (int64_t)j0 * ld + (j0 + we);
-                    g.c_off = P.L_off[s] + (int64_t)(j0 + we) * ld + (j0 + we);
-                    g.lda = ld;
-                    g.ldc = ld;
-                    g.M = M;
-                    g.N = N;
-                    g.K = we;
-                    g.c_in_U = 0;
-                    int32_t pid = (int32_t)P.probs.size();
-                    P.probs.push_back(g);
-                    add_tiles(P, pid, M, N);
-                }
+                const double f = P.sn_f[s], k = P.sn_k[s], m = f - k;
+                L.bytes += asm_bytes(s) + 8.0 * (f * k + m * (m + 1) / 2);   // zero + write panel and U
             }
-            W.ntrsm = (int64_t)P.trsm_tasks.size() / 2 - W.trsm_off;
-            W.nprob = (int64_t)P.probs.size() - W.prob_off;
-            W.ntile = (int64_t)P.tiles.size() - W.tile_off;
-            LP.waves.push_back(W);
+            L.count = (int64_t)P.asm_tasks.size() / 2 - L.off;
+            P.program.push_back(L);
         }
-        // final syrk on U^n with inner dimension k
-        LP.syrk_prob_off = (int64_t)P.probs.size();
-        LP.syrk_tile_off = (int64_t)P.tiles.size();
+        // Blocked factorization of the k pivot columns of every large front, in
+        // lockstep over the level (Fig. 9: w x w potrf kernel, trsm
+        // on the rows below it, trailing update).  The trailing updates follow a
+        // recursive split of the block range (left half factored, then ONE update
+        // of the right half with inner dimension = the left half's width, then the
+        // right half), so most flops run with a long inner dimension instead of
+        // w-wide right-looking steps.  A front whose k ends inside the range
+        // simply drops out of the launches beyond its last block.
+        auto nactive_for = [&](int64_t col) {   // fronts (prefix of `large`) with k > col
+            int32_t na = 0;
+            while (na < (int32_t)large.size() && P.sn_k[large[na]] > col) na++;
+            return na;
+        };
+        std::function<void(int32_t, int32_t)> rec = [&](int32_t a, int32_t b) {
+            if (b - a == 1) {
+                const int32_t j0 = a * w;
+                const int32_t na = nactive_for(j0);
+                Launch Lp{KC_POTRF, j0, large_off, na, 0.0, 0.0, l};
+                Launch Lt{KC_TRSM, j0, (int64_t)P.trsm_tasks.size() / 2, 0, 0.0, 0.0, l};
+                for (int32_t q = 0; q < na; q++) {
+                    const int32_t s = large[q];
+                    const int32_t k = P.sn_k[s], f = P.sn_f[s];
+                    const int32_t we = std::min(w, k - j0);
+                    Lp.flops += (double)we * (we + 1) * (2.0 * we + 1) / 6;
+                    Lp.bytes += 8.0 * we * (we + 1);
+                    for (int32_t r0 = j0 + we; r0 < f; r0 += kTrsmRows) {
+                        P.trsm_tasks.push_back(s);
+                        P.trsm_tasks.push_back(r0);
+                    }
+                    const double rows = f - j0 - we;
+                    Lt.flops += rows * we * we;
+                    Lt.bytes += 8.0 * (2 * rows * we + (double)we * (we + 1) / 2);
+                }
+                Lt.count = (int64_t)P.trsm_tasks.size() / 2 - Lt.off;
+                P.program.push_back(Lp);
+                if (Lt.count) P.program.push_back(Lt);
+                return;
+            }
+            const int32_t mid = a + (b - a + 1) / 2;
+            rec(a, mid);
+            const int32_t c0 = mid * w, c_lo = a * w;
+            const int32_t na = nactive_for(c0);
+            Launch Lu{KC_UPDATE, 0, (int64_t)P.tiles.size(), 0, 0.0, 0.0, l};
+            for (int32_t q = 0; q < na; q++) {
+                const int32_t s = large[q];
+                const int32_t k = P.sn_k[s], f = P.sn_f[s], ld = P.sn_ld[s];
+                const int32_t M = f - c0, N = std::min(b * w, k) - c0, K = c0 - c_lo;
+                if (M <= 0 || N <= 0) continue;
+                GemmProb g;
+                g.a_off = P.L_off[s] + (int64_t)c_lo * ld + c0;
+                g.c_off = P.L_off[s] + (int64_t)c0 * ld + c0;
+                g.lda = ld;
+                g.ldc = ld;
+                g.M = M;
+                g.N = N;
+                g.K = K;
+                g.c_in_U = 0;
+                const int32_t pid = (int32_t)P.probs.size();
+                P.probs.push_back(g);
+                add_tiles(P, pid, M, N);
+                Lu.flops += upd_flops(M, N, K);
+                Lu.bytes += upd_bytes(M, N, K);
+            }
+            Lu.count = (int64_t)P.tiles.size() - Lu.off;
+            if (Lu.count) P.program.push_back(Lu);
+            rec(mid, b);
+        };
+        const int32_t nb = (P.sn_k[large[0]] + w - 1) / w;
+        rec(0, nb);
+        // the syrk on U^n with inner dimension k (one launch for the level)
+        Launch Ls{KC_UPDATE, 1, (int64_t)P.tiles.size(), 0, 0.0, 0.0, l};
         for (int32_t s : large) {
-            int32_t k = P.sn_k[s], f = P.sn_f[s], ld = P.sn_ld[s], m = f - k;
+            const int32_t k = P.sn_k[s], f = P.sn_f[s], ld = P.sn_ld[s], m = f - k;
             if (m <= 0) continue;
             GemmProb g;
             g.a_off = P.L_off[s] + k;
@@ -206,12 +263,14 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
             g.N = m;
             g.K = k;
             g.c_in_U = 1;
-            int32_t pid = (int32_t)P.probs.size();
+            const int32_t pid = (int32_t)P.probs.size();
             P.probs.push_back(g);
             add_tiles(P, pid, m, m);
+            Ls.flops += upd_flops(m, m, k);
+            Ls.bytes += upd_bytes(m, m, k);
         }
-        LP.syrk_nprob = (int64_t)P.probs.size() - LP.syrk_prob_off;
-        LP.syrk_ntile = (int64_t)P.tiles.size() - LP.syrk_tile_off;
+        Ls.count = (int64_t)P.tiles.size() - Ls.off;
+        if (Ls.count) P.program.push_back(Ls);
     }
     return MF_OK;
 }

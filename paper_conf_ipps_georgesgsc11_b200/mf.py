@@ -25,7 +25,7 @@ MF_ERR_NCCL = -5
 EXPORTED_SYMBOLS = (
     "mf_default_options", "mf_create", "mf_analyze", "mf_factor", "mf_solve", "mf_get_info",
     "mf_get_perm", "mf_get_etree", "mf_get_supernodes", "mf_export_panel", "mf_export_diag", "mf_export_L",
-    "mf_destroy", "mf_strerror",
+    "mf_get_program", "mf_set_profiling", "mf_get_kernel_stats", "mf_destroy", "mf_strerror",
 )
 
 
@@ -51,6 +51,19 @@ class Info(ctypes.Structure):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
 
+class KernelStat(ctypes.Structure):
+    _fields_ = [("name", ctypes.c_char * 32), ("launches", ctypes.c_int64), ("ms", ctypes.c_double),
+                ("flops", ctypes.c_double), ("bytes", ctypes.c_double)]
+
+
+MF_KERNEL_CLASSES = 5
+
+
+class LaunchInfo(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int32), ("level", ctypes.c_int32), ("count", ctypes.c_int64),
+                ("flops", ctypes.c_double), ("bytes", ctypes.c_double)]
+
+
 def lib_path() -> str:
     return _LIB_PATH
 
@@ -74,6 +87,9 @@ def _load():
         "mf_export_panel": ([vp, i32, vp], ctypes.c_int),
         "mf_export_diag": ([vp, vp], ctypes.c_int),
         "mf_export_L": ([vp, vp], ctypes.c_int),
+        "mf_get_program": ([vp, ctypes.POINTER(LaunchInfo), i64, ctypes.POINTER(i64)], ctypes.c_int),
+        "mf_set_profiling": ([vp, ctypes.c_int], ctypes.c_int),
+        "mf_get_kernel_stats": ([vp, ctypes.POINTER(KernelStat), ctypes.POINTER(i32)], ctypes.c_int),
         "mf_destroy": ([vp], None),
         "mf_strerror": ([ctypes.c_int], ctypes.c_char_p),
     }
@@ -208,6 +224,23 @@ class Solver:
         out = np.empty(f * k, dtype=np.float64)
         self._check(lib.mf_export_panel(self._h, int(s), out.ctypes.data), "mf_export_panel")
         return out.reshape(k, f).T
+
+    def program(self) -> list[dict]:
+        cnt = ctypes.c_int64()
+        self._check(lib.mf_get_program(self._h, None, 0, ctypes.byref(cnt)), "mf_get_program")
+        arr = (LaunchInfo * max(cnt.value, 1))()
+        self._check(lib.mf_get_program(self._h, arr, cnt.value, ctypes.byref(cnt)), "mf_get_program")
+        return [dict(kind=a.kind, level=a.level, count=a.count, flops=a.flops, bytes=a.bytes) for a in arr[:cnt.value]]
+
+    def set_profiling(self, enable: bool = True):
+        self._check(lib.mf_set_profiling(self._h, int(enable)), "mf_set_profiling")
+
+    def kernel_stats(self) -> list[dict]:
+        arr = (KernelStat * MF_KERNEL_CLASSES)()
+        cnt = ctypes.c_int32()
+        self._check(lib.mf_get_kernel_stats(self._h, arr, ctypes.byref(cnt)), "mf_get_kernel_stats")
+        return [dict(name=a.name.decode(), launches=a.launches, ms=a.ms, flops=a.flops, bytes=a.bytes)
+                for a in arr[:cnt.value]]
 
     def diag(self) -> np.ndarray:
         out = np.empty(self.n, dtype=np.float64)
