@@ -43,6 +43,9 @@ struct mf_ctx {
     double *d_values = nullptr;
     double *d_y = nullptr, *d_bx = nullptr;
     int *d_failed = nullptr;
+    int32_t *d_solve_list = nullptr, *d_sf_tasks = nullptr, *d_sb_tasks = nullptr, *d_sb_groups = nullptr;
+    double *d_partials = nullptr;
+    int *d_counters = nullptr;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     int64_t launches = 0;
     bool profiling = false;
@@ -278,6 +281,10 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     UP(&c->d_sn_rowptr, S.sn_rowptr);
     UP(&c->d_probs, P.probs);
     UP(&c->d_tiles, P.tiles);
+    UP(&c->d_solve_list, P.solve_list);
+    UP(&c->d_sf_tasks, P.sf_tasks);
+    UP(&c->d_sb_tasks, P.sb_tasks);
+    UP(&c->d_sb_groups, P.sb_groups);
 #undef UP
     d.sn_first = sn_first;
     d.sn_k = sn_k;
@@ -304,6 +311,10 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     d.fv = (double *)p;
     if ((r = dev_alloc(c, &p, sizeof(int) * 4)) != MF_OK) return r;
     c->d_failed = (int *)p;
+    if ((r = dev_alloc(c, &p, (P.sb_tasks.size() / 3 + 1) * 64 * sizeof(double))) != MF_OK) return r;
+    c->d_partials = (double *)p;
+    if ((r = dev_alloc(c, &p, (P.sb_groups.size() / 2 + 1) * sizeof(int))) != MF_OK) return r;
+    c->d_counters = (int *)p;
     d.failed = c->d_failed;
     if ((r = dev_alloc(c, &p, std::max<int64_t>(S.nnz_in, 1) * sizeof(double))) != MF_OK) return r;
     c->d_values = (double *)p;
@@ -411,11 +422,28 @@ int mf_solve(mf_ctx *c, const double *b, double *x) {
         bd = c->d_bx;
     }
     launch_permute_in(d, bd, c->d_y, n, st);
-    for (int l = 0; l < P.nlevels; l++)
-        launch_fwd_solve(d, c->d_levels + P.level_ptr[l], P.level_ptr[l + 1] - P.level_ptr[l], c->d_y, st);
-    for (int l = P.nlevels - 1; l >= 0; l--)
-        launch_bwd_solve(d, c->d_levels + P.level_ptr[l], P.level_ptr[l + 1] - P.level_ptr[l], c->d_y,
-                         c->d_sn_rows, c->d_sn_rowptr, st);
+    CK(cudaMemsetAsync(c->d_counters, 0, (P.sb_groups.size() / 2 + 1) * sizeof(int), st));
+    for (const SolveLaunch &L : P.fsolve) {
+        switch (L.kind) {
+            case SK_SMALL_F: launch_fwd_solve(d, c->d_solve_list + L.off, (int)L.count, c->d_y, st); break;
+            case SK_INIT_F: launch_fsolve_init(d, c->d_solve_list + L.off, (int)L.count, c->d_y, st); break;
+            case SK_WAVE_F: launch_fsolve_wave(d, c->d_sf_tasks + 3 * L.off, L.count, L.j0, P.w, c->d_y, st); break;
+        }
+    }
+    for (const SolveLaunch &L : P.bsolve) {
+        switch (L.kind) {
+            case SK_SMALL_B:
+                launch_bwd_solve(d, c->d_solve_list + L.off, (int)L.count, c->d_y, c->d_sn_rows, c->d_sn_rowptr, st);
+                break;
+            case SK_INIT_B:
+                launch_bsolve_init(d, c->d_solve_list + L.off, (int)L.count, c->d_y, c->d_sn_rows, c->d_sn_rowptr, st);
+                break;
+            case SK_WAVE_B:
+                launch_bsolve_wave(d, c->d_sb_tasks + 3 * L.off, L.off, L.count, c->d_sb_groups, L.j0, P.w, c->d_y,
+                                   c->d_partials, c->d_counters, st);
+                break;
+        }
+    }
     double *xd = xdev ? x : c->d_bx;
     launch_permute_out(d, c->d_y, xd, n, st);
     if (!xdev) CK(cudaMemcpyAsync(x, c->d_bx, n * sizeof(double), cudaMemcpyDeviceToHost, st));

@@ -525,6 +525,160 @@ __global__ void __launch_bounds__(kSolveThreads) k_bwd_solve(DevPlan d, const in
     }
 }
 
+// ---- large supernodes: blocked by w = 64 columns, many CTAs per supernode
+__global__ void __launch_bounds__(kSolveThreads) k_fsolve_init(DevPlan d, const int32_t *__restrict__ list,
+                                                               const double *__restrict__ y) {
+    const int s = list[blockIdx.x];
+    const int k = d.sn_k[s], f = d.sn_f[s], first = d.sn_first[s];
+    double *__restrict__ v = d.fv + d.fv_off[s];
+    for (int i = threadIdx.x; i < f; i += kSolveThreads) v[i] = i < k ? y[first + i] : 0.0;
+    __syncthreads();
+    for (int q = d.child_ptr[s]; q < d.child_ptr[s + 1]; q++) {
+        const int c = d.child_list[q];
+        const int kc = d.sn_k[c], mc = d.sn_f[c] - kc;
+        const int32_t *__restrict__ rel = d.relmap + d.relmap_ptr[c];
+        const double *__restrict__ vc = d.fv + d.fv_off[c] + kc;
+        for (int p = threadIdx.x; p < mc; p += kSolveThreads) v[rel[p]] += vc[p];
+        __syncthreads();
+    }
+}
+
+constexpr int kSW = 64, kSLD = 65;   // solve block width and smem leading dimension
+
+__device__ __forceinline__ void load_diag_block(const double *__restrict__ P, int ld, int j0, int we,
+                                                double *__restrict__ Lb) {
+    for (int c = threadIdx.x >> 6; c < we; c += kSolveThreads / 64) {
+        const int r = threadIdx.x & 63;
+        if (r < we && r >= c) Lb[r + c * kSLD] = P[(j0 + r) + (int64_t)(j0 + c) * ld];
+    }
+}
+
+__global__ void __launch_bounds__(kSolveThreads) k_fsolve_wave(DevPlan d, const int32_t *__restrict__ tasks, int j0,
+                                                               int w, double *__restrict__ y) {
+    __shared__ double Lb[kSW * kSLD];
+    __shared__ double xs[kSW];
+    const int s = tasks[3 * blockIdx.x], row0 = tasks[3 * blockIdx.x + 1], writer = tasks[3 * blockIdx.x + 2];
+    const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
+    const int we = min(w, k - j0);
+    const double *__restrict__ P = d.L + d.L_off[s];
+    double *__restrict__ v = d.fv + d.fv_off[s];
+    const int tid = threadIdx.x, lane = tid & 31;
+    load_diag_block(P, ld, j0, we, Lb);
+    __syncthreads();
+    if (tid < 32) {   // L11 x = v[j0:j0+we], right-looking, two entries per lane
+        double a0 = lane < we ? v[j0 + lane] : 0.0, a1 = lane + 32 < we ? v[j0 + lane + 32] : 0.0;
+        for (int c = 0; c < we; c++) {
+            const double xc = __shfl_sync(0xffffffffu, c < 32 ? a0 : a1, c & 31) / Lb[c + c * kSLD];
+            if (lane == 0) xs[c] = xc;
+            if (lane > c && lane < we) a0 -= Lb[lane + c * kSLD] * xc;
+            if (lane + 32 > c && lane + 32 < we) a1 -= Lb[lane + 32 + c * kSLD] * xc;
+        }
+    }
+    __syncthreads();
+    if (writer && tid < we) y[first + j0 + tid] = xs[tid];
+    const int r = row0 + tid;
+    if (r < min(row0 + kSolveRows, f)) {
+        double acc = v[r];
+        for (int c = 0; c < we; c++) acc -= P[r + (int64_t)(j0 + c) * ld] * xs[c];
+        v[r] = acc;
+    }
+}
+
+__global__ void __launch_bounds__(kSolveThreads) k_bsolve_init(DevPlan d, const int32_t *__restrict__ list,
+                                                               const double *__restrict__ y,
+                                                               const int32_t *__restrict__ sn_rows,
+                                                               const int64_t *__restrict__ sn_rowptr) {
+    const int s = list[blockIdx.x];
+    const int k = d.sn_k[s], f = d.sn_f[s];
+    double *__restrict__ v = d.fv + d.fv_off[s];
+    const int32_t *__restrict__ R = sn_rows + sn_rowptr[s];
+    for (int i = k + threadIdx.x; i < f; i += kSolveThreads) v[i] = y[R[i]];
+}
+
+__global__ void __launch_bounds__(kSolveThreads) k_bsolve_wave(DevPlan d, const int32_t *__restrict__ tasks,
+                                                               int64_t task_base, const int32_t *__restrict__ groups,
+                                                               int j0, int w, double *__restrict__ y,
+                                                               double *__restrict__ partials, int *__restrict__ counters) {
+    __shared__ double red[kSolveThreads / 32][kSW];
+    __shared__ double Lb[kSW * kSLD];
+    __shared__ double tv[kSW];
+    __shared__ int is_last;
+    const int s = tasks[3 * blockIdx.x], row0 = tasks[3 * blockIdx.x + 1], grp = tasks[3 * blockIdx.x + 2];
+    const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
+    const int we = min(w, k - j0);
+    const double *__restrict__ P = d.L + d.L_off[s];
+    double *__restrict__ v = d.fv + d.fv_off[s];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    // partial (L2^T v)_c over this CTA's row chunk
+    const int r = row0 + tid;
+    const bool rok = r < min(row0 + kSolveRows, f);
+    const double rv = rok ? v[r] : 0.0;
+    for (int c = 0; c < we; c++) {
+        double p = rok ? P[r + (int64_t)(j0 + c) * ld] * rv : 0.0;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) p += __shfl_xor_sync(0xffffffffu, p, o);
+        if (lane == 0) red[warp][c] = p;
+    }
+    __syncthreads();
+    if (tid < we) {
+        double t = 0.0;
+        for (int q = 0; q < kSolveThreads / 32; q++) t += red[q][tid];
+        partials[(task_base + blockIdx.x) * kSW + tid] = t;
+    }
+    __threadfence();
+    __syncthreads();
+    if (tid == 0) is_last = atomicAdd(&counters[grp], 1) == groups[2 * grp + 1] - 1;
+    __syncthreads();
+    if (!is_last) return;
+    __threadfence();
+    // the last CTA of the group reduces the partials in task order (deterministic) and solves L11^T x = t
+    load_diag_block(P, ld, j0, we, Lb);
+    if (tid < we) {
+        const int t0 = groups[2 * grp], nt = groups[2 * grp + 1];
+        double t = y[first + j0 + tid];
+        for (int q = 0; q < nt; q++) t -= __ldcg(&partials[(int64_t)(t0 + q) * kSW + tid]);
+        tv[tid] = t;
+    }
+    __syncthreads();
+    if (tid < 32) {
+        double a0 = lane < we ? tv[lane] : 0.0, a1 = lane + 32 < we ? tv[lane + 32] : 0.0;
+        for (int c = we - 1; c >= 0; c--) {
+            const double xc = __shfl_sync(0xffffffffu, c < 32 ? a0 : a1, c & 31) / Lb[c + c * kSLD];
+            if (lane == (c & 31)) {
+                if (c < 32) a0 = xc; else a1 = xc;
+            }
+            if (lane < c) a0 -= Lb[c + lane * kSLD] * xc;
+            if (lane + 32 < c) a1 -= Lb[c + (lane + 32) * kSLD] * xc;
+        }
+        if (lane < we) {
+            y[first + j0 + lane] = a0;
+            v[j0 + lane] = a0;
+        }
+        if (lane + 32 < we) {
+            y[first + j0 + lane + 32] = a1;
+            v[j0 + lane + 32] = a1;
+        }
+    }
+}
+
+void launch_fsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, cudaStream_t st) {
+    if (count > 0) k_fsolve_init<<<count, kSolveThreads, 0, st>>>(d, list, y);
+}
+void launch_fsolve_wave(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, double *y,
+                        cudaStream_t st) {
+    if (count > 0) k_fsolve_wave<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, j0, w, y);
+}
+void launch_bsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, const int32_t *sn_rows,
+                        const int64_t *sn_rowptr, cudaStream_t st) {
+    if (count > 0) k_bsolve_init<<<count, kSolveThreads, 0, st>>>(d, list, y, sn_rows, sn_rowptr);
+}
+void launch_bsolve_wave(const DevPlan &d, const int32_t *tasks, int64_t task_base, int64_t count, const int32_t *groups,
+                        int j0, int w, double *y, double *partials, int *counters, cudaStream_t st) {
+    if (count > 0)
+        k_bsolve_wave<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, task_base, groups, j0, w, y, partials,
+                                                                  counters);
+}
+
 void launch_fwd_solve(const DevPlan &d, const int32_t *list, int count, double *y, cudaStream_t st) {
     if (count > 0) k_fwd_solve<<<count, kSolveThreads, 0, st>>>(d, list, y);
 }

@@ -38,6 +38,13 @@ void launch_permute_out(const DevPlan &d, const double *xf, double *x, int64_t n
 void launch_fwd_solve(const DevPlan &d, const int32_t *list, int count, double *y, cudaStream_t st);
 void launch_bwd_solve(const DevPlan &d, const int32_t *list, int count, double *y, const int32_t *sn_rows,
                       const int64_t *sn_rowptr, cudaStream_t st);
+void launch_fsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, cudaStream_t st);
+void launch_fsolve_wave(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, double *y,
+                        cudaStream_t st);
+void launch_bsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, const int32_t *sn_rows,
+                        const int64_t *sn_rowptr, cudaStream_t st);
+void launch_bsolve_wave(const DevPlan &d, const int32_t *tasks, int64_t task_base, int64_t count, const int32_t *groups,
+                        int j0, int w, double *y, double *partials, int *counters, cudaStream_t st);
 int small_front_smem_ok(int fmax);
 void launch_export_diag(const DevPlan &d, int nsuper, double *out, cudaStream_t st);
 

@@ -85,6 +85,21 @@ struct Launch {
     int32_t level;
 };
 
+// Triangular-solve program (forward sweep bottom-up, backward sweep top-down).
+enum SolveKind : int32_t {
+    SK_SMALL_F = 0,   // one CTA per small supernode: gather, trsv, gemv
+    SK_INIT_F = 1,    // large supernodes: v = [y(cols); 0] + extend-add of children's update vectors
+    SK_WAVE_F = 2,    // one diagonal block: trsv (redundant per CTA) + gemv of a row chunk
+    SK_SMALL_B = 3,
+    SK_INIT_B = 4,    // large supernodes: v(k:f) = x(R(k:f))
+    SK_WAVE_B = 5     // one diagonal block: partial L2^T v per row chunk, last CTA reduces + trsv
+};
+struct SolveLaunch {
+    int32_t kind;
+    int32_t j0;
+    int64_t off, count;
+};
+
 struct Plan {
     int32_t nsuper = 0, nlevels = 0, w = 64, small_max = 128, max_front = 0;
     int64_t L_words = 0, U_words = 0, rows_total = 0, relmap_total = 0, fv_words = 0;
@@ -104,12 +119,19 @@ struct Plan {
     std::vector<GemmProb> probs;
     std::vector<TileTask> tiles;
     std::vector<Launch> program;
+    // solve
+    std::vector<int32_t> solve_list;                 // supernode lists (small / large) per launch
+    std::vector<int32_t> sf_tasks;                   // forward waves: (front, row0, writer)
+    std::vector<int32_t> sb_tasks;                   // backward waves: (front, row0, group)
+    std::vector<int32_t> sb_groups;                  // (first task, ntasks) per (front, block)
+    std::vector<SolveLaunch> fsolve, bsolve;
 };
 
 constexpr int kTileM = 128, kTileN = 64;
 constexpr int kAsmCols = 32;
 constexpr int kTrsmRows = 128;
 constexpr int kSmallClasses = 3;
+constexpr int kSolveRows = 256;
 
 int build_plan(const Symbolic &S, const Options &opt, Plan &P);
 

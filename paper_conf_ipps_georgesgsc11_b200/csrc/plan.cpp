@@ -33,6 +33,80 @@ static void add_tiles(Plan &P, int32_t prob, int32_t M, int32_t N) {
         }
 }
 
+// Solve program: per level, small supernodes in one batched launch; large ones
+// (f > small_max) blocked by w columns so that no supernode is handled by a
+// single CTA (the root of c5 has k = 14,900).
+static void build_solve_plan(const Symbolic &S, Plan &P) {
+    (void)S;
+    const int w = P.w;
+    std::vector<std::vector<int32_t>> large(P.nlevels), small(P.nlevels);
+    for (int32_t l = 0; l < P.nlevels; l++) {
+        for (int32_t q = P.level_ptr[l]; q < P.level_ptr[l + 1]; q++) {
+            const int32_t s = P.level_list[q];
+            (P.sn_f[s] > P.small_max ? large[l] : small[l]).push_back(s);
+        }
+        std::stable_sort(large[l].begin(), large[l].end(),
+                         [&](int32_t a, int32_t b) { return P.sn_k[a] > P.sn_k[b]; });
+    }
+    auto push_list = [&](const std::vector<int32_t> &v) {
+        const int64_t off = (int64_t)P.solve_list.size();
+        P.solve_list.insert(P.solve_list.end(), v.begin(), v.end());
+        return off;
+    };
+    for (int32_t l = 0; l < P.nlevels; l++) {
+        if (!small[l].empty()) P.fsolve.push_back({SK_SMALL_F, 0, push_list(small[l]), (int64_t)small[l].size()});
+        if (large[l].empty()) continue;
+        P.fsolve.push_back({SK_INIT_F, 0, push_list(large[l]), (int64_t)large[l].size()});
+        const int32_t kmax = P.sn_k[large[l][0]];
+        for (int32_t j0 = 0; j0 < kmax; j0 += w) {
+            const int64_t off = (int64_t)P.sf_tasks.size() / 3;
+            for (int32_t s : large[l]) {
+                const int32_t k = P.sn_k[s], f = P.sn_f[s];
+                if (k <= j0) break;
+                const int32_t r_begin = j0 + std::min(w, k - j0);
+                int32_t r0 = r_begin;
+                do {
+                    P.sf_tasks.push_back(s);
+                    P.sf_tasks.push_back(r0);
+                    P.sf_tasks.push_back(r0 == r_begin ? 1 : 0);
+                    r0 += kSolveRows;
+                } while (r0 < f);
+            }
+            P.fsolve.push_back({SK_WAVE_F, j0, off, (int64_t)P.sf_tasks.size() / 3 - off});
+        }
+    }
+    for (int32_t l = P.nlevels - 1; l >= 0; l--) {
+        if (!large[l].empty()) {
+            P.bsolve.push_back({SK_INIT_B, 0, push_list(large[l]), (int64_t)large[l].size()});
+            const int32_t kmax = P.sn_k[large[l][0]];
+            const int32_t nb = (kmax + w - 1) / w;
+            for (int32_t b = nb - 1; b >= 0; b--) {
+                const int32_t j0 = b * w;
+                const int64_t off = (int64_t)P.sb_tasks.size() / 3;
+                for (int32_t s : large[l]) {
+                    const int32_t k = P.sn_k[s], f = P.sn_f[s];
+                    if (k <= j0) break;
+                    const int32_t grp = (int32_t)P.sb_groups.size() / 2;
+                    const int32_t first_task = (int32_t)(P.sb_tasks.size() / 3);
+                    const int32_t r_begin = j0 + std::min(w, k - j0);
+                    int32_t r0 = r_begin, nt = 0;
+                    do {
+                        P.sb_tasks.push_back(s);
+                        P.sb_tasks.push_back(r0);
+                        P.sb_tasks.push_back(grp);
+                        nt++;
+                        r0 += kSolveRows;
+                    } while (r0 < f);
+                    P.sb_groups.push_back(first_task);
+                    P.sb_groups.push_back(nt);
+                }
+                P.bsolve.push_back({SK_WAVE_B, j0, off, (int64_t)P.sb_tasks.size() / 3 - off});
+            }
+        }
+        if (!small[l].empty()) P.bsolve.push_back({SK_SMALL_B, 0, push_list(small[l]), (int64_t)small[l].size()});
+    }
+}
+
 int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     P = Plan();
     const int32_t ns = (int32_t)S.sn_parent.size();
@@ -272,6 +346,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         Ls.count = (int64_t)P.tiles.size() - Ls.off;
         if (Ls.count) P.program.push_back(Ls);
     }
+    build_solve_plan(S, P);
     return MF_OK;
 }
 
