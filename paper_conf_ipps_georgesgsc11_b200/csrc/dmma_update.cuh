@@ -1,0 +1,166 @@
+// dmma_update.cuh -- the FP64 DMMA Schur-update kernel (the dense contraction of
+// the factor-update step: the syrk U^n = U^n - L2 L2^T of PAPER.md L27 / Fig. 1,
+// and the trailing syrk/gemm updates of the blocked potrf of PAPER.md L325 /
+// Fig. 9), as a template over its tile / pipeline shape.
+//
+//   C[i][j] -= sum_p A[i][p] A[j][p],  0 <= j < N, j <= i < M   (lower trapezoid)
+//
+// A (M x K) and C are column-major with leading dimensions lda / ldc; A lives in
+// the L arena, C in the L arena (panel update) or the U arena (syrk on U^n).
+//
+// sm_100a has no f64 kind of tcgen05.mma (probe 1), so the FP64
+// tensor path is warp-level mma.sync.m8n8k4.f64 (SASS DMMA.8x8x4).  Operands are
+// staged by 16-byte cp.async (LDGSTS, zero-fill at the edges) into a
+// STAGES-deep shared-memory ring; each warp owns a TM x TN sub-tile whose
+// accumulators start from C (loaded while the first stages are in flight) and
+// accumulate C - A B^T directly (A fragments negated), so the epilogue is a
+// masked store.  Columns are 16-byte aligned (lda even); an odd starting row is
+// handled by loading one row early and shifting the shared-memory window.
+#pragma once
+#include <cstdint>
+
+#include "mf_plan.h"
+
+namespace mf {
+
+__device__ __forceinline__ void cp_async16(void *smem, const void *gmem, bool valid) {
+    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    const int n = valid ? 16 : 0;
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(s), "l"(gmem), "r"(n));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
+
+__device__ __forceinline__ void dmma(double &c0, double &c1, double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+                 : "+d"(c0), "+d"(c1)
+                 : "d"(a), "d"(b));
+}
+
+template <int BM_, int BN_, int BK_, int STAGES_, int WARPS_M_, int WARPS_N_, int MINB_>
+struct UpdCfg {
+    static constexpr int BM = BM_, BN = BN_, BK = BK_, STAGES = STAGES_;
+    static constexpr int WARPS_M = WARPS_M_, WARPS_N = WARPS_N_, MINB = MINB_;
+    static constexpr int NT = 32 * WARPS_M * WARPS_N;
+    static constexpr int TM = BM / WARPS_M, TN = BN / WARPS_N;   // warp tile
+    static constexpr int MB = TM / 8, NB = TN / 8;                // DMMA blocks per warp
+    static constexpr int SA = BM + 4, SB = BN + 4;                // +2 shifted rows, +2 pad (stride % 16 == 4)
+    static constexpr int CHA = (BM + 2) / 2, CHB = (BN + 2) / 2;  // 16-byte chunks per column
+    static constexpr int STAGE_WORDS = BK * (SA + SB);
+    static constexpr size_t SMEM = (size_t)STAGES * STAGE_WORDS * sizeof(double);
+    static_assert(SA % 16 == 4 && SB % 16 == 4, "bank-conflict-free fragment loads");
+    static_assert(TM % 8 == 0 && TN % 8 == 0 && BK % 4 == 0, "tile shape");
+};
+
+template <class Cfg>
+__global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
+    k_update_t(double *__restrict__ Larena, double *__restrict__ Uarena, const GemmProb *__restrict__ probs,
+               const TileTask *__restrict__ tiles) {
+    constexpr int BM = Cfg::BM, BN = Cfg::BN, BK = Cfg::BK, STAGES = Cfg::STAGES, NT = Cfg::NT;
+    constexpr int SA = Cfg::SA, SB = Cfg::SB, CHA = Cfg::CHA, CHB = Cfg::CHB, STAGE_WORDS = Cfg::STAGE_WORDS;
+    constexpr int MB = Cfg::MB, NB = Cfg::NB, TM = Cfg::TM, TN = Cfg::TN;
+    extern __shared__ __align__(16) double sm[];
+    const TileTask t = tiles[blockIdx.x];
+    const GemmProb g = probs[t.prob];
+    const int ti = t.tij >> 16, tj = t.tij & 0xffff;
+    const int i0 = ti * BM, j0 = tj * BN;
+    const int sh = (int)(g.a_off & 1);
+    const double *__restrict__ A = Larena + g.a_off - sh;
+    const int lda = g.lda, K = g.K;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int wm = warp % Cfg::WARPS_M, wn = warp / Cfg::WARPS_M;
+    const int gq = lane >> 2, tq = lane & 3;
+
+    auto load_stage = [&](int stage, int kt) {
+        double *As = sm + stage * STAGE_WORDS;
+        double *Bs = As + BK * SA;
+        const int p0 = kt * BK;
+#pragma unroll 2
+        for (int c = tid; c < BK * (CHA + CHB); c += NT) {
+            if (c < BK * CHA) {
+                const int p = c / CHA, ch = c - p * CHA;
+                const int row = i0 + 2 * ch;
+                const bool ok = (p0 + p < K) && (row - sh < g.M);
+                cp_async16(As + p * SA + 2 * ch, ok ? A + row + (int64_t)(p0 + p) * lda : A, ok);
+            } else {
+                const int cc = c - BK * CHA;
+                const int p = cc / CHB, ch = cc - p * CHB;
+                const int row = j0 + 2 * ch;
+                const bool ok = (p0 + p < K) && (row - sh < g.N);
+                cp_async16(Bs + p * SB + 2 * ch, ok ? A + row + (int64_t)(p0 + p) * lda : A, ok);
+            }
+        }
+    };
+
+    const int KT = (K + BK - 1) / BK;
+#pragma unroll
+    for (int st = 0; st < STAGES - 1; st++) {
+        if (st < KT) load_stage(st, st);
+        cp_async_commit();
+    }
+    double *__restrict__ C = (g.c_in_U ? Uarena : Larena) + g.c_off;
+    const int ldc = g.ldc;
+    double acc[MB][NB][2];
+#pragma unroll
+    for (int mb = 0; mb < MB; mb++) {
+        const int i = i0 + wm * TM + mb * 8 + gq;
+#pragma unroll
+        for (int nb = 0; nb < NB; nb++)
+#pragma unroll
+            for (int e = 0; e < 2; e++) {
+                const int j = j0 + wn * TN + nb * 8 + 2 * tq + e;
+                acc[mb][nb][e] = (i < g.M && j < g.N) ? C[i + (int64_t)j * ldc] : 0.0;
+            }
+    }
+    for (int kt = 0; kt < KT; kt++) {
+        cp_async_wait<STAGES - 2>();
+        __syncthreads();
+        {
+            const int nk = kt + STAGES - 1;
+            if (nk < KT) load_stage(nk % STAGES, nk);
+            cp_async_commit();
+        }
+        const double *As = sm + (kt % STAGES) * STAGE_WORDS + sh + wm * TM + gq;
+        const double *Bs = sm + (kt % STAGES) * STAGE_WORDS + BK * SA + sh + wn * TN + gq;
+#pragma unroll
+        for (int kk = 0; kk < BK / 4; kk++) {
+            double a[MB], b[NB];
+#pragma unroll
+            for (int mb = 0; mb < MB; mb++) a[mb] = -As[(kk * 4 + tq) * SA + mb * 8];
+#pragma unroll
+            for (int nb = 0; nb < NB; nb++) b[nb] = Bs[(kk * 4 + tq) * SB + nb * 8];
+#pragma unroll
+            for (int mb = 0; mb < MB; mb++)
+#pragma unroll
+                for (int nb = 0; nb < NB; nb++) dmma(acc[mb][nb][0], acc[mb][nb][1], a[mb], b[nb]);
+        }
+    }
+    cp_async_wait<0>();
+#pragma unroll
+    for (int mb = 0; mb < MB; mb++) {
+        const int i = i0 + wm * TM + mb * 8 + gq;
+        if (i >= g.M) continue;
+#pragma unroll
+        for (int nb = 0; nb < NB; nb++)
+#pragma unroll
+            for (int e = 0; e < 2; e++) {
+                const int j = j0 + wn * TN + nb * 8 + 2 * tq + e;
+                if (j < g.N && i >= j) C[i + (int64_t)j * ldc] = acc[mb][nb][e];
+            }
+    }
+}
+
+template <class Cfg>
+inline void launch_update_t(double *L, double *U, const GemmProb *probs, const TileTask *tiles, int64_t ntiles,
+                            cudaStream_t st) {
+    if (ntiles <= 0) return;
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(k_update_t<Cfg>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Cfg::SMEM);
+        attr = true;
+    }
+    k_update_t<Cfg><<<(unsigned)ntiles, Cfg::NT, Cfg::SMEM, st>>>(L, U, probs, tiles);
+}
+
+}  // namespace mf

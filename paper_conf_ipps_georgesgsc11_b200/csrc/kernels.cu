@@ -15,6 +15,7 @@
 #include <climits>
 #include <cstdio>
 
+#include "dmma_update.cuh"
 #include "kernels.cuh"
 
 namespace mf {
@@ -292,142 +293,12 @@ void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, in
 }
 
 // ============================================================ DMMA Schur update
-// C[i][j] -= sum_p A[i][p] A[j][p]  for a 128 x 64 output tile, lower-trapezoid
-// mask (i >= j, i < M, j < N).  FP64 tensor cores via mma.sync.m8n8k4.f64
-// (SASS DMMA.8x8x4), operands staged by 16-byte cp.async (LDGSTS) in a
-// 3-stage ring, 8 warps each owning a 32 x 32 sub-tile (32 fp64 accumulators
-// per thread), two CTAs per SM.
-namespace gemm {
-constexpr int BM = kTileM, BN = kTileN, BK = 16, STAGES = 3, NT = 256;
-constexpr int SA = BM + 4;   // 130 rows needed (odd-row alignment shift) + pad: 132 % 16 == 4 (conflict-free)
-constexpr int SB = BN + 4;   // 66 rows needed + pad: 68 % 16 == 4
-constexpr int CHA = (BM + 2) / 2, CHB = (BN + 2) / 2;   // 16-byte chunks per column (65, 33)
-constexpr int STAGE_WORDS = BK * (SA + SB);
-constexpr size_t SMEM = (size_t)STAGES * STAGE_WORDS * sizeof(double);
-}  // namespace gemm
-
-__device__ __forceinline__ void cp_async16(void *smem, const void *gmem, bool valid) {
-    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
-    const int n = valid ? 16 : 0;
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(s), "l"(gmem), "r"(n));
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
-
-__device__ __forceinline__ void dmma(double &c0, double &c1, double a, double b) {
-    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
-                 : "+d"(c0), "+d"(c1)
-                 : "d"(a), "d"(b));
-}
-
-__global__ void __launch_bounds__(gemm::NT, 2) k_update(double *__restrict__ Larena, double *__restrict__ Uarena,
-                                                        const GemmProb *__restrict__ probs,
-                                                        const TileTask *__restrict__ tiles) {
-    using namespace gemm;
-    extern __shared__ __align__(16) double sm[];
-    const TileTask t = tiles[blockIdx.x];
-    const GemmProb g = probs[t.prob];
-    const int ti = t.tij >> 16, tj = t.tij & 0xffff;
-    const int i0 = ti * BM, j0 = tj * BN;
-    const int sh = (int)(g.a_off & 1);   // columns are 16B aligned (even lda); shift odd row starts
-    const double *__restrict__ A = Larena + g.a_off - sh;   // aligned base of row -sh
-    const int lda = g.lda, K = g.K;
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int wm = warp & 3, wn = warp >> 2;   // 4 x 2 warps of 32 x 32
-    const int gq = lane >> 2, tq = lane & 3;
-
-    auto load_stage = [&](int stage, int kt) {
-        double *As = sm + stage * STAGE_WORDS;
-        double *Bs = As + BK * SA;
-        const int p0 = kt * BK;
-        for (int c = tid; c < BK * (CHA + CHB); c += NT) {
-            if (c < BK * CHA) {
-                const int p = c / CHA, ch = c - p * CHA;
-                const int row = i0 + 2 * ch;          // aligned row index (relative to -sh)
-                const bool ok = (p0 + p < K) && (row - sh < g.M);
-                cp_async16(As + p * SA + 2 * ch, ok ? A + row + (int64_t)(p0 + p) * lda : A, ok);
-            } else {
-                const int cc = c - BK * CHA;
-                const int p = cc / CHB, ch = cc - p * CHB;
-                const int row = j0 + 2 * ch;
-                const bool ok = (p0 + p < K) && (row - sh < g.N);
-                cp_async16(Bs + p * SB + 2 * ch, ok ? A + row + (int64_t)(p0 + p) * lda : A, ok);
-            }
-        }
-    };
-
-    // accumulators start from C (loaded while the first stages are in flight);
-    // the DMMA then accumulates C - A B^T directly, so the epilogue is a store
-    double *__restrict__ C = (g.c_in_U ? Uarena : Larena) + g.c_off;
-    const int ldc = g.ldc;
-    double acc[4][4][2];
-#pragma unroll
-    for (int mb = 0; mb < 4; mb++) {
-        const int i = i0 + wm * 32 + mb * 8 + gq;
-#pragma unroll
-        for (int nb = 0; nb < 4; nb++)
-#pragma unroll
-            for (int e = 0; e < 2; e++) {
-                const int j = j0 + wn * 32 + nb * 8 + 2 * tq + e;
-                acc[mb][nb][e] = (i < g.M && j < g.N) ? C[i + (int64_t)j * ldc] : 0.0;
-            }
-    }
-
-    const int KT = (K + BK - 1) / BK;
-#pragma unroll
-    for (int st = 0; st < STAGES - 1; st++) {
-        if (st < KT) load_stage(st, st);
-        cp_async_commit();
-    }
-    for (int kt = 0; kt < KT; kt++) {
-        cp_async_wait<STAGES - 2>();
-        __syncthreads();
-        {
-            const int nk = kt + STAGES - 1;
-            if (nk < KT) load_stage(nk % STAGES, nk);
-            cp_async_commit();
-        }
-        const double *As = sm + (kt % STAGES) * STAGE_WORDS + sh + wm * 32 + gq;
-        const double *Bs = sm + (kt % STAGES) * STAGE_WORDS + BK * SA + sh + wn * 32 + gq;
-#pragma unroll
-        for (int kk = 0; kk < BK / 4; kk++) {
-            double a[4], b[4];
-#pragma unroll
-            for (int mb = 0; mb < 4; mb++) a[mb] = -As[(kk * 4 + tq) * SA + mb * 8];
-#pragma unroll
-            for (int nb = 0; nb < 4; nb++) b[nb] = Bs[(kk * 4 + tq) * SB + nb * 8];
-#pragma unroll
-            for (int mb = 0; mb < 4; mb++)
-#pragma unroll
-                for (int nb = 0; nb < 4; nb++) dmma(acc[mb][nb][0], acc[mb][nb][1], a[mb], b[nb]);
-        }
-    }
-    cp_async_wait<0>();
-    // epilogue: store on the lower-trapezoid mask
-#pragma unroll
-    for (int mb = 0; mb < 4; mb++) {
-        const int i = i0 + wm * 32 + mb * 8 + gq;
-        if (i >= g.M) continue;
-#pragma unroll
-        for (int nb = 0; nb < 4; nb++) {
-#pragma unroll
-            for (int e = 0; e < 2; e++) {
-                const int j = j0 + wn * 32 + nb * 8 + 2 * tq + e;
-                if (j < g.N && i >= j) C[i + (int64_t)j * ldc] = acc[mb][nb][e];
-            }
-        }
-    }
-}
+// The production tile shape (kTileM x kTileN in mf_plan.h); variants are
+// benchmarked in tools/ubench/update_variants.cu.
+using UpdProd = UpdCfg<kTileM, kTileN, 16, 3, 2, 2, 4>;   // 29.3 TF/s on M=N=8192,K=4096 (ubench)
 
 void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, cudaStream_t st) {
-    if (ntiles <= 0) return;
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(k_update, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)gemm::SMEM);
-        attr = true;
-    }
-    k_update<<<(unsigned)ntiles, gemm::NT, gemm::SMEM, st>>>(d.L, d.U, probs, tiles);
+    launch_update_t<UpdProd>(d.L, d.U, probs, tiles, ntiles, st);
 }
 
 void launch_init_failed(int *failed, cudaStream_t st) { k_init_failed<<<1, 1, 0, st>>>(failed); }

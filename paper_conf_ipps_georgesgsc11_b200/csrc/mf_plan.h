@@ -127,7 +127,7 @@ struct Plan {
     std::vector<SolveLaunch> fsolve, bsolve;
 };
 
-constexpr int kTileM = 128, kTileN = 64;
+constexpr int kTileM = 64, kTileN = 64;
 constexpr int kAsmCols = 32;
 constexpr int kTrsmRows = 128;
 constexpr int kSmallClasses = 3;
