@@ -239,7 +239,6 @@ def main():
     sampler = ClockSampler(local)
     sampler.start()
     time.sleep(0.3)
-    S.set_profiling(True)
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
     barrier()
@@ -252,7 +251,14 @@ def main():
     barrier()
     clocks = sampler.stop()
     ms = e0.elapsed_time(e1) / args.steps
+    # per-kernel CUDA-event timing: the same steps again with one event pair per
+    # launch on the ctx stream (eager launches instead of the CUDA graph)
+    S.set_profiling(True)
+    for _ in range(args.steps):
+        S.factor(vals_d)
+    torch.cuda.synchronize()
     stats = S.kernel_stats()
+    prof_ms = S.info()["t_factor"] * 1e3
     S.set_profiling(False)
     info = S.info()
     if world > 1:
@@ -295,14 +301,15 @@ def main():
                 "unit": "TFLOP/s", "frac": achieved / (peak_meas / 1e12), "traffic": traffic,
                 "peak_source": "cuBLAS DGEMM 8192^3 burst measured in this run (fp64 DMMA path)",
                 "frac_of_nominal_37.2": achieved / (PEAK_NOMINAL_FP64 / 1e12),
-                "launches": dom["launches"] // max(args.steps, 1), "share_of_step": dom["ms"] / (ms * args.steps)}
+                "launches": dom["launches"] // max(args.steps, 1), "share_of_step": dom["ms"] / (prof_ms * args.steps),
+                "timing": "CUDA events around every launch on the ctx stream, profiled replay of the timed steps"}
     else:
         hbm = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"] \
             if os.path.exists(os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6650.0
         achieved = dom["bytes"] / (dom["ms"] * 1e-3) / 1e9
         roof = {"kernel": dom["name"], "bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
                 "frac": achieved / hbm, "traffic": traffic,
-                "launches": dom["launches"] // max(args.steps, 1), "share_of_step": dom["ms"] / (ms * args.steps)}
+                "launches": dom["launches"] // max(args.steps, 1), "share_of_step": dom["ms"] / (prof_ms * args.steps)}
 
     line = {
         "metric": "fp64 factorization GFLOP/s", "value": value, "unit": "GFLOP/s", "n_gpus": world,
@@ -322,6 +329,7 @@ def main():
         "gpu_launches": int(info["launches_factor"]) * args.steps,
         "roofline": roof,
         "kernels": [{k: (round(v, 4) if isinstance(v, float) else v) for k, v in s.items()} for s in stats],
+        "profiled_ms_per_step": prof_ms,
     }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         sym, subset, gflop, root = oracle_sample(A, perm, args.cpu_sample_gflop)

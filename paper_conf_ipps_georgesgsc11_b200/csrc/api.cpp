@@ -49,6 +49,9 @@ struct mf_ctx {
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     int64_t launches = 0;
     bool profiling = false;
+    bool use_graph = true;
+    cudaGraph_t graph = nullptr;
+    cudaGraphExec_t graph_exec = nullptr;
     std::vector<cudaEvent_t> prof_events;
     mf_kernel_stat kstats[KC_COUNT];
     int64_t prof_factors = 0;
@@ -87,7 +90,15 @@ int dev_alloc(mf_ctx *c, void **dst, size_t bytes) {
     return MF_OK;
 }
 
+void drop_graph(mf_ctx *c) {
+    if (c->graph_exec) cudaGraphExecDestroy(c->graph_exec);
+    if (c->graph) cudaGraphDestroy(c->graph);
+    c->graph_exec = nullptr;
+    c->graph = nullptr;
+}
+
 void free_device(mf_ctx *c) {
+    drop_graph(c);
     for (void *p : c->allocs) cudaFree(p);
     c->allocs.clear();
     c->d = DevPlan{};
@@ -236,6 +247,7 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
         CK(cudaSetDevice(c->device));
         cudaStreamSynchronize(c->stream);
         free_device(c);
+        if (kernels_init()) return MF_ERR_CUDA;
     }
     c->state = 0;
     int st = analyze_symbolic(n, colptr, rowind, perm, c->opt, c->S);
@@ -351,28 +363,53 @@ int mf_factor(mf_ctx *c, const double *values) {
         vals = c->d_values;
     }
     int64_t launches = 0;
-    launch_init_failed(c->d_failed, st);
-    launches++;
     const bool prof = c->profiling;
-    if (prof && c->prof_events.size() < 2 * P.program.size()) {
-        for (size_t i = c->prof_events.size(); i < 2 * P.program.size(); i++) {
-            cudaEvent_t e;
-            CK(cudaEventCreate(&e));
-            c->prof_events.push_back(e);
+    // The launch program: init flag + every launch of P.program, in order.
+    auto issue = [&](const double *v, bool with_events) -> int {
+        launch_init_failed(c->d_failed, st);
+        for (size_t li = 0; li < P.program.size(); li++) {
+            const Launch &L = P.program[li];
+            if (with_events) CK(cudaEventRecord(c->prof_events[2 * li], st));
+            switch (L.kind) {
+                case KC_SMALL: launch_small_fronts(d, c->d_small + L.off, (int)L.count, L.param, v, st); break;
+                case KC_ASSEMBLE: launch_assemble(d, c->d_asm + 2 * L.off, L.count, v, st); break;
+                case KC_POTRF: launch_potrf_diag(d, c->d_large + L.off, (int)L.count, L.param, P.w, st); break;
+                case KC_TRSM: launch_trsm_panel(d, c->d_trsm + 2 * L.off, L.count, L.param, P.w, st); break;
+                case KC_UPDATE: launch_update(d, c->d_probs, c->d_tiles + L.off, L.count, st); break;
+            }
+            if (with_events) CK(cudaEventRecord(c->prof_events[2 * li + 1], st));
         }
-    }
-    for (size_t li = 0; li < P.program.size(); li++) {
-        const Launch &L = P.program[li];
-        if (prof) CK(cudaEventRecord(c->prof_events[2 * li], st));
-        switch (L.kind) {
-            case KC_SMALL: launch_small_fronts(d, c->d_small + L.off, (int)L.count, L.param, vals, st); break;
-            case KC_ASSEMBLE: launch_assemble(d, c->d_asm + 2 * L.off, L.count, vals, st); break;
-            case KC_POTRF: launch_potrf_diag(d, c->d_large + L.off, (int)L.count, L.param, P.w, st); break;
-            case KC_TRSM: launch_trsm_panel(d, c->d_trsm + 2 * L.off, L.count, L.param, P.w, st); break;
-            case KC_UPDATE: launch_update(d, c->d_probs, c->d_tiles + L.off, L.count, st); break;
+        return MF_OK;
+    };
+    launches = 1 + (int64_t)P.program.size();
+    if (prof) {
+        if (c->prof_events.size() < 2 * P.program.size()) {
+            for (size_t i = c->prof_events.size(); i < 2 * P.program.size(); i++) {
+                cudaEvent_t e;
+                CK(cudaEventCreate(&e));
+                c->prof_events.push_back(e);
+            }
         }
-        if (prof) CK(cudaEventRecord(c->prof_events[2 * li + 1], st));
-        launches++;
+        int r = issue(vals, true);
+        if (r) return r;
+    } else if (c->use_graph) {
+        // replay one CUDA graph of the whole program; it always reads the ctx's value buffer
+        if (vals != c->d_values && c->S.nnz_in > 0)
+            CK(cudaMemcpyAsync(c->d_values, vals, c->S.nnz_in * sizeof(double), cudaMemcpyDeviceToDevice, st));
+        if (!c->graph_exec) {
+            CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
+            int r = issue(c->d_values, false);
+            cudaGraph_t g = nullptr;
+            cudaError_t e = cudaStreamEndCapture(st, &g);
+            if (r) return r;
+            CK(e);
+            c->graph = g;
+            CK(cudaGraphInstantiate(&c->graph_exec, g, 0));
+        }
+        CK(cudaGraphLaunch(c->graph_exec, st));
+    } else {
+        int r = issue(vals, false);
+        if (r) return r;
     }
     CK(cudaGetLastError());
     int failed = INT_MAX;

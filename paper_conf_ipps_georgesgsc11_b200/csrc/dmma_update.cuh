@@ -155,10 +155,12 @@ template <class Cfg>
 inline void launch_update_t(double *L, double *U, const GemmProb *probs, const TileTask *tiles, int64_t ntiles,
                             cudaStream_t st) {
     if (ntiles <= 0) return;
-    static bool attr = false;
-    if (!attr) {
-        cudaFuncSetAttribute(k_update_t<Cfg>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Cfg::SMEM);
-        attr = true;
+    if (Cfg::SMEM > 48 * 1024) {   // idempotent; libmf also sets it up front (kernels_init) before graph capture
+        static bool attr = false;
+        if (!attr) {
+            cudaFuncSetAttribute(k_update_t<Cfg>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Cfg::SMEM);
+            attr = true;
+        }
     }
     k_update_t<Cfg><<<(unsigned)ntiles, Cfg::NT, Cfg::SMEM, st>>>(L, U, probs, tiles);
 }

@@ -113,22 +113,20 @@ void launch_small_fronts(const DevPlan &d, const int32_t *list, int count, int f
     } else if (fmax <= 64) {
         k_small_front<128><<<count, 128, smem, st>>>(d, list, values);
     } else {
-        static bool attr = false;
-        if (!attr) {
-            cudaFuncSetAttribute(k_small_front<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-            attr = true;
-        }
         k_small_front<256><<<count, 256, smem, st>>>(d, list, values);
     }
 }
 
 // ============================================================ large-front assembly
-// Task = (front s, first local column c0): zero columns [c0, c0+32) of the
-// front, write the A entries, then extend-add every child's U^c columns that
-// map into these columns (child order ascending, barrier between children, so
-// the summation order is fixed).  Columns < k live in the L panel, columns >= k
-// in U^s.
+// Task = (front s, first local column c0): columns [c0, c0+32) of the front.
+// Columns < k live in the L panel, columns >= k in U^s.
 constexpr int kAsmThreads = 256;
+// Each warp owns whole destination columns (round-robin over the task's 32
+// columns): it zeroes a column, writes its A entries, then adds the matching
+// column of every child's U^c in ascending child order.  Because one warp
+// performs every write to its columns, the order is fixed without barriers or
+// atomics.  The child column that lands in destination column c is found by
+// binary search in the child's (increasing) relative map.
 __global__ void __launch_bounds__(kAsmThreads) k_assemble(DevPlan d, const int32_t *__restrict__ tasks,
                                                           const double *__restrict__ values) {
     const int s = tasks[2 * blockIdx.x], c0 = tasks[2 * blockIdx.x + 1];
@@ -136,51 +134,52 @@ __global__ void __launch_bounds__(kAsmThreads) k_assemble(DevPlan d, const int32
     const int c1 = min(c0 + kAsmCols, f);
     double *__restrict__ P = d.L + d.L_off[s];
     double *__restrict__ Us = d.U + d.U_off[s];
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     constexpr int NW = kAsmThreads / 32;
+    const int q0 = d.child_ptr[s], q1 = d.child_ptr[s + 1];
     for (int c = c0 + warp; c < c1; c += NW) {
+        // destination column: panel column c (rows 0..f-1) or U column c-k (rows c..f-1)
+        double *__restrict__ col;
+        int rlo;
         if (c < k) {
-            for (int i = lane; i < f; i += 32) P[i + (int64_t)c * ld] = 0.0;
+            col = P + (int64_t)c * ld;
+            rlo = 0;
         } else {
-            const int cu = c - k;
-            for (int i = cu + lane; i < m; i += 32) Us[i + (int64_t)cu * m] = 0.0;
+            col = Us + (int64_t)(c - k) * m - k;   // index by front row r >= c
+            rlo = c;
         }
-    }
-    __syncthreads();
-    for (int c = c0 + warp; c < min(c1, k); c += NW) {
-        const int64_t e0 = d.bcolptr[first + c], e1 = d.bcolptr[first + c + 1];
-        for (int64_t e = e0 + lane; e < e1; e += 32) P[d.blrow[e] + (int64_t)c * ld] = sum_values(d, values, e);
-    }
-    __syncthreads();
-    __shared__ int qrange[2];
-    for (int q = d.child_ptr[s]; q < d.child_ptr[s + 1]; q++) {
-        const int ch = d.child_list[q];
-        const int mc = d.sn_f[ch] - d.sn_k[ch];
-        const int32_t *__restrict__ rel = d.relmap + d.relmap_ptr[ch];
-        const double *__restrict__ Uc = d.U + d.U_off[ch];
-        if (tid < 2) {   // child columns qa..qb-1 map into [c0, c1): rel is increasing
-            const int target = tid == 0 ? c0 : c1;
+        for (int r = rlo + lane; r < f; r += 32) col[r] = 0.0;
+        __syncwarp();
+        if (c < k) {
+            const int64_t e0 = d.bcolptr[first + c], e1 = d.bcolptr[first + c + 1];
+            for (int64_t e = e0 + lane; e < e1; e += 32) col[d.blrow[e]] = sum_values(d, values, e);
+            __syncwarp();
+        }
+        for (int q = q0; q < q1; q++) {
+            const int ch = d.child_list[q];
+            const int mc = d.sn_f[ch] - d.sn_k[ch];
+            const int32_t *__restrict__ rel = d.relmap + d.relmap_ptr[ch];
             int lo = 0, hi = mc;
             while (lo < hi) {
                 const int mid = (lo + hi) >> 1;
-                if (rel[mid] < target) lo = mid + 1; else hi = mid;
+                if (__ldg(rel + mid) < c) lo = mid + 1; else hi = mid;
             }
-            qrange[tid] = lo;
-        }
-        __syncthreads();
-        const int qa = qrange[0], qb = qrange[1];
-        for (int qc = qa + warp; qc < qb; qc += NW) {
-            const int dc = rel[qc];
-            const double *__restrict__ ucol = Uc + (int64_t)qc * mc;
-            if (dc < k) {
-                double *__restrict__ pcol = P + (int64_t)dc * ld;
-                for (int p = qc + lane; p < mc; p += 32) pcol[rel[p]] += ucol[p];
-            } else {
-                double *__restrict__ ucol_dst = Us + (int64_t)(dc - k) * m - k;
-                for (int p = qc + lane; p < mc; p += 32) ucol_dst[rel[p]] += ucol[p];
+            if (lo >= mc || __ldg(rel + lo) != c) continue;
+            const double *__restrict__ ucol = d.U + d.U_off[ch] + (int64_t)lo * mc;
+            int p = lo + lane;
+            for (; p + 96 < mc; p += 128) {   // 4 independent gathers in flight per lane
+                const int r0 = __ldg(rel + p), r1 = __ldg(rel + p + 32), r2 = __ldg(rel + p + 64), r3 = __ldg(rel + p + 96);
+                const double u0 = __ldg(ucol + p), u1 = __ldg(ucol + p + 32), u2 = __ldg(ucol + p + 64),
+                             u3 = __ldg(ucol + p + 96);
+                const double v0 = col[r0], v1 = col[r1], v2 = col[r2], v3 = col[r3];
+                col[r0] = v0 + u0;
+                col[r1] = v1 + u1;
+                col[r2] = v2 + u2;
+                col[r3] = v3 + u3;
             }
+            for (; p < mc; p += 32) col[__ldg(rel + p)] += __ldg(ucol + p);
+            __syncwarp();
         }
-        __syncthreads();
     }
 }
 
@@ -194,45 +193,113 @@ void launch_assemble(const DevPlan &d, const int32_t *tasks, int64_t count, cons
 // one CTA per active front factors its diagonal block
 // [j0, j0+we) x [j0, j0+we) in shared memory (right-looking, unblocked).
 constexpr int kWmax = 64;
-constexpr int kPotrfThreads = 256;   // 4 threads per row of the 64 x 64 block
+constexpr int kPotrfThreads = 256;
+// Blocked in-CTA potrf of the 64 x 64 diagonal block, 16 columns at a time:
+//  (a) warp 0 factors the 16 x 16 diagonal sub-block in registers (lane l owns
+//      row l; pivots broadcast by shuffles, no barriers),
+//  (b) one thread per row solves the rows below it against that sub-block,
+//  (c) all threads apply the rank-16 update to the trailing lower triangle.
+// The per-pivot critical path is one rsqrt + a few shuffles instead of two
+// block-wide barriers.  1/L_jj uses rsqrt (exact for the power-of-4 pivots of
+// the manufactured inputs); L_jj = d * rsqrt(d).
 __global__ void __launch_bounds__(kPotrfThreads) k_potrf_diag(DevPlan d, const int32_t *__restrict__ fronts,
                                                               int j0, int w) {
-    constexpr int LDA = kWmax + 1;        // row-major, odd stride: conflict-free row-per-thread access
+    constexpr int LDA = kWmax;            // column-major: A[c * LDA + r]
     __shared__ double A[kWmax * LDA];
-    __shared__ double sh_inv;
+    __shared__ double sinv[kWmax];
     const int s = fronts[blockIdx.x];
     const int k = d.sn_k[s], ld = d.sn_ld[s], first = d.sn_first[s];
     const int we = min(w, k - j0);
     double *__restrict__ P = d.L + d.L_off[s] + (int64_t)j0 * ld + j0;
-    const int tid = threadIdx.x, i = tid >> 2, h = tid & 3;
-    for (int c = tid >> 6; c < we; c += kPotrfThreads / 64) {
-        const int r = tid & 63;
-        if (r < we) A[r * LDA + c] = P[r + (int64_t)c * ld];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    {
+        const int i = tid & 63, h = tid >> 6;
+        double v[kWmax / 4];
+#pragma unroll
+        for (int t = 0; t < kWmax / 4; t++) {
+            const int c = h + 4 * t;
+            v[t] = (i < we && c < we) ? P[i + (int64_t)c * ld] : 0.0;
+        }
+#pragma unroll
+        for (int t = 0; t < kWmax / 4; t++) A[(h + 4 * t) * LDA + i] = v[t];
     }
     __syncthreads();
-    for (int j = 0; j < we; j++) {
-        // phase 1: the thread that last updated A[j][j] takes the pivot
-        if (i == j && h == 0) {
-            const double djj = A[j * LDA + j];
-            const double piv = sqrt(djj);
-            note_pivot(d, djj, first + j0 + j);
-            A[j * LDA + j] = piv;
-            sh_inv = 1.0 / piv;
+#pragma unroll 1
+    for (int s0 = 0; s0 < we; s0 += 16) {
+        const int nb = min(16, we - s0);
+        // (a) 16 x 16 diagonal sub-block in registers of warp 0
+        if (warp == 0) {
+            const int l = lane & 15;
+            double a[16];
+#pragma unroll
+            for (int q = 0; q < 16; q++) a[q] = (q <= l && l < nb) ? A[(s0 + q) * LDA + s0 + l] : 0.0;
+#pragma unroll
+            for (int q = 0; q < 16; q++) {
+                if (q < nb) {
+                    const double dq = __shfl_sync(0xffffffffu, a[q], q);
+                    const double inv = rsqrt(dq);
+                    const double piv = dq * inv;
+                    if (lane == q) {
+                        note_pivot(d, dq, first + j0 + s0 + q);
+                        sinv[s0 + q] = inv;
+                        a[q] = piv;
+                    } else if (l > q) {
+                        a[q] *= inv;
+                    }
+#pragma unroll
+                    for (int c = q + 1; c < 16; c++) {
+                        const double lc = __shfl_sync(0xffffffffu, a[q], c);
+                        if (l >= c) a[c] -= a[q] * lc;
+                    }
+                }
+            }
+            if (lane < nb) {
+#pragma unroll
+                for (int q = 0; q < 16; q++)
+                    if (q <= lane) {
+                        A[(s0 + q) * LDA + s0 + lane] = a[q];
+                        P[(s0 + lane) + (int64_t)(s0 + q) * ld] = a[q];
+                    }
+            }
         }
         __syncthreads();
-        // phase 2: scale column j
-        if (h == 0 && i > j && i < we) A[i * LDA + j] *= sh_inv;
-        __syncthreads();
-        // phase 3: rank-1 update of row i, columns (j, i]; A[c][j] is final for c <= i
-        if (i > j && i < we) {
-            const double l = A[i * LDA + j];
-            for (int c = j + 1 + h; c <= i; c += 4) A[i * LDA + c] -= l * A[c * LDA + j];
+        const int r0 = s0 + 16;
+        if (r0 >= we) break;
+        // (b) rows r in [r0, we): x L_sub^T = a  (one thread per row)
+        if (tid < we - r0) {
+            const int r = r0 + tid;
+            double x[16];
+#pragma unroll
+            for (int q = 0; q < 16; q++) x[q] = A[(s0 + q) * LDA + r];
+#pragma unroll
+            for (int q = 0; q < 16; q++) {
+                x[q] *= sinv[s0 + q];
+#pragma unroll
+                for (int q2 = q + 1; q2 < 16; q2++) x[q2] -= x[q] * A[(s0 + q) * LDA + s0 + q2];
+            }
+#pragma unroll
+            for (int q = 0; q < 16; q++) {
+                A[(s0 + q) * LDA + r] = x[q];
+                P[r + (int64_t)(s0 + q) * ld] = x[q];
+            }
         }
-    }
-    __syncthreads();
-    for (int c = tid >> 6; c < we; c += kPotrfThreads / 64) {
-        const int r = tid & 63;
-        if (r < we && r >= c) P[r + (int64_t)c * ld] = A[r * LDA + c];
+        __syncthreads();
+        // (c) trailing update: A[c][i] -= sum_q L[i][q] L[c][q], r0 <= c <= i < we
+        {
+            const int i = tid & 63, h = tid >> 6;
+            if (i >= r0 && i < we) {
+                double li[16];
+#pragma unroll
+                for (int q = 0; q < 16; q++) li[q] = A[(s0 + q) * LDA + i];
+                for (int c = r0 + h; c <= i; c += 4) {
+                    double acc = A[c * LDA + i];
+#pragma unroll
+                    for (int q = 0; q < 16; q++) acc -= li[q] * A[(s0 + q) * LDA + c];
+                    A[c * LDA + i] = acc;
+                }
+            }
+        }
+        __syncthreads();
     }
 }
 
@@ -246,50 +313,112 @@ void launch_potrf_diag(const DevPlan &d, const int32_t *fronts, int count, int j
 // span the rest of L1 and all of L2: "we perform trsm on a (m + k - w) x w
 // matrix which spans both L1 and L2").  Substitution order
 // (ascending columns), no explicit inverse: integer-exact on manufactured inputs.
-constexpr int kTrsmThreads = kTrsmRows;   // one thread per row
+constexpr int kTrsmThreads = kTrsmRows;   // 4 warps, each owning 32 rows
+constexpr int kTLD = kWmax + 1;             // smem leading dimension (odd: row-per-thread access is conflict-free)
+constexpr size_t kTrsmSmem = (size_t)(kWmax * kTLD + kTrsmRows * kTLD + kWmax) * sizeof(double);
+// X L11^T = B by blocked substitution: for each 8-column block, every thread
+// solves its own row over the block (scalar), then its warp applies the block
+// to the remaining columns of its 32 rows with DMMA (m8n8k4 f64).  Warps never
+// share rows, so only warp-level synchronisation is needed.  No explicit
+// inverse of L11: integer-exact on the manufactured inputs.
 __global__ void __launch_bounds__(kTrsmThreads, 2) k_trsm_panel(DevPlan d, const int32_t *__restrict__ tasks,
                                                                 int j0, int w) {
-    __shared__ __align__(16) double Ls[kWmax * kWmax];   // column-major L11 (padded with identity)
-    __shared__ double inv[kWmax];
+    extern __shared__ double tsm[];
+    double *Ls = tsm;                           // L11, column-major [row + col * kTLD], identity-padded
+    double *X = tsm + kWmax * kTLD;             // rows x 64, row-major [row * kTLD + col]
+    double *inv = X + kTrsmRows * kTLD;
     const int s = tasks[2 * blockIdx.x], r0 = tasks[2 * blockIdx.x + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s];
     const int we = min(w, k - j0);
+    const int nr = min(kTrsmRows, f - r0);
     const double *__restrict__ D = d.L + d.L_off[s] + (int64_t)j0 * ld + j0;
     double *__restrict__ B = d.L + d.L_off[s] + (int64_t)j0 * ld + r0;
-    const int tid = threadIdx.x;
-    for (int idx = tid; idx < kWmax * kWmax; idx += kTrsmThreads) {
-        const int i = idx & (kWmax - 1), c = idx / kWmax;
-        double v = (i == c) ? 1.0 : 0.0;
-        if (i < we && c < we && i >= c) v = D[i + (int64_t)c * ld];
-        Ls[idx] = v;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    {   // batched loads: every thread keeps 16 global loads in flight
+        const int r = tid & 63, c_base = tid >> 6;
+        double v[16];
+#pragma unroll
+        for (int t = 0; t < 16; t++) {   // L11: 64 x 64, this thread's columns c_base + 2t (+32 below)
+            const int c = c_base + 2 * t;
+            v[t] = (r < we && c < we && r >= c) ? D[r + (int64_t)c * ld] : 0.0;
+        }
+#pragma unroll
+        for (int t = 0; t < 16; t++) {
+            const int c = c_base + 2 * t;
+            Ls[r + c * kTLD] = (r == c && !(r < we)) ? 1.0 : v[t];
+        }
+#pragma unroll
+        for (int t = 0; t < 16; t++) {
+            const int c = c_base + 2 * t + 32;
+            v[t] = (r < we && c < we && r >= c) ? D[r + (int64_t)c * ld] : 0.0;
+        }
+#pragma unroll
+        for (int t = 0; t < 16; t++) {
+            const int c = c_base + 2 * t + 32;
+            Ls[r + c * kTLD] = (r == c && !(r < we)) ? 1.0 : v[t];
+        }
+#pragma unroll
+        for (int q = 0; q < kWmax / 16; q++) {
+#pragma unroll
+            for (int t = 0; t < 16; t++) {
+                const int c = q * 16 + t;
+                v[t] = (tid < nr && c < we) ? B[tid + (int64_t)c * ld] : 0.0;
+            }
+#pragma unroll
+            for (int t = 0; t < 16; t++) X[tid * kTLD + q * 16 + t] = v[t];
+        }
     }
     __syncthreads();
-    if (tid < kWmax) inv[tid] = 1.0 / Ls[tid * kWmax + tid];
-    const bool row_ok = tid < f - r0;
-    double x[kWmax];
-#pragma unroll
-    for (int c = 0; c < kWmax; c++) x[c] = (row_ok && c < we) ? B[tid + (int64_t)c * ld] : 0.0;
+    if (tid < kWmax) inv[tid] = __drcp_rn(Ls[tid + tid * kTLD]);
     __syncthreads();
-    // x L11^T = b by substitution, ascending columns (no explicit inverse of L11):
-    // x_c = (b_c - sum_{p<c} x_p L_cp) / L_cc, the sum accumulated in ascending p
+    double *Xr = X + tid * kTLD;                // this thread's row
+    const int gq = lane >> 2, tq = lane & 3;
+    double *Xw = X + (warp * 32) * kTLD;        // this warp's 32 rows
+    const int ncb = (we + 7) / 8;
 #pragma unroll
-    for (int c = 0; c < kWmax; c++) {
-        const double *Lr = Ls + c;                 // row c of L11: Ls[c + p * kWmax]
-        double acc = x[c];
+    for (int cb = 0; cb < kWmax / 8; cb++) {
+        if (cb >= ncb) break;
+        const int c0 = cb * 8;
+        double xv[8];
 #pragma unroll
-        for (int p = 0; p < c; p++) acc -= x[p] * Lr[p * kWmax];
-        x[c] = acc * inv[c];
+        for (int q = 0; q < 8; q++) xv[q] = Xr[c0 + q];
+#pragma unroll
+        for (int q = 0; q < 8; q++) {
+            xv[q] *= inv[c0 + q];
+#pragma unroll
+            for (int q2 = q + 1; q2 < 8; q2++) xv[q2] -= xv[q] * Ls[(c0 + q2) + (c0 + q) * kTLD];
+        }
+#pragma unroll
+        for (int q = 0; q < 8; q++) Xr[c0 + q] = xv[q];
+        __syncwarp();
+        // X[:, c0+8:] -= X[:, c0:c0+8] * L[c0+8:, c0:c0+8]^T  (rows of this warp)
+#pragma unroll
+        for (int nb = cb + 1; nb < kWmax / 8; nb++) {
+            if (nb >= ncb) break;
+#pragma unroll
+            for (int mb = 0; mb < 4; mb++) {
+                double *xrow = Xw + (mb * 8 + gq) * kTLD;
+                double acc0 = xrow[nb * 8 + 2 * tq], acc1 = xrow[nb * 8 + 2 * tq + 1];
+#pragma unroll
+                for (int kk = 0; kk < 2; kk++) {
+                    const double a = -xrow[c0 + kk * 4 + tq];
+                    const double b = Ls[(nb * 8 + gq) + (c0 + kk * 4 + tq) * kTLD];
+                    dmma(acc0, acc1, a, b);
+                }
+                xrow[nb * 8 + 2 * tq] = acc0;
+                xrow[nb * 8 + 2 * tq + 1] = acc1;
+            }
+        }
+        __syncwarp();
     }
-    if (row_ok) {
-#pragma unroll
-        for (int c = 0; c < kWmax; c++)
-            if (c < we) B[tid + (int64_t)c * ld] = x[c];
-    }
+    __syncthreads();
+    for (int c = 0; c < we; c++)
+        if (tid < nr) B[tid + (int64_t)c * ld] = X[tid * kTLD + c];
 }
 
 void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, cudaStream_t st) {
     if (count <= 0) return;
-    k_trsm_panel<<<(unsigned)count, kTrsmThreads, 0, st>>>(d, tasks, j0, w);
+    k_trsm_panel<<<(unsigned)count, kTrsmThreads, kTrsmSmem, st>>>(d, tasks, j0, w);
 }
 
 // ============================================================ DMMA Schur update
@@ -298,10 +427,24 @@ void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, in
 using UpdProd = UpdCfg<kTileM, kTileN, 16, 3, 2, 2, 4>;   // 29.3 TF/s on M=N=8192,K=4096 (ubench)
 
 void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, cudaStream_t st) {
-    launch_update_t<UpdProd>(d.L, d.U, probs, tiles, ntiles, st);
+    if (ntiles <= 0) return;   // attributes were set by kernels_init()
+    k_update_t<UpdProd><<<(unsigned)ntiles, UpdProd::NT, UpdProd::SMEM, st>>>(d.L, d.U, probs, tiles);
 }
 
 void launch_init_failed(int *failed, cudaStream_t st) { k_init_failed<<<1, 1, 0, st>>>(failed); }
+
+// Kernel attributes (dynamic shared memory above 48 KB), set once per device
+// before any launch -- in particular before the factorization is captured
+// into a CUDA graph.
+int kernels_init() {
+    cudaError_t e = cudaSuccess;
+    e = cudaFuncSetAttribute(k_small_front<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_trsm_panel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTrsmSmem);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_update_t<UpdProd>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)UpdProd::SMEM);
+    return e == cudaSuccess ? 0 : -1;
+}
 
 // diag(L) in final labels (one warp per supernode)
 __global__ void k_export_diag(DevPlan d, int nsuper, double *__restrict__ out) {

@@ -46,6 +46,7 @@ void launch_bsolve_init(const DevPlan &d, const int32_t *list, int count, const 
 void launch_bsolve_wave(const DevPlan &d, const int32_t *tasks, int64_t task_base, int64_t count, const int32_t *groups,
                         int j0, int w, double *y, double *partials, int *counters, cudaStream_t st);
 int small_front_smem_ok(int fmax);
+int kernels_init();
 void launch_export_diag(const DevPlan &d, int nsuper, double *out, cudaStream_t st);
 
 }  // namespace mf
