@@ -14,8 +14,8 @@
 // STAGES-deep shared-memory ring; each warp owns a TM x TN sub-tile whose
 // accumulators start from C (loaded while the first stages are in flight) and
 // accumulate C - A B^T directly (A fragments negated), so the epilogue is a
-// masked store.  Columns are 16-byte aligned (lda even); an odd starting row is
-// handled by loading one row early and shifting the shared-memory window.
+// masked store.  Columns are 16-byte aligned (lda even); problems whose first
+// row is odd are staged with 8-byte cp.async instead of 16-byte chunks.
 #pragma once
 #include <cstdint>
 
@@ -27,6 +27,11 @@ __device__ __forceinline__ void cp_async16(void *smem, const void *gmem, bool va
     const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
     const int n = valid ? 16 : 0;
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(s), "l"(gmem), "r"(n));
+}
+__device__ __forceinline__ void cp_async8(void *smem, const void *gmem, bool valid) {
+    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    const int n = valid ? 8 : 0;
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(s), "l"(gmem), "r"(n));
 }
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
 template <int N>
@@ -45,8 +50,16 @@ struct UpdCfg {
     static constexpr int NT = 32 * WARPS_M * WARPS_N;
     static constexpr int TM = BM / WARPS_M, TN = BN / WARPS_N;   // warp tile
     static constexpr int MB = TM / 8, NB = TN / 8;                // DMMA blocks per warp
-    static constexpr int SA = BM + 4, SB = BN + 4;                // +2 shifted rows, +2 pad (stride % 16 == 4)
-    static constexpr int CHA = (BM + 2) / 2, CHB = (BN + 2) / 2;  // 16-byte chunks per column
+    static constexpr int SA = BM + 4, SB = BN + 4;                // pad: stride % 16 == 4 (conflict-free fragments)
+    // operand staging: 16-byte chunks (2 rows) when the problem's first row is
+    // even, 8-byte elements otherwise; every thread keeps a fixed row slot and
+    // walks the k dimension with a fixed stride, so there is no index math in
+    // the main loop.
+    static constexpr int CPA = BM / 2, CPB = BN / 2;              // 16-byte chunks per column
+    static_assert(NT % CPA == 0 && NT % CPB == 0 && NT % BM == 0 && NT % BN == 0, "staging map");
+    static constexpr int PSA16 = NT / CPA, PSB16 = NT / CPB;      // k stride of a thread (16-byte path)
+    static constexpr int PSA8 = NT / BM, PSB8 = NT / BN;          // k stride of a thread (8-byte path)
+    static_assert(BK % PSA16 == 0 && BK % PSB16 == 0 && BK % PSA8 == 0 && BK % PSB8 == 0, "staging map");
     static constexpr int STAGE_WORDS = BK * (SA + SB);
     static constexpr size_t SMEM = (size_t)STAGES * STAGE_WORDS * sizeof(double);
     static_assert(SA % 16 == 4 && SB % 16 == 4, "bank-conflict-free fragment loads");
@@ -58,37 +71,53 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
     k_update_t(double *__restrict__ Larena, double *__restrict__ Uarena, const GemmProb *__restrict__ probs,
                const TileTask *__restrict__ tiles) {
     constexpr int BM = Cfg::BM, BN = Cfg::BN, BK = Cfg::BK, STAGES = Cfg::STAGES, NT = Cfg::NT;
-    constexpr int SA = Cfg::SA, SB = Cfg::SB, CHA = Cfg::CHA, CHB = Cfg::CHB, STAGE_WORDS = Cfg::STAGE_WORDS;
+    constexpr int SA = Cfg::SA, SB = Cfg::SB, STAGE_WORDS = Cfg::STAGE_WORDS;
     constexpr int MB = Cfg::MB, NB = Cfg::NB, TM = Cfg::TM, TN = Cfg::TN;
     extern __shared__ __align__(16) double sm[];
     const TileTask t = tiles[blockIdx.x];
     const GemmProb g = probs[t.prob];
     const int ti = t.tij >> 16, tj = t.tij & 0xffff;
     const int i0 = ti * BM, j0 = tj * BN;
-    const int sh = (int)(g.a_off & 1);
-    const double *__restrict__ A = Larena + g.a_off - sh;
+    const bool odd = (g.a_off & 1) != 0;   // columns are 16-byte aligned (even lda); rows may start odd
+    const double *__restrict__ A = Larena + g.a_off;
     const int lda = g.lda, K = g.K;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int wm = warp % Cfg::WARPS_M, wn = warp / Cfg::WARPS_M;
     const int gq = lane >> 2, tq = lane & 3;
+    // fixed staging slots of this thread
+    const int ra16 = 2 * (tid % Cfg::CPA), pa16 = tid / Cfg::CPA;
+    const int rb16 = 2 * (tid % Cfg::CPB), pb16 = tid / Cfg::CPB;
+    const int ra8 = tid % BM, pa8 = tid / BM;
+    const int rb8 = tid % BN, pb8 = tid / BN;
+    const bool oka16 = i0 + ra16 < g.M, okb16 = j0 + rb16 < g.N;   // pair (r, r+1): r+1 may run past M: harmless
+    const bool oka8 = i0 + ra8 < g.M, okb8 = j0 + rb8 < g.N;
 
     auto load_stage = [&](int stage, int kt) {
         double *As = sm + stage * STAGE_WORDS;
         double *Bs = As + BK * SA;
         const int p0 = kt * BK;
-#pragma unroll 2
-        for (int c = tid; c < BK * (CHA + CHB); c += NT) {
-            if (c < BK * CHA) {
-                const int p = c / CHA, ch = c - p * CHA;
-                const int row = i0 + 2 * ch;
-                const bool ok = (p0 + p < K) && (row - sh < g.M);
-                cp_async16(As + p * SA + 2 * ch, ok ? A + row + (int64_t)(p0 + p) * lda : A, ok);
-            } else {
-                const int cc = c - BK * CHA;
-                const int p = cc / CHB, ch = cc - p * CHB;
-                const int row = j0 + 2 * ch;
-                const bool ok = (p0 + p < K) && (row - sh < g.N);
-                cp_async16(Bs + p * SB + 2 * ch, ok ? A + row + (int64_t)(p0 + p) * lda : A, ok);
+        const double *__restrict__ Ak = A + (int64_t)p0 * lda;
+        if (!odd) {
+#pragma unroll
+            for (int p = pa16; p < BK; p += Cfg::PSA16) {
+                const bool ok = oka16 && (p0 + p < K);
+                cp_async16(As + p * SA + ra16, ok ? Ak + i0 + ra16 + (int64_t)p * lda : A, ok);
+            }
+#pragma unroll
+            for (int p = pb16; p < BK; p += Cfg::PSB16) {
+                const bool ok = okb16 && (p0 + p < K);
+                cp_async16(Bs + p * SB + rb16, ok ? Ak + j0 + rb16 + (int64_t)p * lda : A, ok);
+            }
+        } else {
+#pragma unroll
+            for (int p = pa8; p < BK; p += Cfg::PSA8) {
+                const bool ok = oka8 && (p0 + p < K);
+                cp_async8(As + p * SA + ra8, ok ? Ak + i0 + ra8 + (int64_t)p * lda : A, ok);
+            }
+#pragma unroll
+            for (int p = pb8; p < BK; p += Cfg::PSB8) {
+                const bool ok = okb8 && (p0 + p < K);
+                cp_async8(Bs + p * SB + rb8, ok ? Ak + j0 + rb8 + (int64_t)p * lda : A, ok);
             }
         }
     };
@@ -121,8 +150,8 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
             if (nk < KT) load_stage(nk % STAGES, nk);
             cp_async_commit();
         }
-        const double *As = sm + (kt % STAGES) * STAGE_WORDS + sh + wm * TM + gq;
-        const double *Bs = sm + (kt % STAGES) * STAGE_WORDS + BK * SA + sh + wn * TN + gq;
+        const double *As = sm + (kt % STAGES) * STAGE_WORDS + wm * TM + gq;
+        const double *Bs = sm + (kt % STAGES) * STAGE_WORDS + BK * SA + wn * TN + gq;
 #pragma unroll
         for (int kk = 0; kk < BK / 4; kk++) {
             double a[MB], b[NB];

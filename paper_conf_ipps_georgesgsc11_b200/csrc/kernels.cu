@@ -424,7 +424,7 @@ void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, in
 // ============================================================ DMMA Schur update
 // The production tile shape (kTileM x kTileN in mf_plan.h); variants are
 // benchmarked in tools/ubench/update_variants.cu.
-using UpdProd = UpdCfg<kTileM, kTileN, 16, 3, 2, 2, 4>;   // 29.3 TF/s on M=N=8192,K=4096 (ubench)
+using UpdProd = UpdCfg<kTileM, kTileN, 16, 3, 2, 2, 4>;   // 33.5 TF/s on M=N=8192,K=4096 (ubench, even rows)
 
 void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, cudaStream_t st) {
     if (ntiles <= 0) return;   // attributes were set by kernels_init()
