@@ -34,6 +34,20 @@ __device__ __forceinline__ void note_pivot(const DevPlan &d, double djj, int col
 
 __global__ void k_init_failed(int *failed) { *failed = INT_MAX; }
 
+// 1/sqrt(x) for a pivot: float MUFU seed + two fp64 Newton steps (~1 ulp; exactly
+// 2^-p for x = 4^p, so the manufactured integer factors stay exact).  Outside the
+// float range (or for x <= 0 / NaN) it falls back to the library rsqrt.
+__device__ __forceinline__ double pivot_rsqrt(double x) {
+    if (!(x > 1e-30 && x < 1e30)) return rsqrt(x);
+    double y = (double)rsqrtf((float)x);
+    double h = x * y;
+    double r = fma(-h, y, 1.0);
+    y = fma(0.5 * y, r, y);
+    h = x * y;
+    r = fma(-h, y, 1.0);
+    return fma(0.5 * y, r, y);
+}
+
 // ============================================================ small fronts
 // One CTA per front; the whole f x f front lives in shared memory (column-major,
 // leading dimension f).  Assembly, potrf, trsm and the syrk on U^n are fused:
@@ -314,66 +328,62 @@ void launch_potrf_diag(const DevPlan &d, const int32_t *fronts, int count, int j
 // matrix which spans both L1 and L2").  Substitution order
 // (ascending columns), no explicit inverse: integer-exact on manufactured inputs.
 constexpr int kTrsmThreads = kTrsmRows;   // 4 warps, each owning 32 rows
-constexpr int kTLD = kWmax + 1;             // smem leading dimension (odd: row-per-thread access is conflict-free)
-constexpr size_t kTrsmSmem = (size_t)(kWmax * kTLD + kTrsmRows * kTLD + kWmax) * sizeof(double);
+constexpr int kLLD = kWmax + 2;             // L11 smem: column-major, even stride (16-byte cp.async)
+constexpr int kXLD = kTrsmRows + 2;         // X smem: column-major, even stride
+constexpr size_t kTrsmSmem = (size_t)(kWmax * kLLD + kWmax * kXLD + kWmax) * sizeof(double);
 // X L11^T = B by blocked substitution: for each 8-column block, every thread
 // solves its own row over the block (scalar), then its warp applies the block
 // to the remaining columns of its 32 rows with DMMA (m8n8k4 f64).  Warps never
 // share rows, so only warp-level synchronisation is needed.  No explicit
-// inverse of L11: integer-exact on the manufactured inputs.
+// inverse of L11: integer-exact on the manufactured inputs.  L11 and the row
+// block are staged with cp.async (all loads in flight at once).
 __global__ void __launch_bounds__(kTrsmThreads, 2) k_trsm_panel(DevPlan d, const int32_t *__restrict__ tasks,
                                                                 int j0, int w) {
-    extern __shared__ double tsm[];
-    double *Ls = tsm;                           // L11, column-major [row + col * kTLD], identity-padded
-    double *X = tsm + kWmax * kTLD;             // rows x 64, row-major [row * kTLD + col]
-    double *inv = X + kTrsmRows * kTLD;
+    extern __shared__ __align__(16) double tsm[];
+    double *Ls = tsm;                           // L11[r][c] at Ls[r + c * kLLD]
+    double *X = tsm + kWmax * kLLD;             // X[r][c]   at X[r + c * kXLD]
+    double *inv = X + kWmax * kXLD;
     const int s = tasks[2 * blockIdx.x], r0 = tasks[2 * blockIdx.x + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s];
     const int we = min(w, k - j0);
     const int nr = min(kTrsmRows, f - r0);
-    const double *__restrict__ D = d.L + d.L_off[s] + (int64_t)j0 * ld + j0;
+    const double *__restrict__ D = d.L + d.L_off[s] + (int64_t)j0 * ld + j0;   // 16B aligned: j0 even, ld even
     double *__restrict__ B = d.L + d.L_off[s] + (int64_t)j0 * ld + r0;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    {   // batched loads: every thread keeps 16 global loads in flight
-        const int r = tid & 63, c_base = tid >> 6;
-        double v[16];
-#pragma unroll
-        for (int t = 0; t < 16; t++) {   // L11: 64 x 64, this thread's columns c_base + 2t (+32 below)
-            const int c = c_base + 2 * t;
-            v[t] = (r < we && c < we && r >= c) ? D[r + (int64_t)c * ld] : 0.0;
+    // L11: 64 x we, pairs of rows per 16-byte chunk (rows >= we padded below)
+    for (int q = tid; q < (kWmax / 2) * kWmax; q += kTrsmThreads) {
+        const int rr = 2 * (q % (kWmax / 2)), c = q / (kWmax / 2);
+        const bool ok = c < we && rr < we;
+        cp_async16(Ls + rr + c * kLLD, ok ? D + rr + (int64_t)c * ld : D, ok);
+    }
+    if ((r0 & 1) == 0) {
+        for (int q = tid; q < (kTrsmRows / 2) * kWmax; q += kTrsmThreads) {
+            const int rr = 2 * (q % (kTrsmRows / 2)), c = q / (kTrsmRows / 2);
+            const bool ok = c < we && rr < nr;
+            cp_async16(X + rr + c * kXLD, ok ? B + rr + (int64_t)c * ld : B, ok);
         }
-#pragma unroll
-        for (int t = 0; t < 16; t++) {
-            const int c = c_base + 2 * t;
-            Ls[r + c * kTLD] = (r == c && !(r < we)) ? 1.0 : v[t];
+    } else {
+        for (int c = 0; c < kWmax; c++) {
+            const bool ok = c < we && tid < nr;
+            cp_async8(X + tid + c * kXLD, ok ? B + tid + (int64_t)c * ld : B, ok);
         }
-#pragma unroll
-        for (int t = 0; t < 16; t++) {
-            const int c = c_base + 2 * t + 32;
-            v[t] = (r < we && c < we && r >= c) ? D[r + (int64_t)c * ld] : 0.0;
-        }
-#pragma unroll
-        for (int t = 0; t < 16; t++) {
-            const int c = c_base + 2 * t + 32;
-            Ls[r + c * kTLD] = (r == c && !(r < we)) ? 1.0 : v[t];
-        }
-#pragma unroll
-        for (int q = 0; q < kWmax / 16; q++) {
-#pragma unroll
-            for (int t = 0; t < 16; t++) {
-                const int c = q * 16 + t;
-                v[t] = (tid < nr && c < we) ? B[tid + (int64_t)c * ld] : 0.0;
-            }
-#pragma unroll
-            for (int t = 0; t < 16; t++) X[tid * kTLD + q * 16 + t] = v[t];
+    }
+    cp_async_commit();
+    cp_async_wait<0>();
+    __syncthreads();
+    // identity padding of L11 beyond we (rows/cols); strict upper part is never read
+    if (tid < kWmax) {
+        if (tid >= we) {
+            for (int c = 0; c < kWmax; c++) Ls[tid + c * kLLD] = (c == tid) ? 1.0 : 0.0;
+        } else {
+            for (int c = we; c < kWmax; c++) Ls[tid + c * kLLD] = 0.0;
         }
     }
     __syncthreads();
-    if (tid < kWmax) inv[tid] = __drcp_rn(Ls[tid + tid * kTLD]);
+    if (tid < kWmax) inv[tid] = __drcp_rn(Ls[tid + tid * kLLD]);
     __syncthreads();
-    double *Xr = X + tid * kTLD;                // this thread's row
     const int gq = lane >> 2, tq = lane & 3;
-    double *Xw = X + (warp * 32) * kTLD;        // this warp's 32 rows
+    double *Xw = X + warp * 32;                 // this warp's 32 rows
     const int ncb = (we + 7) / 8;
 #pragma unroll
     for (int cb = 0; cb < kWmax / 8; cb++) {
@@ -381,15 +391,15 @@ __global__ void __launch_bounds__(kTrsmThreads, 2) k_trsm_panel(DevPlan d, const
         const int c0 = cb * 8;
         double xv[8];
 #pragma unroll
-        for (int q = 0; q < 8; q++) xv[q] = Xr[c0 + q];
+        for (int q = 0; q < 8; q++) xv[q] = X[tid + (c0 + q) * kXLD];
 #pragma unroll
         for (int q = 0; q < 8; q++) {
             xv[q] *= inv[c0 + q];
 #pragma unroll
-            for (int q2 = q + 1; q2 < 8; q2++) xv[q2] -= xv[q] * Ls[(c0 + q2) + (c0 + q) * kTLD];
+            for (int q2 = q + 1; q2 < 8; q2++) xv[q2] -= xv[q] * Ls[(c0 + q2) + (c0 + q) * kLLD];
         }
 #pragma unroll
-        for (int q = 0; q < 8; q++) Xr[c0 + q] = xv[q];
+        for (int q = 0; q < 8; q++) X[tid + (c0 + q) * kXLD] = xv[q];
         __syncwarp();
         // X[:, c0+8:] -= X[:, c0:c0+8] * L[c0+8:, c0:c0+8]^T  (rows of this warp)
 #pragma unroll
@@ -397,23 +407,23 @@ __global__ void __launch_bounds__(kTrsmThreads, 2) k_trsm_panel(DevPlan d, const
             if (nb >= ncb) break;
 #pragma unroll
             for (int mb = 0; mb < 4; mb++) {
-                double *xrow = Xw + (mb * 8 + gq) * kTLD;
-                double acc0 = xrow[nb * 8 + 2 * tq], acc1 = xrow[nb * 8 + 2 * tq + 1];
+                double *xr = Xw + mb * 8 + gq;
+                double acc0 = xr[(nb * 8 + 2 * tq) * kXLD], acc1 = xr[(nb * 8 + 2 * tq + 1) * kXLD];
 #pragma unroll
                 for (int kk = 0; kk < 2; kk++) {
-                    const double a = -xrow[c0 + kk * 4 + tq];
-                    const double b = Ls[(nb * 8 + gq) + (c0 + kk * 4 + tq) * kTLD];
+                    const double a = -xr[(c0 + kk * 4 + tq) * kXLD];
+                    const double b = Ls[(nb * 8 + gq) + (c0 + kk * 4 + tq) * kLLD];
                     dmma(acc0, acc1, a, b);
                 }
-                xrow[nb * 8 + 2 * tq] = acc0;
-                xrow[nb * 8 + 2 * tq + 1] = acc1;
+                xr[(nb * 8 + 2 * tq) * kXLD] = acc0;
+                xr[(nb * 8 + 2 * tq + 1) * kXLD] = acc1;
             }
         }
         __syncwarp();
     }
     __syncthreads();
     for (int c = 0; c < we; c++)
-        if (tid < nr) B[tid + (int64_t)c * ld] = X[tid * kTLD + c];
+        if (tid < nr) B[tid + (int64_t)c * ld] = X[tid + c * kXLD];
 }
 
 void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, cudaStream_t st) {
