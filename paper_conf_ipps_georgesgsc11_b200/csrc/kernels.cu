@@ -48,80 +48,144 @@ __device__ __forceinline__ double pivot_rsqrt(double x) {
     return fma(0.5 * y, r, y);
 }
 
+// ============================================================ shared building block
+// Factor the nb x nb diagonal sub-block A[s0:s0+nb, s0:s0+nb] (nb <= 16,
+// column-major, leading dimension lda, already updated) in the registers of the
+// calling warp: lane l < 16 owns row s0+l, pivots are broadcast by shuffles, so
+// the pivot chain needs no block barrier.  Writes L back to A (and to gP, if
+// given), 1/L_jj to sinv[s0+j], and flags non-positive pivots (reading C8).
+__device__ __forceinline__ void warp_factor16(double *A, int lda, int s0, int nb, double *sinv, const DevPlan &d,
+                                              int first_col, double *__restrict__ gP, int64_t gld) {
+    const int lane = threadIdx.x & 31, l = lane & 15;
+    double a[16];
+#pragma unroll
+    for (int q = 0; q < 16; q++) a[q] = (q <= l && l < nb) ? A[(s0 + q) * lda + s0 + l] : 0.0;
+#pragma unroll
+    for (int q = 0; q < 16; q++) {
+        if (q < nb) {
+            const double dq = __shfl_sync(0xffffffffu, a[q], q);
+            const double inv = rsqrt(dq);
+            const double piv = dq * inv;
+            if (lane == q) {
+                note_pivot(d, dq, first_col + q);
+                sinv[s0 + q] = inv;
+                a[q] = piv;
+            } else if (l > q) {
+                a[q] *= inv;
+            }
+#pragma unroll
+            for (int c = q + 1; c < 16; c++) {
+                const double lc = __shfl_sync(0xffffffffu, a[q], c);
+                if (l >= c) a[c] -= a[q] * lc;
+            }
+        }
+    }
+    if (lane < nb) {
+#pragma unroll
+        for (int q = 0; q < 16; q++)
+            if (q <= lane) {
+                A[(s0 + q) * lda + s0 + lane] = a[q];
+                if (gP) gP[(s0 + lane) + (s0 + q) * gld] = a[q];
+            }
+    }
+}
+
 // ============================================================ small fronts
 // One CTA per front; the whole f x f front lives in shared memory (column-major,
-// leading dimension f).  Assembly, potrf, trsm and the syrk on U^n are fused:
-// the k pivot columns are eliminated right-looking, which produces L1, L2 and
-// U^n = F22 - L2 L2^T in place.  Writes the L panel and U^n to HBM.
+// leading dimension f).  Assembly (zero, A entries, extend-add of the children
+// in ascending order), then the F-U step on the k pivot columns in blocks of
+// 16: the diagonal sub-block in the registers of warp 0, the rows below it one
+// thread per row (substitution), and the rank-16 update of the trailing lower
+// triangle (which includes U^n = F22 - L2 L2^T).  Writes the L panel and U^n.
 template <int NT>
 __global__ void __launch_bounds__(NT) k_small_front(DevPlan d, const int32_t *__restrict__ list,
                                                     const double *__restrict__ values) {
     extern __shared__ double F[];
+    constexpr int NW = NT / 32;
+    constexpr int RP = NT < 128 ? NT : 128;   // rows per pass of the trailing update
+    constexpr int H = NT / RP;                // column groups
     const int s = list[blockIdx.x];
     const int k = d.sn_k[s], f = d.sn_f[s], m = f - k, first = d.sn_first[s];
-    const int tid = threadIdx.x;
+    double *sinv = F + f * f;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     for (int i = tid; i < f * f; i += NT) F[i] = 0.0;
     __syncthreads();
-    // A entries of the k pivot columns: warp per column, lanes over entries
-    {
-        const int warp = tid >> 5, lane = tid & 31;
-        for (int j = warp; j < k; j += NT / 32) {
-            const int64_t e0 = d.bcolptr[first + j], e1 = d.bcolptr[first + j + 1];
-            for (int64_t e = e0 + lane; e < e1; e += 32) F[d.blrow[e] + j * f] = sum_values(d, values, e);
-        }
+    for (int j = warp; j < k; j += NW) {        // A entries: warp per column
+        const int64_t e0 = d.bcolptr[first + j], e1 = d.bcolptr[first + j + 1];
+        for (int64_t e = e0 + lane; e < e1; e += 32) F[d.blrow[e] + j * f] = sum_values(d, values, e);
     }
     __syncthreads();
-    // extend-add of the children's U^c, ascending child order
-    for (int q = d.child_ptr[s]; q < d.child_ptr[s + 1]; q++) {
+    for (int q = d.child_ptr[s]; q < d.child_ptr[s + 1]; q++) {   // extend-add, ascending children
         const int c = d.child_list[q];
         const int mc = d.sn_f[c] - d.sn_k[c];
         const int32_t *__restrict__ rel = d.relmap + d.relmap_ptr[c];
         const double *__restrict__ Uc = d.U + d.U_off[c];
-        for (int idx = tid; idx < mc * mc; idx += NT) {
-            const int p = idx % mc, qq = idx / mc;
-            if (p >= qq) F[rel[p] + rel[qq] * f] += Uc[idx];
+        for (int qq = warp; qq < mc; qq += NW) {
+            double *dst = F + rel[qq] * f;
+            const double *ucol = Uc + qq * mc;
+            for (int p = qq + lane; p < mc; p += 32) dst[rel[p]] += ucol[p];
         }
         __syncthreads();
     }
-    // right-looking elimination of the k pivot columns over the whole front
-    for (int j = 0; j < k; j++) {
-        const double djj = F[j + j * f];
-        const double piv = sqrt(djj);
-        for (int i = j + 1 + tid; i < f; i += NT) F[i + j * f] /= piv;
+    for (int s0 = 0; s0 < k; s0 += 16) {
+        const int nb = min(16, k - s0);
+        if (warp == 0) warp_factor16(F, f, s0, nb, sinv, d, first + s0, nullptr, 0);
         __syncthreads();
-        if (tid == 0) {
-            note_pivot(d, djj, first + j);
-            F[j + j * f] = piv;
+        const int r0 = s0 + nb;
+        if (r0 >= f) break;
+        for (int r = r0 + tid; r < f; r += NT) {   // rows below: x L_sub^T = a
+            double x[16];
+#pragma unroll
+            for (int q = 0; q < 16; q++) x[q] = q < nb ? F[r + (s0 + q) * f] : 0.0;
+#pragma unroll
+            for (int q = 0; q < 16; q++) {
+                if (q < nb) {
+                    x[q] *= sinv[s0 + q];
+#pragma unroll
+                    for (int q2 = q + 1; q2 < 16; q2++)
+                        if (q2 < nb) x[q2] -= x[q] * F[(s0 + q2) + (s0 + q) * f];
+                }
+            }
+#pragma unroll
+            for (int q = 0; q < 16; q++)
+                if (q < nb) F[r + (s0 + q) * f] = x[q];
         }
-        const int nr = f - j - 1;
-        for (int idx = tid; idx < nr * nr; idx += NT) {
-            const int i = j + 1 + idx % nr, c = j + 1 + idx / nr;
-            if (i >= c) F[i + c * f] -= F[i + j * f] * F[c + j * f];
+        __syncthreads();
+        // trailing update, rows/cols [r0, f): F[i][c] -= sum_q L[i][q] L[c][q]
+        for (int i = r0 + (tid % RP), h = tid / RP; i < f; i += RP) {
+            {
+                double li[16];
+#pragma unroll
+                for (int q = 0; q < 16; q++) li[q] = q < nb ? F[i + (s0 + q) * f] : 0.0;
+                for (int c = r0 + h; c <= i; c += H) {
+                    double acc = F[i + c * f];
+#pragma unroll
+                    for (int q = 0; q < 16; q++)
+                        if (q < nb) acc -= li[q] * F[c + (s0 + q) * f];
+                    F[i + c * f] = acc;
+                }
+            }
         }
         __syncthreads();
     }
     // write the L panel (upper triangle of L1 = 0) and U^n (lower triangle)
     double *__restrict__ P = d.L + d.L_off[s];
     const int ld = d.sn_ld[s];
-    for (int idx = tid; idx < f * k; idx += NT) {
-        const int i = idx % f, j = idx / f;
-        P[i + (int64_t)j * ld] = i >= j ? F[i + j * f] : 0.0;
-    }
+    for (int j = warp; j < k; j += NW)
+        for (int i = lane; i < f; i += 32) P[i + (int64_t)j * ld] = i >= j ? F[i + j * f] : 0.0;
     if (m > 0) {
         double *__restrict__ Us = d.U + d.U_off[s];
-        for (int idx = tid; idx < m * m; idx += NT) {
-            const int i = idx % m, c = idx / m;
-            if (i >= c) Us[idx] = F[(k + i) + (k + c) * f];
-        }
+        for (int c = warp; c < m; c += NW)
+            for (int i = c + lane; i < m; i += 32) Us[i + c * m] = F[(k + i) + (k + c) * f];
     }
 }
 
-int small_front_smem_ok(int fmax) { return (size_t)fmax * fmax * sizeof(double) <= 227 * 1024; }
+int small_front_smem_ok(int fmax) { return (size_t)(fmax * fmax + fmax) * sizeof(double) <= 227 * 1024; }
 
 void launch_small_fronts(const DevPlan &d, const int32_t *list, int count, int fmax, const double *values,
                          cudaStream_t st) {
     if (count <= 0) return;
-    const size_t smem = (size_t)fmax * fmax * sizeof(double);
+    const size_t smem = (size_t)(fmax * fmax + fmax) * sizeof(double);
     if (fmax <= 32) {
         k_small_front<64><<<count, 64, smem, st>>>(d, list, values);
     } else if (fmax <= 64) {
@@ -135,22 +199,53 @@ void launch_small_fronts(const DevPlan &d, const int32_t *list, int count, int f
 // Task = (front s, first local column c0): columns [c0, c0+32) of the front.
 // Columns < k live in the L panel, columns >= k in U^s.
 constexpr int kAsmThreads = 256;
+constexpr int kAsmChunk = 512;   // rows per shared-memory staging chunk (per warp)
 // Each warp owns whole destination columns (round-robin over the task's 32
-// columns): it zeroes a column, writes its A entries, then adds the matching
-// column of every child's U^c in ascending child order.  Because one warp
-// performs every write to its columns, the order is fixed without barriers or
-// atomics.  The child column that lands in destination column c is found by
-// binary search in the child's (increasing) relative map.
+// columns) and builds each column chunk by chunk in shared memory: zero, its A
+// entries, then every child's matching U^c column in ascending child order --
+// and writes the finished chunk to HBM once.  One warp performs every update of
+// its entries, so the summation order (0 + A + U^c1 + U^c2 + ...) is fixed
+// without barriers or atomics, and the destination is written exactly once
+// (no zero-fill pass, no read-modify-write).  Child column q lands in
+// destination column c iff rel[q] == c (rel is increasing: binary search); its
+// rows falling in a chunk are a contiguous range of rel.
+__device__ __forceinline__ int lower_bound_rel(const int32_t *__restrict__ rel, int lo, int hi, int key) {
+    while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        if (__ldg(rel + mid) < key) lo = mid + 1; else hi = mid;
+    }
+    return lo;
+}
+
+constexpr int kAsmMaxCh = 32;   // children handled through the shared column map (more: searched per column)
 __global__ void __launch_bounds__(kAsmThreads) k_assemble(DevPlan d, const int32_t *__restrict__ tasks,
                                                           const double *__restrict__ values) {
+    constexpr int NW = kAsmThreads / 32;
+    __shared__ double sbuf[NW][kAsmChunk];
+    __shared__ int colmap[kAsmMaxCh][kAsmCols];   // child column landing in column c0 + x, or -1
+    __shared__ int s_cp[NW][kAsmMaxCh];           // per warp and child: next child row to add
     const int s = tasks[2 * blockIdx.x], c0 = tasks[2 * blockIdx.x + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], m = f - k, ld = d.sn_ld[s], first = d.sn_first[s];
     const int c1 = min(c0 + kAsmCols, f);
     double *__restrict__ P = d.L + d.L_off[s];
     double *__restrict__ Us = d.U + d.U_off[s];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    constexpr int NW = kAsmThreads / 32;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    double *buf = sbuf[warp];
+    int *cp = s_cp[warp];
     const int q0 = d.child_ptr[s], q1 = d.child_ptr[s + 1];
+    const int nch = q1 - q0, nmap = min(nch, kAsmMaxCh);
+    // column map: the child columns q with rel[q] in [c0, c1) form one contiguous range per child
+    for (int i = tid; i < nmap * kAsmCols; i += kAsmThreads) colmap[i / kAsmCols][i % kAsmCols] = -1;
+    __syncthreads();
+    for (int j = warp; j < nmap; j += NW) {
+        const int ch = d.child_list[q0 + j];
+        const int mc = d.sn_f[ch] - d.sn_k[ch];
+        const int32_t *__restrict__ rel = d.relmap + d.relmap_ptr[ch];
+        const int qa = lower_bound_rel(rel, 0, mc, c0);
+        const int qb = lower_bound_rel(rel, qa, mc, c1);
+        for (int q = qa + lane; q < qb; q += 32) colmap[j][__ldg(rel + q) - c0] = q;
+    }
+    __syncthreads();
     for (int c = c0 + warp; c < c1; c += NW) {
         // destination column: panel column c (rows 0..f-1) or U column c-k (rows c..f-1)
         double *__restrict__ col;
@@ -162,36 +257,62 @@ __global__ void __launch_bounds__(kAsmThreads) k_assemble(DevPlan d, const int32
             col = Us + (int64_t)(c - k) * m - k;   // index by front row r >= c
             rlo = c;
         }
-        for (int r = rlo + lane; r < f; r += 32) col[r] = 0.0;
+        if (lane < nmap) cp[lane] = colmap[lane][c - c0];   // rel[qc] = c >= rlo: start at the diagonal
         __syncwarp();
-        if (c < k) {
-            const int64_t e0 = d.bcolptr[first + c], e1 = d.bcolptr[first + c + 1];
-            for (int64_t e = e0 + lane; e < e1; e += 32) col[d.blrow[e]] = sum_values(d, values, e);
+        const int64_t e0 = c < k ? d.bcolptr[first + c] : 0, e1 = c < k ? d.bcolptr[first + c + 1] : 0;
+        for (int r0 = rlo; r0 < f; r0 += kAsmChunk) {
+            const int r1 = min(r0 + kAsmChunk, f);
+            for (int r = r0 + lane; r < r1; r += 32) buf[r - r0] = 0.0;
             __syncwarp();
-        }
-        for (int q = q0; q < q1; q++) {
-            const int ch = d.child_list[q];
-            const int mc = d.sn_f[ch] - d.sn_k[ch];
-            const int32_t *__restrict__ rel = d.relmap + d.relmap_ptr[ch];
-            int lo = 0, hi = mc;
-            while (lo < hi) {
-                const int mid = (lo + hi) >> 1;
-                if (__ldg(rel + mid) < c) lo = mid + 1; else hi = mid;
+            for (int64_t e = e0 + lane; e < e1; e += 32) {
+                const int r = d.blrow[e];
+                if (r >= r0 && r < r1) buf[r - r0] = sum_values(d, values, e);
             }
-            if (lo >= mc || __ldg(rel + lo) != c) continue;
-            const double *__restrict__ ucol = d.U + d.U_off[ch] + (int64_t)lo * mc;
-            int p = lo + lane;
-            for (; p + 96 < mc; p += 128) {   // 4 independent gathers in flight per lane
-                const int r0 = __ldg(rel + p), r1 = __ldg(rel + p + 32), r2 = __ldg(rel + p + 64), r3 = __ldg(rel + p + 96);
-                const double u0 = __ldg(ucol + p), u1 = __ldg(ucol + p + 32), u2 = __ldg(ucol + p + 64),
-                             u3 = __ldg(ucol + p + 96);
-                const double v0 = col[r0], v1 = col[r1], v2 = col[r2], v3 = col[r3];
-                col[r0] = v0 + u0;
-                col[r1] = v1 + u1;
-                col[r2] = v2 + u2;
-                col[r3] = v3 + u3;
+            __syncwarp();
+            for (int j = 0; j < nch; j++) {
+                const int ch = d.child_list[q0 + j];
+                const int mc = d.sn_f[ch] - d.sn_k[ch];
+                const int32_t *__restrict__ rel = d.relmap + d.relmap_ptr[ch];
+                int qc, p;
+                if (j < kAsmMaxCh) {
+                    qc = colmap[j][c - c0];
+                    if (qc < 0) continue;
+                    p = cp[j];
+                } else {   // rare: more children than the map holds
+                    qc = lower_bound_rel(rel, 0, mc, c);
+                    if (qc >= mc || __ldg(rel + qc) != c) continue;
+                    p = lower_bound_rel(rel, qc, mc, r0);
+                }
+                const double *__restrict__ ucol = d.U + d.U_off[ch] + (int64_t)qc * mc;
+                // consume child rows p, p+1, ... while rel < r1 (rel is increasing): 256 rows per
+                // step (8 loads of each kind in flight per lane), the stop found by warp ballots
+                while (p < mc) {
+                    int rr[8];
+                    double uu[8];
+#pragma unroll
+                    for (int t = 0; t < 8; t++) {
+                        const int idx = p + 32 * t + lane;
+                        rr[t] = idx < mc ? __ldg(rel + idx) : INT_MAX;
+                        uu[t] = idx < mc ? __ldg(ucol + idx) : 0.0;
+                    }
+                    int taken = 0;
+                    bool stop = false;
+#pragma unroll
+                    for (int t = 0; t < 8; t++) {
+                        const bool in = rr[t] < r1;
+                        if (in) buf[rr[t] - r0] += uu[t];
+                        const int n_in = __popc(__ballot_sync(0xffffffffu, in));
+                        if (!stop) taken += n_in;
+                        stop = stop || n_in < 32;
+                    }
+                    p += taken;
+                    if (stop) break;
+                }
+                __syncwarp();
+                if (j < kAsmMaxCh && lane == 0) cp[j] = p;
             }
-            for (; p < mc; p += 32) col[__ldg(rel + p)] += __ldg(ucol + p);
+            __syncwarp();
+            for (int r = r0 + lane; r < r1; r += 32) col[r] = buf[r - r0];
             __syncwarp();
         }
     }
@@ -242,40 +363,7 @@ __global__ void __launch_bounds__(kPotrfThreads) k_potrf_diag(DevPlan d, const i
     for (int s0 = 0; s0 < we; s0 += 16) {
         const int nb = min(16, we - s0);
         // (a) 16 x 16 diagonal sub-block in registers of warp 0
-        if (warp == 0) {
-            const int l = lane & 15;
-            double a[16];
-#pragma unroll
-            for (int q = 0; q < 16; q++) a[q] = (q <= l && l < nb) ? A[(s0 + q) * LDA + s0 + l] : 0.0;
-#pragma unroll
-            for (int q = 0; q < 16; q++) {
-                if (q < nb) {
-                    const double dq = __shfl_sync(0xffffffffu, a[q], q);
-                    const double inv = rsqrt(dq);
-                    const double piv = dq * inv;
-                    if (lane == q) {
-                        note_pivot(d, dq, first + j0 + s0 + q);
-                        sinv[s0 + q] = inv;
-                        a[q] = piv;
-                    } else if (l > q) {
-                        a[q] *= inv;
-                    }
-#pragma unroll
-                    for (int c = q + 1; c < 16; c++) {
-                        const double lc = __shfl_sync(0xffffffffu, a[q], c);
-                        if (l >= c) a[c] -= a[q] * lc;
-                    }
-                }
-            }
-            if (lane < nb) {
-#pragma unroll
-                for (int q = 0; q < 16; q++)
-                    if (q <= lane) {
-                        A[(s0 + q) * LDA + s0 + lane] = a[q];
-                        P[(s0 + lane) + (int64_t)(s0 + q) * ld] = a[q];
-                    }
-            }
-        }
+        if (warp == 0) warp_factor16(A, LDA, s0, nb, sinv, d, first + j0 + s0, P, ld);
         __syncthreads();
         const int r0 = s0 + 16;
         if (r0 >= we) break;

@@ -128,7 +128,7 @@ struct Plan {
 };
 
 constexpr int kTileM = 64, kTileN = 64;
-constexpr int kAsmCols = 32;
+constexpr int kAsmCols = 16;
 constexpr int kTrsmRows = 128;
 constexpr int kSmallClasses = 3;
 constexpr int kSolveRows = 256;
