@@ -67,6 +67,8 @@ typedef struct {
     int32_t device;           /* CUDA device ordinal (-1 = current)                                */
     int32_t host_only;        /* 1 = symbolic analysis + planning only, no device (mf_factor/mf_solve
                                  then return MF_ERR_STATE); lets CPU-only hosts inspect the plan   */
+    int32_t nranks;           /* GPUs (one process each) sharing the factorization (default 1)     */
+    int32_t rank;             /* this process's rank in [0, nranks)                                 */
     void *stream;             /* cudaStream_t to run on (NULL = the ctx creates its own)           */
 } mf_options;
 
@@ -103,6 +105,29 @@ typedef struct {
 } mf_kernel_stat;
 
 #define MF_KERNEL_CLASSES 5
+
+/* Multi-GPU exchange.  With nranks > 1 every rank passes the
+ * same n/colptr/rowind/perm/values/b; elimination subtrees are mapped to ranks and
+ * the supernodes above them ("top") are factored by rank 0.  The library hands
+ * the data movement to a caller-supplied callback (NCCL through torch.distributed
+ * in the Python binding), called by every rank with matching lists:
+ *   SEND/RECV  point-to-point, `peer` = the other rank;
+ *   BCAST      in place, root = `peer`;
+ *   ALLREDUCE_SUM (float64) / ALLREDUCE_MIN_I32 (int32), in place.
+ * Buffers are device pointers; the ctx stream is synchronized before the call and
+ * the callback must return only when the transfers are complete (0 = success). */
+#define MF_XFER_SEND 1
+#define MF_XFER_RECV 2
+#define MF_XFER_BCAST 3
+#define MF_XFER_ALLREDUCE_SUM 4
+#define MF_XFER_ALLREDUCE_MIN_I32 5
+typedef struct {
+    int32_t op;
+    int32_t peer;
+    void *ptr;
+    int64_t bytes;
+} mf_xfer;
+typedef int (*mf_exchange_fn)(void *user, const mf_xfer *ops, int64_t nops);
 
 /* Fill *opt with the defaults. */
 int mf_default_options(mf_options *opt);
@@ -164,6 +189,15 @@ typedef struct {
 
 /* out may be NULL to query *count only. */
 int mf_get_program(const mf_ctx *ctx, mf_launch_info *out, int64_t max, int64_t *count);
+
+/* Register the exchange callback (required before mf_factor when nranks > 1). */
+int mf_set_exchange(mf_ctx *ctx, mf_exchange_fn fn, void *user);
+
+/* Subtree-to-GPU mapping of the analyzed pattern: owner[nsuper] (rank factoring
+ * each supernode) and top[nsuper] (1 = factored by rank 0 after the exchange).
+ * rank_load[nranks] = executed flops of each rank's subtrees; *top_load = flops
+ * of the top.  Any pointer may be NULL. */
+int mf_get_mapping(const mf_ctx *ctx, int32_t *owner, int8_t *top, double *rank_load, double *top_load);
 
 /* Enable (1) / disable (0) per-launch CUDA-event timing in mf_factor; resets the stats. */
 int mf_set_profiling(mf_ctx *ctx, int enable);

@@ -50,8 +50,12 @@ struct mf_ctx {
     int64_t launches = 0;
     bool profiling = false;
     bool use_graph = true;
-    cudaGraph_t graph = nullptr;
-    cudaGraphExec_t graph_exec = nullptr;
+    cudaGraph_t graph = nullptr, graph_top = nullptr;
+    cudaGraphExec_t graph_exec = nullptr, graph_top_exec = nullptr;
+    mf_exchange_fn xfn = nullptr;
+    void *xuser = nullptr;
+    double *d_ytmp = nullptr;
+    int32_t *d_top_list = nullptr, *d_own_list = nullptr;
     std::vector<cudaEvent_t> prof_events;
     mf_kernel_stat kstats[KC_COUNT];
     int64_t prof_factors = 0;
@@ -93,8 +97,12 @@ int dev_alloc(mf_ctx *c, void **dst, size_t bytes) {
 void drop_graph(mf_ctx *c) {
     if (c->graph_exec) cudaGraphExecDestroy(c->graph_exec);
     if (c->graph) cudaGraphDestroy(c->graph);
+    if (c->graph_top_exec) cudaGraphExecDestroy(c->graph_top_exec);
+    if (c->graph_top) cudaGraphDestroy(c->graph_top);
     c->graph_exec = nullptr;
     c->graph = nullptr;
+    c->graph_top_exec = nullptr;
+    c->graph_top = nullptr;
 }
 
 void free_device(mf_ctx *c) {
@@ -167,6 +175,9 @@ int mf_default_options(mf_options *o) {
     o->small_front_max = d.small_front_max;
     o->panel_w = d.panel_w;
     o->device = -1;
+    o->host_only = 0;
+    o->nranks = 1;
+    o->rank = 0;
     o->stream = nullptr;
     return MF_OK;
 }
@@ -188,6 +199,12 @@ int mf_create(mf_ctx **out, const mf_options *o) {
     }
     c->opt.small_front_max = o->small_front_max;
     c->opt.panel_w = o->panel_w;
+    if (o->nranks < 1 || o->rank < 0 || o->rank >= o->nranks) {
+        delete c;
+        return MF_ERR_ARG;
+    }
+    c->opt.nranks = o->nranks;
+    c->opt.rank = o->rank;
     c->host_only = o->host_only != 0;
     c->info.failed_col = -1;
     if (c->host_only) {   // symbolic analysis + plan only; never touches CUDA
@@ -297,6 +314,8 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     UP(&c->d_sf_tasks, P.sf_tasks);
     UP(&c->d_sb_tasks, P.sb_tasks);
     UP(&c->d_sb_groups, P.sb_groups);
+    UP(&c->d_top_list, P.top_list);
+    UP(&c->d_own_list, P.own_list);
 #undef UP
     d.sn_first = sn_first;
     d.sn_k = sn_k;
@@ -333,6 +352,8 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(n, 1) * sizeof(double))) != MF_OK) return r;
     c->d_y = (double *)p;
     if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(n, 1) * sizeof(double))) != MF_OK) return r;
+    c->d_ytmp = (double *)p;
+    if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(n, 1) * sizeof(double))) != MF_OK) return r;
     c->d_bx = (double *)p;
     // the L arena starts zeroed once so that never-written padding words are defined
     CK(cudaMemsetAsync(d.L, 0, P.L_words * sizeof(double), c->stream));
@@ -345,31 +366,21 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     return MF_OK;
 }
 
-int mf_factor(mf_ctx *c, const double *values) {
-    if (!c || !values) return MF_ERR_ARG;
-    if (c->state < 1 || c->host_only) return MF_ERR_STATE;
-    CK(cudaSetDevice(c->device));
+namespace {
+
+// Run one launch program (the whole factorization for one rank, or rank 0's top
+// part) on the ctx stream: eagerly with per-launch events when profiling,
+// otherwise as a CUDA graph captured on first use.
+int run_program(mf_ctx *c, const std::vector<Launch> &prog, const double *vals, bool with_init, size_t ev_base,
+                cudaGraph_t *graph, cudaGraphExec_t *exec) {
     const Plan &P = c->P;
     const DevPlan &d = c->d;
     cudaStream_t st = c->stream;
-    const int64_t nv = (int64_t)c->S.bvidx.size() ? (int64_t)c->S.bvidx.size() : 0;
-    CK(cudaEventRecord(c->ev0, st));
-    const double *vals = values;
-    if (!is_device_ptr(values)) {
-        // bvidx indexes the caller's array; copy the whole array (colptr[n] entries)
-        const int64_t nall = c->S.nnz_in;
-        (void)nv;
-        if (nall > 0) CK(cudaMemcpyAsync(c->d_values, values, nall * sizeof(double), cudaMemcpyHostToDevice, st));
-        vals = c->d_values;
-    }
-    int64_t launches = 0;
-    const bool prof = c->profiling;
-    // The launch program: init flag + every launch of P.program, in order.
     auto issue = [&](const double *v, bool with_events) -> int {
-        launch_init_failed(c->d_failed, st);
-        for (size_t li = 0; li < P.program.size(); li++) {
-            const Launch &L = P.program[li];
-            if (with_events) CK(cudaEventRecord(c->prof_events[2 * li], st));
+        if (with_init) launch_init_failed(c->d_failed, st);
+        for (size_t li = 0; li < prog.size(); li++) {
+            const Launch &L = prog[li];
+            if (with_events) CK(cudaEventRecord(c->prof_events[ev_base + 2 * li], st));
             switch (L.kind) {
                 case KC_SMALL: launch_small_fronts(d, c->d_small + L.off, (int)L.count, L.param, v, st); break;
                 case KC_ASSEMBLE: launch_assemble(d, c->d_asm + 2 * L.off, L.count, v, st); break;
@@ -377,39 +388,103 @@ int mf_factor(mf_ctx *c, const double *values) {
                 case KC_TRSM: launch_trsm_panel(d, c->d_trsm + 2 * L.off, L.count, L.param, P.w, st); break;
                 case KC_UPDATE: launch_update(d, c->d_probs, c->d_tiles + L.off, L.count, st); break;
             }
-            if (with_events) CK(cudaEventRecord(c->prof_events[2 * li + 1], st));
+            if (with_events) CK(cudaEventRecord(c->prof_events[ev_base + 2 * li + 1], st));
         }
         return MF_OK;
     };
-    launches = 1 + (int64_t)P.program.size();
-    if (prof) {
-        if (c->prof_events.size() < 2 * P.program.size()) {
-            for (size_t i = c->prof_events.size(); i < 2 * P.program.size(); i++) {
-                cudaEvent_t e;
-                CK(cudaEventCreate(&e));
-                c->prof_events.push_back(e);
-            }
-        }
-        int r = issue(vals, true);
+    if (c->profiling) return issue(vals, true);
+    if (!c->use_graph) return issue(vals, false);
+    // the graph always reads the ctx's value buffer
+    if (vals != c->d_values && c->S.nnz_in > 0 && with_init)
+        CK(cudaMemcpyAsync(c->d_values, vals, c->S.nnz_in * sizeof(double), cudaMemcpyDeviceToDevice, st));
+    if (!*exec) {
+        CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
+        int r = issue(c->d_values, false);
+        cudaGraph_t g = nullptr;
+        cudaError_t e = cudaStreamEndCapture(st, &g);
         if (r) return r;
-    } else if (c->use_graph) {
-        // replay one CUDA graph of the whole program; it always reads the ctx's value buffer
-        if (vals != c->d_values && c->S.nnz_in > 0)
-            CK(cudaMemcpyAsync(c->d_values, vals, c->S.nnz_in * sizeof(double), cudaMemcpyDeviceToDevice, st));
-        if (!c->graph_exec) {
-            CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
-            int r = issue(c->d_values, false);
-            cudaGraph_t g = nullptr;
-            cudaError_t e = cudaStreamEndCapture(st, &g);
+        CK(e);
+        *graph = g;
+        CK(cudaGraphInstantiate(exec, g, 0));
+    }
+    CK(cudaGraphLaunch(*exec, st));
+    return MF_OK;
+}
+
+// Hand a list of transfers to the caller's exchange callback (multi-GPU only);
+// the ctx stream is drained first, so the buffers are final.
+int exchange(mf_ctx *c, std::vector<mf_xfer> &ops) {
+    // every rank calls the callback at every exchange point, even with nothing to
+    // move, so the caller's collectives stay aligned across ranks
+    if (!c->xfn) return MF_ERR_STATE;
+    CK(cudaStreamSynchronize(c->stream));
+    const int r = c->xfn(c->xuser, ops.empty() ? nullptr : ops.data(), (int64_t)ops.size());
+    return r ? MF_ERR_NCCL : MF_OK;
+}
+
+void accumulate_stats(mf_ctx *c, const std::vector<Launch> &prog, size_t ev_base) {
+    for (size_t li = 0; li < prog.size(); li++) {
+        const Launch &L = prog[li];
+        float t = 0.f;
+        cudaEventElapsedTime(&t, c->prof_events[ev_base + 2 * li], c->prof_events[ev_base + 2 * li + 1]);
+        mf_kernel_stat &K = c->kstats[L.kind];
+        K.launches += 1;
+        K.ms += t;
+        K.flops += L.flops;
+        K.bytes += L.bytes;
+    }
+}
+
+}  // namespace
+
+int mf_factor(mf_ctx *c, const double *values) {
+    if (!c || !values) return MF_ERR_ARG;
+    if (c->state < 1 || c->host_only) return MF_ERR_STATE;
+    CK(cudaSetDevice(c->device));
+    const Plan &P = c->P;
+    cudaStream_t st = c->stream;
+    const bool multi = P.nranks > 1;
+    if (multi && !c->xfn) return MF_ERR_STATE;
+    CK(cudaEventRecord(c->ev0, st));
+    const double *vals = values;
+    if (!is_device_ptr(values)) {
+        // bvidx indexes the caller's array; copy the whole array (colptr[n] entries)
+        if (c->S.nnz_in > 0)
+            CK(cudaMemcpyAsync(c->d_values, values, c->S.nnz_in * sizeof(double), cudaMemcpyHostToDevice, st));
+        vals = c->d_values;
+    }
+    const bool prof = c->profiling;
+    const size_t nev = 2 * (P.program.size() + P.program_top.size());
+    if (prof && c->prof_events.size() < nev) {
+        for (size_t i = c->prof_events.size(); i < nev; i++) {
+            cudaEvent_t e;
+            CK(cudaEventCreate(&e));
+            c->prof_events.push_back(e);
+        }
+    }
+    int r = run_program(c, P.program, vals, true, 0, &c->graph, &c->graph_exec);
+    if (r) return r;
+    int64_t launches = 1 + (int64_t)P.program.size();
+    if (multi) {
+        // (1) the frontier roots' update matrices travel to rank 0
+        std::vector<mf_xfer> ops;
+        for (int32_t root : P.frontier_roots) {
+            const int32_t own = P.owner[root], m = P.sn_f[root] - P.sn_k[root];
+            if (own == 0 || m <= 0) continue;
+            if (P.rank == own || P.rank == 0)
+                ops.push_back(mf_xfer{P.rank == own ? MF_XFER_SEND : MF_XFER_RECV, P.rank == own ? 0 : own,
+                                      c->d.U + P.U_off[root], (int64_t)m * m * (int64_t)sizeof(double)});
+        }
+        if ((r = exchange(c, ops))) return r;
+        // (2) rank 0 factors the top supernodes
+        if (!P.program_top.empty()) {
+            r = run_program(c, P.program_top, vals, false, 2 * P.program.size(), &c->graph_top, &c->graph_top_exec);
             if (r) return r;
-            CK(e);
-            c->graph = g;
-            CK(cudaGraphInstantiate(&c->graph_exec, g, 0));
+            launches += (int64_t)P.program_top.size();
         }
-        CK(cudaGraphLaunch(c->graph_exec, st));
-    } else {
-        int r = issue(vals, false);
-        if (r) return r;
+        // (3) first failing pivot over all ranks
+        std::vector<mf_xfer> red{mf_xfer{MF_XFER_ALLREDUCE_MIN_I32, 0, c->d_failed, (int64_t)sizeof(int)}};
+        if ((r = exchange(c, red))) return r;
     }
     CK(cudaGetLastError());
     int failed = INT_MAX;
@@ -421,16 +496,8 @@ int mf_factor(mf_ctx *c, const double *values) {
     c->info.t_factor = ms * 1e-3;
     c->info.launches_factor = launches;
     if (prof) {
-        for (size_t li = 0; li < P.program.size(); li++) {
-            const Launch &L = P.program[li];
-            float t = 0.f;
-            cudaEventElapsedTime(&t, c->prof_events[2 * li], c->prof_events[2 * li + 1]);
-            mf_kernel_stat &K = c->kstats[L.kind];
-            K.launches += 1;
-            K.ms += t;
-            K.flops += L.flops;
-            K.bytes += L.bytes;
-        }
+        accumulate_stats(c, P.program, 0);
+        accumulate_stats(c, P.program_top, 2 * P.program.size());
         c->prof_factors++;
     }
     if (failed != INT_MAX) {
@@ -443,32 +510,16 @@ int mf_factor(mf_ctx *c, const double *values) {
     return MF_OK;
 }
 
-int mf_solve(mf_ctx *c, const double *b, double *x) {
-    if (!c || !b || !x || b == x) return MF_ERR_ARG;
-    if (c->state != 2 || c->host_only) return MF_ERR_STATE;
-    CK(cudaSetDevice(c->device));
+namespace {
+void run_solve_program(mf_ctx *c, const std::vector<SolveLaunch> &prog) {
     const Plan &P = c->P;
     const DevPlan &d = c->d;
     cudaStream_t st = c->stream;
-    const int64_t n = c->S.n;
-    CK(cudaEventRecord(c->ev0, st));
-    const bool bdev = is_device_ptr(b), xdev = is_device_ptr(x);
-    const double *bd = b;
-    if (!bdev) {
-        CK(cudaMemcpyAsync(c->d_bx, b, n * sizeof(double), cudaMemcpyHostToDevice, st));
-        bd = c->d_bx;
-    }
-    launch_permute_in(d, bd, c->d_y, n, st);
-    CK(cudaMemsetAsync(c->d_counters, 0, (P.sb_groups.size() / 2 + 1) * sizeof(int), st));
-    for (const SolveLaunch &L : P.fsolve) {
+    for (const SolveLaunch &L : prog) {
         switch (L.kind) {
             case SK_SMALL_F: launch_fwd_solve(d, c->d_solve_list + L.off, (int)L.count, c->d_y, st); break;
             case SK_INIT_F: launch_fsolve_init(d, c->d_solve_list + L.off, (int)L.count, c->d_y, st); break;
             case SK_WAVE_F: launch_fsolve_wave(d, c->d_sf_tasks + 3 * L.off, L.count, L.j0, P.w, c->d_y, st); break;
-        }
-    }
-    for (const SolveLaunch &L : P.bsolve) {
-        switch (L.kind) {
             case SK_SMALL_B:
                 launch_bwd_solve(d, c->d_solve_list + L.off, (int)L.count, c->d_y, c->d_sn_rows, c->d_sn_rowptr, st);
                 break;
@@ -481,6 +532,55 @@ int mf_solve(mf_ctx *c, const double *b, double *x) {
                 break;
         }
     }
+}
+}  // namespace
+
+int mf_solve(mf_ctx *c, const double *b, double *x) {
+    if (!c || !b || !x || b == x) return MF_ERR_ARG;
+    if (c->state != 2 || c->host_only) return MF_ERR_STATE;
+    CK(cudaSetDevice(c->device));
+    const Plan &P = c->P;
+    const DevPlan &d = c->d;
+    cudaStream_t st = c->stream;
+    const int64_t n = c->S.n;
+    const bool multi = P.nranks > 1;
+    CK(cudaEventRecord(c->ev0, st));
+    const bool bdev = is_device_ptr(b), xdev = is_device_ptr(x);
+    const double *bd = b;
+    if (!bdev) {
+        CK(cudaMemcpyAsync(c->d_bx, b, n * sizeof(double), cudaMemcpyHostToDevice, st));
+        bd = c->d_bx;
+    }
+    launch_permute_in(d, bd, c->d_y, n, st);
+    CK(cudaMemsetAsync(c->d_counters, 0, (P.sb_groups.size() / 2 + 1) * sizeof(int), st));
+    int r;
+    run_solve_program(c, P.fsolve);                  // forward, own subtrees
+    if (multi) {
+        std::vector<mf_xfer> ops;                      // frontier roots' update vectors -> rank 0
+        for (int32_t root : P.frontier_roots) {
+            const int32_t own = P.owner[root];
+            if (own == 0 || P.sn_f[root] == P.sn_k[root]) continue;
+            if (P.rank == own || P.rank == 0)
+                ops.push_back(mf_xfer{P.rank == own ? MF_XFER_SEND : MF_XFER_RECV, P.rank == own ? 0 : own,
+                                      c->d.fv + P.fv_off[root], (int64_t)P.sn_f[root] * (int64_t)sizeof(double)});
+        }
+        if ((r = exchange(c, ops))) return r;
+        run_solve_program(c, P.fsolve_top);          // rank 0: forward + backward on the top
+        run_solve_program(c, P.bsolve_top);
+        // rank 0's top solution -> every rank (y columns of the top supernodes)
+        if (P.rank == 0) CK(cudaMemcpyAsync(c->d_ytmp, c->d_y, n * sizeof(double), cudaMemcpyDeviceToDevice, st));
+        std::vector<mf_xfer> bc{mf_xfer{MF_XFER_BCAST, 0, c->d_ytmp, n * (int64_t)sizeof(double)}};
+        if ((r = exchange(c, bc))) return r;
+        if (P.rank != 0) launch_copy_cols(d, c->d_top_list, (int)P.top_list.size(), c->d_ytmp, c->d_y, st);
+    }
+    run_solve_program(c, P.bsolve);                  // backward, own subtrees
+    if (multi) {   // every rank contributes its own columns; the sum is the full solution
+        CK(cudaMemsetAsync(c->d_ytmp, 0, n * sizeof(double), st));
+        launch_copy_cols(d, c->d_own_list, (int)P.own_list.size(), c->d_y, c->d_ytmp, st);
+        std::vector<mf_xfer> ar{mf_xfer{MF_XFER_ALLREDUCE_SUM, 0, c->d_ytmp, n * (int64_t)sizeof(double)}};
+        if ((r = exchange(c, ar))) return r;
+        CK(cudaMemcpyAsync(c->d_y, c->d_ytmp, n * sizeof(double), cudaMemcpyDeviceToDevice, st));
+    }
     double *xd = xdev ? x : c->d_bx;
     launch_permute_out(d, c->d_y, xd, n, st);
     if (!xdev) CK(cudaMemcpyAsync(x, c->d_bx, n * sizeof(double), cudaMemcpyDeviceToHost, st));
@@ -490,6 +590,13 @@ int mf_solve(mf_ctx *c, const double *b, double *x) {
     float ms = 0.f;
     cudaEventElapsedTime(&ms, c->ev0, c->ev1);
     c->info.t_solve = ms * 1e-3;
+    return MF_OK;
+}
+
+int mf_set_exchange(mf_ctx *c, mf_exchange_fn fn, void *user) {
+    if (!c) return MF_ERR_ARG;
+    c->xfn = fn;
+    c->xuser = user;
     return MF_OK;
 }
 
@@ -550,6 +657,18 @@ int mf_set_profiling(mf_ctx *c, int enable) {
         snprintf(c->kstats[k].name, sizeof(c->kstats[k].name), "%s", kKernelNames[k]);
     }
     c->prof_factors = 0;
+    return MF_OK;
+}
+
+int mf_get_mapping(const mf_ctx *c, int32_t *owner, int8_t *top, double *rank_load, double *top_load) {
+    if (!c) return MF_ERR_ARG;
+    if (c->state < 1) return MF_ERR_STATE;
+    const Plan &P = c->P;
+    if (owner) std::memcpy(owner, P.owner.data(), P.owner.size() * sizeof(int32_t));
+    if (top)
+        for (size_t i = 0; i < P.top.size(); i++) top[i] = P.top[i];
+    if (rank_load) std::memcpy(rank_load, P.rank_load.data(), P.rank_load.size() * sizeof(double));
+    if (top_load) *top_load = P.top_load;
     return MF_OK;
 }
 

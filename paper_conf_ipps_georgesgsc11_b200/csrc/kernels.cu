@@ -791,6 +791,18 @@ void launch_bsolve_wave(const DevPlan &d, const int32_t *tasks, int64_t task_bas
                                                                   counters);
 }
 
+// dst[first_s + j] = src[first_s + j] for the columns of the listed supernodes
+__global__ void k_copy_cols(DevPlan d, const int32_t *__restrict__ list, const double *__restrict__ src,
+                            double *__restrict__ dst) {
+    const int s = list[blockIdx.x];
+    const int k = d.sn_k[s], first = d.sn_first[s];
+    for (int j = threadIdx.x; j < k; j += blockDim.x) dst[first + j] = src[first + j];
+}
+void launch_copy_cols(const DevPlan &d, const int32_t *list, int count, const double *src, double *dst,
+                      cudaStream_t st) {
+    if (count > 0) k_copy_cols<<<count, 128, 0, st>>>(d, list, src, dst);
+}
+
 void launch_fwd_solve(const DevPlan &d, const int32_t *list, int count, double *y, cudaStream_t st) {
     if (count > 0) k_fwd_solve<<<count, kSolveThreads, 0, st>>>(d, list, y);
 }

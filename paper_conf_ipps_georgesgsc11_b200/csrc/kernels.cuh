@@ -47,6 +47,8 @@ void launch_bsolve_wave(const DevPlan &d, const int32_t *tasks, int64_t task_bas
                         int j0, int w, double *y, double *partials, int *counters, cudaStream_t st);
 int small_front_smem_ok(int fmax);
 int kernels_init();
+void launch_copy_cols(const DevPlan &d, const int32_t *list, int count, const double *src, double *dst,
+                      cudaStream_t st);
 void launch_export_diag(const DevPlan &d, int nsuper, double *out, cudaStream_t st);
 
 }  // namespace mf

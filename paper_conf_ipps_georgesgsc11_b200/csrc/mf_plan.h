@@ -19,6 +19,8 @@ struct Options {
     double zrelax[3] = {0.8, 0.1, 0.05};
     int small_front_max = 128;
     int panel_w = 64;
+    int nranks = 1;   // GPUs sharing one factorization (one process per GPU)
+    int rank = 0;
 };
 
 // ---------------------------------------------------------------- symbolic
@@ -125,6 +127,18 @@ struct Plan {
     std::vector<int32_t> sb_tasks;                   // backward waves: (front, row0, group)
     std::vector<int32_t> sb_groups;                  // (first task, ntasks) per (front, block)
     std::vector<SolveLaunch> fsolve, bsolve;
+    // ---- multi-GPU: subtree-to-GPU mapping.  Subtrees below a
+    // frontier are factored by their owner; the supernodes above the frontier ("top")
+    // are factored by rank 0 after the frontier roots' update matrices arrive.
+    int32_t nranks = 1, rank = 0;
+    std::vector<int32_t> owner;                      // rank factoring each supernode
+    std::vector<char> top;                           // above the frontier (rank 0)
+    std::vector<int32_t> frontier_roots;             // subtree roots whose parent is top
+    std::vector<double> rank_load;                   // executed flops per rank (subtrees)
+    double top_load = 0;
+    std::vector<Launch> program_top;                 // rank 0: top supernodes
+    std::vector<SolveLaunch> fsolve_top, bsolve_top; // rank 0: top supernodes
+    std::vector<int32_t> top_list, own_list;         // supernode lists (copy / mask kernels)
 };
 
 constexpr int kTileM = 64, kTileN = 64;

@@ -36,13 +36,15 @@ static void add_tiles(Plan &P, int32_t prob, int32_t M, int32_t N) {
 // Solve program: per level, small supernodes in one batched launch; large ones
 // (f > small_max) blocked by w columns so that no supernode is handled by a
 // single CTA (the root of c5 has k = 14,900).
-static void build_solve_plan(const Symbolic &S, Plan &P) {
+static void build_solve_plan(const Symbolic &S, Plan &P, const std::vector<char> &include,
+                             std::vector<SolveLaunch> &fsolve, std::vector<SolveLaunch> &bsolve) {
     (void)S;
     const int w = P.w;
     std::vector<std::vector<int32_t>> large(P.nlevels), small(P.nlevels);
     for (int32_t l = 0; l < P.nlevels; l++) {
         for (int32_t q = P.level_ptr[l]; q < P.level_ptr[l + 1]; q++) {
             const int32_t s = P.level_list[q];
+            if (!include[s]) continue;
             (P.sn_f[s] > P.small_max ? large[l] : small[l]).push_back(s);
         }
         std::stable_sort(large[l].begin(), large[l].end(),
@@ -54,9 +56,9 @@ static void build_solve_plan(const Symbolic &S, Plan &P) {
         return off;
     };
     for (int32_t l = 0; l < P.nlevels; l++) {
-        if (!small[l].empty()) P.fsolve.push_back({SK_SMALL_F, 0, push_list(small[l]), (int64_t)small[l].size()});
+        if (!small[l].empty()) fsolve.push_back({SK_SMALL_F, 0, push_list(small[l]), (int64_t)small[l].size()});
         if (large[l].empty()) continue;
-        P.fsolve.push_back({SK_INIT_F, 0, push_list(large[l]), (int64_t)large[l].size()});
+        fsolve.push_back({SK_INIT_F, 0, push_list(large[l]), (int64_t)large[l].size()});
         const int32_t kmax = P.sn_k[large[l][0]];
         for (int32_t j0 = 0; j0 < kmax; j0 += w) {
             const int64_t off = (int64_t)P.sf_tasks.size() / 3;
@@ -72,12 +74,12 @@ static void build_solve_plan(const Symbolic &S, Plan &P) {
                     r0 += kSolveRows;
                 } while (r0 < f);
             }
-            P.fsolve.push_back({SK_WAVE_F, j0, off, (int64_t)P.sf_tasks.size() / 3 - off});
+            fsolve.push_back({SK_WAVE_F, j0, off, (int64_t)P.sf_tasks.size() / 3 - off});
         }
     }
     for (int32_t l = P.nlevels - 1; l >= 0; l--) {
         if (!large[l].empty()) {
-            P.bsolve.push_back({SK_INIT_B, 0, push_list(large[l]), (int64_t)large[l].size()});
+            bsolve.push_back({SK_INIT_B, 0, push_list(large[l]), (int64_t)large[l].size()});
             const int32_t kmax = P.sn_k[large[l][0]];
             const int32_t nb = (kmax + w - 1) / w;
             for (int32_t b = nb - 1; b >= 0; b--) {
@@ -100,17 +102,103 @@ static void build_solve_plan(const Symbolic &S, Plan &P) {
                     P.sb_groups.push_back(first_task);
                     P.sb_groups.push_back(nt);
                 }
-                P.bsolve.push_back({SK_WAVE_B, j0, off, (int64_t)P.sb_tasks.size() / 3 - off});
+                bsolve.push_back({SK_WAVE_B, j0, off, (int64_t)P.sb_tasks.size() / 3 - off});
             }
         }
-        if (!small[l].empty()) P.bsolve.push_back({SK_SMALL_B, 0, push_list(small[l]), (int64_t)small[l].size()});
+        if (!small[l].empty()) bsolve.push_back({SK_SMALL_B, 0, push_list(small[l]), (int64_t)small[l].size()});
     }
+}
+
+// Subtree-to-GPU mapping (proportional/LPT): start from the
+// tree roots as the frontier; repeatedly move the heaviest expandable frontier
+// subtree's root into the "top" (its children join the frontier), assign the
+// frontier subtrees to ranks by LPT on executed flops, and keep the frontier
+// with the smallest makespan = max rank load + top load (rank 0 factors the top
+// after every frontier root's update matrix has arrived).
+static void map_subtrees(Plan &P, const std::vector<double> &front_load) {
+    const int32_t ns = P.nsuper, R = P.nranks;
+    P.owner.assign(ns, 0);
+    P.top.assign(ns, 0);
+    P.frontier_roots.clear();
+    P.rank_load.assign(R, 0.0);
+    P.top_load = 0;
+    std::vector<double> sub(front_load);
+    for (int32_t s = 0; s < ns; s++)
+        for (int32_t q = P.child_ptr[s]; q < P.child_ptr[s + 1]; q++) sub[s] += sub[P.child_list[q]];
+    std::vector<int32_t> roots;
+    std::vector<int32_t> parent(ns, -1);
+    for (int32_t s = 0; s < ns; s++)
+        for (int32_t q = P.child_ptr[s]; q < P.child_ptr[s + 1]; q++) parent[P.child_list[q]] = s;
+    for (int32_t s = 0; s < ns; s++)
+        if (parent[s] < 0) roots.push_back(s);
+    if (R <= 1) {
+        P.rank_load[0] = 0;
+        for (int32_t r : roots) P.rank_load[0] += sub[r];
+        return;
+    }
+    auto lpt = [&](const std::vector<int32_t> &fr, std::vector<int32_t> &assign, std::vector<double> &load) {
+        std::vector<int32_t> ord(fr.size());
+        std::iota(ord.begin(), ord.end(), 0);
+        std::stable_sort(ord.begin(), ord.end(), [&](int32_t a, int32_t b) { return sub[fr[a]] > sub[fr[b]]; });
+        load.assign(R, 0.0);
+        assign.assign(fr.size(), 0);
+        for (int32_t i : ord) {
+            int32_t best = 0;
+            for (int32_t r = 1; r < R; r++)
+                if (load[r] < load[best]) best = r;
+            assign[i] = best;
+            load[best] += sub[fr[i]];
+        }
+        return *std::max_element(load.begin(), load.end());
+    };
+    std::vector<int32_t> fr = roots, best_fr = roots, assign, best_assign;
+    std::vector<double> load, best_load;
+    std::vector<char> is_top(ns, 0), best_top(ns, 0);
+    double topl = 0, best_make = lpt(fr, best_assign, best_load);
+    for (int iter = 0; iter < 64 * R && (int)fr.size() < 64 * R; iter++) {
+        int32_t pick = -1;
+        for (size_t i = 0; i < fr.size(); i++)
+            if (P.child_ptr[fr[i] + 1] > P.child_ptr[fr[i]] && (pick < 0 || sub[fr[i]] > sub[fr[pick]])) pick = (int32_t)i;
+        if (pick < 0) break;
+        const int32_t v = fr[pick];
+        fr.erase(fr.begin() + pick);
+        is_top[v] = 1;
+        topl += front_load[v];
+        for (int32_t q = P.child_ptr[v]; q < P.child_ptr[v + 1]; q++) fr.push_back(P.child_list[q]);
+        const double make = lpt(fr, assign, load) + topl;
+        if (make < best_make) {
+            best_make = make;
+            best_fr = fr;
+            best_assign = assign;
+            best_load = load;
+            best_top = is_top;
+        }
+    }
+    P.top = best_top;
+    P.rank_load = best_load;
+    for (int32_t s = 0; s < ns; s++)
+        if (P.top[s]) P.top_load += front_load[s];
+    // owner of every supernode below the frontier = owner of its frontier root
+    for (size_t i = 0; i < best_fr.size(); i++) {
+        const int32_t rt = best_fr[i];
+        P.frontier_roots.push_back(rt);
+        std::vector<int32_t> stack{rt};
+        while (!stack.empty()) {
+            const int32_t v = stack.back();
+            stack.pop_back();
+            P.owner[v] = best_assign[i];
+            for (int32_t q = P.child_ptr[v]; q < P.child_ptr[v + 1]; q++) stack.push_back(P.child_list[q]);
+        }
+    }
+    std::sort(P.frontier_roots.begin(), P.frontier_roots.end());
 }
 
 int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     P = Plan();
     const int32_t ns = (int32_t)S.sn_parent.size();
     P.nsuper = ns;
+    P.nranks = std::max(1, opt.nranks);
+    P.rank = opt.rank;
     P.w = opt.panel_w;
     P.small_max = opt.small_front_max;
     P.sn_k.resize(ns);
@@ -218,8 +306,33 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     };
     auto upd_flops = [](double M, double N, double K) { return 2.0 * K * (N * (N + 1) / 2 + (M - N) * N); };
     auto upd_bytes = [](double M, double N, double K) { return 8.0 * (M * K + 2 * (N * (N + 1) / 2 + (M - N) * N)); };
+    // ---- subtree-to-GPU mapping and the per-rank inclusion masks
+    {
+        std::vector<double> front_load(ns);
+        for (int32_t s = 0; s < ns; s++) {
+            const double k = P.sn_k[s], m = P.sn_f[s] - P.sn_k[s];
+            front_load[s] = k * m * m + m * k * (k + 1) + k * (k + 1) * (2 * k + 1) / 6;
+        }
+        map_subtrees(P, front_load);
+    }
+    std::vector<char> inc_local(ns), inc_top(ns);
+    for (int32_t s = 0; s < ns; s++) {
+        inc_local[s] = !P.top[s] && P.owner[s] == P.rank;
+        inc_top[s] = P.top[s] && P.rank == 0;
+        if (P.top[s]) P.top_list.push_back(s);                      // every rank: y columns broadcast by rank 0
+        if (inc_local[s] || inc_top[s]) P.own_list.push_back(s);   // columns this rank finalises
+    }
+    std::vector<Launch> *cur = &P.program;
+    const std::vector<char> *inc = &inc_local;
+    for (int pass = 0; pass < 2; pass++) {
+    if (pass == 1) {
+        cur = &P.program_top;
+        inc = &inc_top;
+    }
     for (int32_t l = 0; l < nlev; l++) {
-        std::vector<int32_t> fronts(P.level_list.begin() + P.level_ptr[l], P.level_list.begin() + P.level_ptr[l + 1]);
+        std::vector<int32_t> fronts;
+        for (int32_t q = P.level_ptr[l]; q < P.level_ptr[l + 1]; q++)
+            if ((*inc)[P.level_list[q]]) fronts.push_back(P.level_list[q]);
         for (int cls = 0; cls < kSmallClasses; cls++) {
             const int lo = cls == 0 ? 0 : P.small_class_fmax[cls - 1];
             Launch L{KC_SMALL, P.small_class_fmax[cls], (int64_t)P.small_list.size(), 0, 0.0, 0.0, l};
@@ -231,7 +344,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
                     L.bytes += asm_bytes(s) + 8.0 * (panel_words(s) + m * (m + 1) / 2);
                 }
             L.count = (int64_t)P.small_list.size() - L.off;
-            if (L.count) P.program.push_back(L);
+            if (L.count) cur->push_back(L);
         }
         std::vector<int32_t> large;
         for (int32_t s : fronts)
@@ -252,7 +365,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
                 L.bytes += asm_bytes(s) + 8.0 * (f * k + m * (m + 1) / 2);   // zero + write panel and U
             }
             L.count = (int64_t)P.asm_tasks.size() / 2 - L.off;
-            P.program.push_back(L);
+            cur->push_back(L);
         }
         // Blocked factorization of the k pivot columns of every large front, in
         // lockstep over the level (Fig. 9: w x w potrf kernel, trsm
@@ -288,8 +401,8 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
                     Lt.bytes += 8.0 * (2 * rows * we + (double)we * (we + 1) / 2);
                 }
                 Lt.count = (int64_t)P.trsm_tasks.size() / 2 - Lt.off;
-                P.program.push_back(Lp);
-                if (Lt.count) P.program.push_back(Lt);
+                cur->push_back(Lp);
+                if (Lt.count) cur->push_back(Lt);
                 return;
             }
             const int32_t mid = a + (b - a + 1) / 2;
@@ -318,7 +431,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
                 Lu.bytes += upd_bytes(M, N, K);
             }
             Lu.count = (int64_t)P.tiles.size() - Lu.off;
-            if (Lu.count) P.program.push_back(Lu);
+            if (Lu.count) cur->push_back(Lu);
             rec(mid, b);
         };
         const int32_t nb = (P.sn_k[large[0]] + w - 1) / w;
@@ -344,9 +457,11 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
             Ls.bytes += upd_bytes(m, m, k);
         }
         Ls.count = (int64_t)P.tiles.size() - Ls.off;
-        if (Ls.count) P.program.push_back(Ls);
+        if (Ls.count) cur->push_back(Ls);
     }
-    build_solve_plan(S, P);
+    }   // pass
+    build_solve_plan(S, P, inc_local, P.fsolve, P.bsolve);
+    build_solve_plan(S, P, inc_top, P.fsolve_top, P.bsolve_top);
     return MF_OK;
 }
 

@@ -25,7 +25,7 @@ MF_ERR_NCCL = -5
 EXPORTED_SYMBOLS = (
     "mf_default_options", "mf_create", "mf_analyze", "mf_factor", "mf_solve", "mf_get_info",
     "mf_get_perm", "mf_get_etree", "mf_get_supernodes", "mf_export_panel", "mf_export_diag", "mf_export_L",
-    "mf_get_program", "mf_set_profiling", "mf_get_kernel_stats", "mf_destroy", "mf_strerror",
+    "mf_get_program", "mf_set_profiling", "mf_get_kernel_stats", "mf_set_exchange", "mf_get_mapping", "mf_destroy", "mf_strerror",
 )
 
 
@@ -33,7 +33,8 @@ class Options(ctypes.Structure):
     _fields_ = [
         ("amalgamate", ctypes.c_int32), ("nrelax", ctypes.c_int32 * 3), ("zrelax", ctypes.c_double * 3),
         ("small_front_max", ctypes.c_int32), ("panel_w", ctypes.c_int32), ("device", ctypes.c_int32),
-        ("host_only", ctypes.c_int32), ("stream", ctypes.c_void_p),
+        ("host_only", ctypes.c_int32), ("nranks", ctypes.c_int32), ("rank", ctypes.c_int32),
+        ("stream", ctypes.c_void_p),
     ]
 
 
@@ -57,6 +58,15 @@ class KernelStat(ctypes.Structure):
 
 
 MF_KERNEL_CLASSES = 5
+
+MF_XFER_SEND, MF_XFER_RECV, MF_XFER_BCAST, MF_XFER_ALLREDUCE_SUM, MF_XFER_ALLREDUCE_MIN_I32 = 1, 2, 3, 4, 5
+
+
+class Xfer(ctypes.Structure):
+    _fields_ = [("op", ctypes.c_int32), ("peer", ctypes.c_int32), ("ptr", ctypes.c_void_p), ("bytes", ctypes.c_int64)]
+
+
+EXCHANGE_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.POINTER(Xfer), ctypes.c_int64)
 
 
 class LaunchInfo(ctypes.Structure):
@@ -88,6 +98,8 @@ def _load():
         "mf_export_diag": ([vp, vp], ctypes.c_int),
         "mf_export_L": ([vp, vp], ctypes.c_int),
         "mf_get_program": ([vp, ctypes.POINTER(LaunchInfo), i64, ctypes.POINTER(i64)], ctypes.c_int),
+        "mf_set_exchange": ([vp, EXCHANGE_FN, vp], ctypes.c_int),
+        "mf_get_mapping": ([vp, vp, vp, vp, vp], ctypes.c_int),
         "mf_set_profiling": ([vp, ctypes.c_int], ctypes.c_int),
         "mf_get_kernel_stats": ([vp, ctypes.POINTER(KernelStat), ctypes.POINTER(i32)], ctypes.c_int),
         "mf_destroy": ([vp], None),
@@ -134,7 +146,8 @@ class Solver:
     """mf_create / mf_analyze / mf_factor / mf_solve on one context."""
 
     def __init__(self, amalgamate: bool = True, small_front_max: int | None = None, panel_w: int | None = None,
-                 device: int = -1, stream: int | None = None, host_only: bool = False):
+                 device: int = -1, stream: int | None = None, host_only: bool = False,
+                 nranks: int = 1, rank: int = 0, exchange=None):
         o = Options()
         lib.mf_default_options(ctypes.byref(o))
         o.amalgamate = int(amalgamate)
@@ -144,6 +157,8 @@ class Solver:
             o.panel_w = panel_w
         o.device = device
         o.host_only = int(host_only)
+        o.nranks = nranks
+        o.rank = rank
         o.stream = stream
         h = ctypes.c_void_p()
         r = lib.mf_create(ctypes.byref(h), ctypes.byref(o))
@@ -151,6 +166,34 @@ class Solver:
             raise MfError(r, "mf_create")
         self._h = h
         self.n = None
+        self.nranks, self.rank = nranks, rank
+        self._xcb = None
+        if exchange is not None:
+            self.set_exchange(exchange)
+
+    def set_exchange(self, fn):
+        """fn(list of (op, peer, device_ptr, nbytes)) -> None; must complete the transfers."""
+        def _cb(_user, ops, nops):
+            try:
+                fn([(ops[i].op, ops[i].peer, ops[i].ptr, ops[i].bytes) for i in range(nops)])
+                return 0
+            except Exception as e:  # noqa: BLE001 -- reported through the C return code
+                import traceback
+                traceback.print_exc()
+                return 1
+        self._xcb = EXCHANGE_FN(_cb)
+        self._check(lib.mf_set_exchange(self._h, self._xcb, None), "mf_set_exchange")
+
+    def mapping(self):
+        inf = self.info()
+        ns = inf["nsuper"]
+        owner = np.empty(ns, dtype=np.int32)
+        top = np.empty(ns, dtype=np.int8)
+        load = np.empty(self.nranks, dtype=np.float64)
+        tl = ctypes.c_double()
+        self._check(lib.mf_get_mapping(self._h, owner.ctypes.data, top.ctypes.data, load.ctypes.data,
+                                       ctypes.byref(tl)), "mf_get_mapping")
+        return owner, top.astype(bool), load, tl.value
 
     def close(self):
         if getattr(self, "_h", None):
