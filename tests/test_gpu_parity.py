@@ -28,10 +28,10 @@ def mf():
     return m
 
 
-def c11(Pg, Po):
+def c11(Pg, Po, tau=1e-6):
     """Reading C11 floored relative error of one panel (columns = columns of L)."""
     colmax = np.abs(Po).max(axis=0)
-    den = np.maximum(np.abs(Po), 1e-6 * colmax[None, :])
+    den = np.maximum(np.abs(Po), tau * colmax[None, :])
     den[den == 0] = 1.0
     return float((np.abs(Pg - Po) / den).max())
 
@@ -45,7 +45,7 @@ def factor_both(mf, A, perm, supernodes=None, **opts):
     return S, sym, panels
 
 
-def check_panels(S, sym, panels, exact=False):
+def check_panels(S, sym, panels, exact=False, tau=1e-6):
     worst = 0.0
     for s, Po in panels.items():
         f, k = Po.shape
@@ -54,7 +54,7 @@ def check_panels(S, sym, panels, exact=False):
         if exact:
             np.testing.assert_array_equal(Pg, Po)
         else:
-            worst = max(worst, c11(Pg, Po))
+            worst = max(worst, c11(Pg, Po, tau))
         if sym.Li is not None:   # amalgamation padding must be exactly 0
             R = sym.rows(s)
             for jj in range(k):
@@ -254,7 +254,7 @@ def test_degenerate_inputs(mf):
     assert S.solve(np.zeros(0)).size == 0
 
 
-@pytest.mark.parametrize("name", ["c5"])
+@pytest.mark.parametrize("name", ["c5", "c4", "c3", "c2"])
 def test_full_size_sampled(mf, name):
     """BASELINE config at full size, in bench.py's launch configuration: sampled
     whole subtrees vs the oracle (subset factorization), closed-form log det and
@@ -277,13 +277,22 @@ def test_full_size_sampled(mf, name):
         while stack:
             v = stack.pop(); subset.add(v); stack.extend(ch[v])
     panels = oracle.factor(A, sym, subset=subset)
-    check_panels(S, sym, panels)
-    # closed-form log det of 27I - T(x)T(x)T
+    # Reading C11: elasticity is not an M-matrix; its cancellation-noise entries
+    # (down to ~1e-18 of the column max) agree only to fp64 roundoff of the
+    # column max (observed 4.7e-16 * colmax in c4's 7728 x 1875 fronts), so the
+    # relative floor is 1e-4 of the column max there (1e-6 for the stencils).
+    check_panels(S, sym, panels, tau=1e-4 if c["kind"] == "elast" else 1e-6)
+    # closed-form log det of the Laplacian stencils (Kronecker-sum eigenvalues)
     N = c["N"]
     th = np.arange(1, N + 1) * np.pi / (N + 1)
     t1 = 1 + 2 * np.cos(th)
-    ld = float(np.sum(np.log(27 - t1[:, None, None] * t1[None, :, None] * t1[None, None, :])))
-    assert 2 * np.sum(np.log(S.diag())) == pytest.approx(ld, rel=1e-12)
+    k1 = 4 * np.sin(th / 2) ** 2
+    lam = {"27pt": lambda: 27 - t1[:, None, None] * t1[None, :, None] * t1[None, None, :],
+           "9pt": lambda: 9 - t1[:, None] * t1[None, :],
+           "7pt": lambda: k1[:, None, None] + k1[None, :, None] + k1[None, None, :]}.get(c["kind"])
+    if lam is not None:
+        ld = float(np.sum(np.log(lam())))
+        assert 2 * np.sum(np.log(S.diag())) == pytest.approx(ld, rel=1e-12)
     b = spmv(A, G.rhs(A.n, 0))
     x = S.solve(b)
     assert backward_error(A, x, b) <= TOL_BE
