@@ -104,7 +104,7 @@ typedef struct {
     double bytes;
 } mf_kernel_stat;
 
-#define MF_KERNEL_CLASSES 5
+#define MF_KERNEL_CLASSES 6
 
 /* Multi-GPU exchange.  With nranks > 1 every rank passes the
  * same n/colptr/rowind/perm/values/b; elimination subtrees are mapped to ranks and

@@ -347,6 +347,11 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     if ((r = dev_alloc(c, &p, (P.sb_groups.size() / 2 + 1) * sizeof(int))) != MF_OK) return r;
     c->d_counters = (int *)p;
     d.failed = c->d_failed;
+    d.epoch = reinterpret_cast<const unsigned *>(c->d_failed + 1);
+    if ((r = dev_alloc(c, &p, std::max<int32_t>(P.nsuper, 1) * sizeof(unsigned))) != MF_OK) return r;
+    d.leaf_flag = (unsigned *)p;
+    CK(cudaMemsetAsync(d.leaf_flag, 0, std::max<int32_t>(P.nsuper, 1) * sizeof(unsigned), c->stream));
+    CK(cudaMemsetAsync(c->d_failed, 0, sizeof(int) * 4, c->stream));
     if ((r = dev_alloc(c, &p, std::max<int64_t>(S.nnz_in, 1) * sizeof(double))) != MF_OK) return r;
     c->d_values = (double *)p;
     if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(n, 1) * sizeof(double))) != MF_OK) return r;
@@ -387,6 +392,9 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, const double *vals, 
                 case KC_POTRF: launch_potrf_diag(d, c->d_large + L.off, (int)L.count, L.param, P.w, st); break;
                 case KC_TRSM: launch_trsm_panel(d, c->d_trsm + 2 * L.off, L.count, L.param, P.w, st); break;
                 case KC_UPDATE: launch_update(d, c->d_probs, c->d_tiles + L.off, L.count, st); break;
+                case KC_LEAF:
+                    launch_leaf(d, c->d_large + L.off, (int)L.count, c->d_trsm + 2 * L.off2, L.count2, L.param, P.w, st);
+                    break;
             }
             if (with_events) CK(cudaEventRecord(c->prof_events[ev_base + 2 * li + 1], st));
         }
@@ -647,7 +655,7 @@ int mf_export_panel(const mf_ctx *c, int32_t s, double *out) {
 }
 
 static const char *kKernelNames[KC_COUNT] = {"small_front_fused", "assemble_extend_add", "potrf_diag",
-                                             "trsm_panel", "dmma_schur_update"};
+                                             "trsm_panel", "dmma_schur_update", "leaf_potrf_trsm"};
 
 int mf_set_profiling(mf_ctx *c, int enable) {
     if (!c) return MF_ERR_ARG;

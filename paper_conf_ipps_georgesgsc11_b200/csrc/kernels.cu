@@ -32,7 +32,10 @@ __device__ __forceinline__ void note_pivot(const DevPlan &d, double djj, int col
     if (!(djj > 0.0)) atomicMin(d.failed, col);   // non-positive or NaN pivot (reading C8)
 }
 
-__global__ void k_init_failed(int *failed) { *failed = INT_MAX; }
+__global__ void k_init_failed(int *failed, unsigned *epoch) {
+    *failed = INT_MAX;
+    *epoch += 1;   // new factorization: fused-leaf flags of the previous one no longer match
+}
 
 // 1/sqrt(x) for a pivot: float MUFU seed + two fp64 Newton steps (~1 ulp; exactly
 // 2^-p for x = 4^p, so the manufactured integer factors stay exact).  Outside the
@@ -337,26 +340,24 @@ constexpr int kPotrfThreads = 256;
 // The per-pivot critical path is one rsqrt + a few shuffles instead of two
 // block-wide barriers.  1/L_jj uses rsqrt (exact for the power-of-4 pivots of
 // the manufactured inputs); L_jj = d * rsqrt(d).
-__global__ void __launch_bounds__(kPotrfThreads) k_potrf_diag(DevPlan d, const int32_t *__restrict__ fronts,
-                                                              int j0, int w) {
+template <int NT>
+__device__ __forceinline__ void potrf_block(const DevPlan &d, int s, int j0, int w, double *A, double *sinv) {
     constexpr int LDA = kWmax;            // column-major: A[c * LDA + r]
-    __shared__ double A[kWmax * LDA];
-    __shared__ double sinv[kWmax];
-    const int s = fronts[blockIdx.x];
+    constexpr int G = NT / 64;            // column groups
     const int k = d.sn_k[s], ld = d.sn_ld[s], first = d.sn_first[s];
     const int we = min(w, k - j0);
     double *__restrict__ P = d.L + d.L_off[s] + (int64_t)j0 * ld + j0;
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int tid = threadIdx.x, warp = tid >> 5;
     {
         const int i = tid & 63, h = tid >> 6;
-        double v[kWmax / 4];
+        double v[kWmax / G];
 #pragma unroll
-        for (int t = 0; t < kWmax / 4; t++) {
-            const int c = h + 4 * t;
+        for (int t = 0; t < kWmax / G; t++) {
+            const int c = h + G * t;
             v[t] = (i < we && c < we) ? P[i + (int64_t)c * ld] : 0.0;
         }
 #pragma unroll
-        for (int t = 0; t < kWmax / 4; t++) A[(h + 4 * t) * LDA + i] = v[t];
+        for (int t = 0; t < kWmax / G; t++) A[(h + G * t) * LDA + i] = v[t];
     }
     __syncthreads();
 #pragma unroll 1
@@ -393,7 +394,7 @@ __global__ void __launch_bounds__(kPotrfThreads) k_potrf_diag(DevPlan d, const i
                 double li[16];
 #pragma unroll
                 for (int q = 0; q < 16; q++) li[q] = A[(s0 + q) * LDA + i];
-                for (int c = r0 + h; c <= i; c += 4) {
+                for (int c = r0 + h; c <= i; c += G) {
                     double acc = A[c * LDA + i];
 #pragma unroll
                     for (int q = 0; q < 16; q++) acc -= li[q] * A[(s0 + q) * LDA + c];
@@ -403,6 +404,13 @@ __global__ void __launch_bounds__(kPotrfThreads) k_potrf_diag(DevPlan d, const i
         }
         __syncthreads();
     }
+}
+
+__global__ void __launch_bounds__(kPotrfThreads) k_potrf_diag(DevPlan d, const int32_t *__restrict__ fronts,
+                                                              int j0, int w) {
+    __shared__ double A[kWmax * kWmax];
+    __shared__ double sinv[kWmax];
+    potrf_block<kPotrfThreads>(d, fronts[blockIdx.x], j0, w, A, sinv);
 }
 
 void launch_potrf_diag(const DevPlan &d, const int32_t *fronts, int count, int j0, int w, cudaStream_t st) {
@@ -425,25 +433,31 @@ constexpr size_t kTrsmSmem = (size_t)(kWmax * kLLD + kWmax * kXLD + kWmax) * siz
 // share rows, so only warp-level synchronisation is needed.  No explicit
 // inverse of L11: integer-exact on the manufactured inputs.  L11 and the row
 // block are staged with cp.async (all loads in flight at once).
-__global__ void __launch_bounds__(kTrsmThreads, 2) k_trsm_panel(DevPlan d, const int32_t *__restrict__ tasks,
-                                                                int j0, int w) {
-    extern __shared__ __align__(16) double tsm[];
+// wait until `flag` holds `expect` (written by the CTA that factored the diagonal
+// block, after a fence); used by the fused potrf+trsm leaf launch
+__device__ __forceinline__ void wait_flag(const unsigned *flag, unsigned expect) {
+    if (threadIdx.x == 0) {
+        unsigned v;
+        do {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(flag) : "memory");
+            if (v != expect) __nanosleep(200);
+        } while (v != expect);
+    }
+    __syncthreads();
+}
+
+__device__ __forceinline__ void trsm_block(const DevPlan &d, int s, int r0, int j0, int w, double *tsm,
+                                           const unsigned *flag, unsigned expect) {
     double *Ls = tsm;                           // L11[r][c] at Ls[r + c * kLLD]
     double *X = tsm + kWmax * kLLD;             // X[r][c]   at X[r + c * kXLD]
     double *inv = X + kWmax * kXLD;
-    const int s = tasks[2 * blockIdx.x], r0 = tasks[2 * blockIdx.x + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s];
     const int we = min(w, k - j0);
     const int nr = min(kTrsmRows, f - r0);
     const double *__restrict__ D = d.L + d.L_off[s] + (int64_t)j0 * ld + j0;   // 16B aligned: j0 even, ld even
     double *__restrict__ B = d.L + d.L_off[s] + (int64_t)j0 * ld + r0;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    // L11: 64 x we, pairs of rows per 16-byte chunk (rows >= we padded below)
-    for (int q = tid; q < (kWmax / 2) * kWmax; q += kTrsmThreads) {
-        const int rr = 2 * (q % (kWmax / 2)), c = q / (kWmax / 2);
-        const bool ok = c < we && rr < we;
-        cp_async16(Ls + rr + c * kLLD, ok ? D + rr + (int64_t)c * ld : D, ok);
-    }
+    // the row block first (independent of the diagonal block) ...
     if ((r0 & 1) == 0) {
         for (int q = tid; q < (kTrsmRows / 2) * kWmax; q += kTrsmThreads) {
             const int rr = 2 * (q % (kTrsmRows / 2)), c = q / (kTrsmRows / 2);
@@ -455,6 +469,16 @@ __global__ void __launch_bounds__(kTrsmThreads, 2) k_trsm_panel(DevPlan d, const
             const bool ok = c < we && tid < nr;
             cp_async8(X + tid + c * kXLD, ok ? B + tid + (int64_t)c * ld : B, ok);
         }
+    }
+    cp_async_commit();
+    // ... then L11 (64 x we, pairs of rows per 16-byte chunk; rows >= we padded below),
+    // once the diagonal block is final (fused leaf launch: wait for its flag; the
+    // 16-byte cp.async.cg path reads L2, never a stale L1 line)
+    if (flag) wait_flag(flag, expect);
+    for (int q = tid; q < (kWmax / 2) * kWmax; q += kTrsmThreads) {
+        const int rr = 2 * (q % (kWmax / 2)), c = q / (kWmax / 2);
+        const bool ok = c < we && rr < we;
+        cp_async16(Ls + rr + c * kLLD, ok ? D + rr + (int64_t)c * ld : D, ok);
     }
     cp_async_commit();
     cp_async_wait<0>();
@@ -514,6 +538,42 @@ __global__ void __launch_bounds__(kTrsmThreads, 2) k_trsm_panel(DevPlan d, const
         if (tid < nr) B[tid + (int64_t)c * ld] = X[tid + c * kXLD];
 }
 
+__global__ void __launch_bounds__(kTrsmThreads, 2) k_trsm_panel(DevPlan d, const int32_t *__restrict__ tasks,
+                                                                int j0, int w) {
+    extern __shared__ __align__(16) double tsm[];
+    trsm_block(d, tasks[2 * blockIdx.x], tasks[2 * blockIdx.x + 1], j0, w, tsm, nullptr, 0);
+}
+
+// Fused leaf: blocks [0, npotrf) factor the diagonal blocks of the active fronts
+// (then publish a per-front flag), blocks [npotrf, ...) solve the row blocks below;
+// each TRSM block stages its rows, waits for its front's flag, then loads L11.
+// The diagonal-block CTAs have the lowest block indices, so they are dispatched
+// first and never wait: no deadlock.  Saves one launch (and the row-block load
+// latency) per leaf on the sequential chain of the top fronts.
+__global__ void __launch_bounds__(kTrsmThreads, 2) k_leaf(DevPlan d, const int32_t *__restrict__ fronts, int npotrf,
+                                                          const int32_t *__restrict__ tasks, int j0, int w) {
+    extern __shared__ __align__(16) double tsm[];
+    const unsigned expect = ((*d.epoch & 0x3fffffu) << 10) | (unsigned)(j0 / w + 1);   // w >= 16: < 1024 leaves
+    if ((int)blockIdx.x < npotrf) {
+        const int s = fronts[blockIdx.x];
+        potrf_block<kTrsmThreads>(d, s, j0, w, tsm, tsm + kWmax * kWmax);
+        __threadfence();
+        __syncthreads();
+        if (threadIdx.x == 0)
+            asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(d.leaf_flag + s), "r"(expect) : "memory");
+        return;
+    }
+    const int t = blockIdx.x - npotrf;
+    const int s = tasks[2 * t];
+    trsm_block(d, s, tasks[2 * t + 1], j0, w, tsm, d.leaf_flag + s, expect);
+}
+
+void launch_leaf(const DevPlan &d, const int32_t *fronts, int npotrf, const int32_t *tasks, int64_t ntrsm, int j0,
+                 int w, cudaStream_t st) {
+    if (npotrf <= 0) return;
+    k_leaf<<<(unsigned)(npotrf + ntrsm), kTrsmThreads, kTrsmSmem, st>>>(d, fronts, npotrf, tasks, j0, w);
+}
+
 void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, cudaStream_t st) {
     if (count <= 0) return;
     k_trsm_panel<<<(unsigned)count, kTrsmThreads, kTrsmSmem, st>>>(d, tasks, j0, w);
@@ -529,7 +589,7 @@ void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tile
     k_update_t<UpdProd><<<(unsigned)ntiles, UpdProd::NT, UpdProd::SMEM, st>>>(d.L, d.U, probs, tiles);
 }
 
-void launch_init_failed(int *failed, cudaStream_t st) { k_init_failed<<<1, 1, 0, st>>>(failed); }
+void launch_init_failed(int *failed, cudaStream_t st) { k_init_failed<<<1, 1, 0, st>>>(failed, reinterpret_cast<unsigned *>(failed + 1)); }
 
 // Kernel attributes (dynamic shared memory above 48 KB), set once per device
 // before any launch -- in particular before the factorization is captured
@@ -539,6 +599,8 @@ int kernels_init() {
     e = cudaFuncSetAttribute(k_small_front<256>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     if (e == cudaSuccess)
         e = cudaFuncSetAttribute(k_trsm_panel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTrsmSmem);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_leaf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTrsmSmem);
     if (e == cudaSuccess)
         e = cudaFuncSetAttribute(k_update_t<UpdProd>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)UpdProd::SMEM);
     return e == cudaSuccess ? 0 : -1;

@@ -23,6 +23,8 @@ struct DevPlan {
     const int64_t *bvidx;
     const int32_t *perm;     // final perm (new -> old)
     int *failed;             // min failing pivot column (final labels); INT_MAX = none
+    const unsigned *epoch;   // factorization counter (= failed + 1), bumped by the init kernel
+    unsigned *leaf_flag;     // per supernode: fused-leaf "diagonal block done" flag
 };
 
 // launchers (all asynchronous on `st`)
@@ -30,6 +32,8 @@ void launch_init_failed(int *failed, cudaStream_t st);
 void launch_small_fronts(const DevPlan &d, const int32_t *list, int count, int fmax, const double *values,
                          cudaStream_t st);
 void launch_assemble(const DevPlan &d, const int32_t *tasks, int64_t count, const double *values, cudaStream_t st);
+void launch_leaf(const DevPlan &d, const int32_t *fronts, int npotrf, const int32_t *tasks, int64_t ntrsm, int j0,
+                 int w, cudaStream_t st);
 void launch_potrf_diag(const DevPlan &d, const int32_t *fronts, int count, int j0, int w, cudaStream_t st);
 void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, cudaStream_t st);
 void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, cudaStream_t st);

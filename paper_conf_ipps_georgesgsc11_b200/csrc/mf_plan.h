@@ -75,8 +75,10 @@ enum KernelClass : int32_t {
     KC_POTRF = 2,     // w x w diagonal-block potrf
     KC_TRSM = 3,      // panel trsm below the diagonal block
     KC_UPDATE = 4,    // DMMA Schur update (panel trailing update and the syrk on U^n)
-    KC_COUNT = 5
+    KC_LEAF = 5,      // fused potrf + trsm of one diagonal block (few active fronts)
+    KC_COUNT = 6
 };
+constexpr int kFuseLeafMaxFronts = 8;
 
 struct Launch {
     int32_t kind;       // KernelClass
@@ -85,6 +87,7 @@ struct Launch {
     double flops;       // algorithmic flops of this launch
     double bytes;       // algorithmic HBM bytes of this launch
     int32_t level;
+    int64_t off2 = 0, count2 = 0;   // KC_LEAF: the trsm tasks (off/count = the fronts)
 };
 
 // Triangular-solve program (forward sweep bottom-up, backward sweep top-down).

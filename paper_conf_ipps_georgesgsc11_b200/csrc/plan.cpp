@@ -401,6 +401,13 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
                     Lt.bytes += 8.0 * (2 * rows * we + (double)we * (we + 1) / 2);
                 }
                 Lt.count = (int64_t)P.trsm_tasks.size() / 2 - Lt.off;
+                if (na <= kFuseLeafMaxFronts && Lt.count) {   // one launch: potrf CTAs + flag-waiting trsm CTAs
+                    Launch Lf{KC_LEAF, j0, Lp.off, Lp.count, Lp.flops + Lt.flops, Lp.bytes + Lt.bytes, l};
+                    Lf.off2 = Lt.off;
+                    Lf.count2 = Lt.count;
+                    cur->push_back(Lf);
+                    return;
+                }
                 cur->push_back(Lp);
                 if (Lt.count) cur->push_back(Lt);
                 return;

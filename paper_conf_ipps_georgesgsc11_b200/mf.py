@@ -57,7 +57,7 @@ class KernelStat(ctypes.Structure):
                 ("flops", ctypes.c_double), ("bytes", ctypes.c_double)]
 
 
-MF_KERNEL_CLASSES = 5
+MF_KERNEL_CLASSES = 6
 
 MF_XFER_SEND, MF_XFER_RECV, MF_XFER_BCAST, MF_XFER_ALLREDUCE_SUM, MF_XFER_ALLREDUCE_MIN_I32 = 1, 2, 3, 4, 5
 
