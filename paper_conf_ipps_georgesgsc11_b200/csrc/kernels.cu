@@ -183,13 +183,92 @@ __global__ void __launch_bounds__(NT) k_small_front(DevPlan d, const int32_t *__
     }
 }
 
+// ============================================================ tiny fronts (f <= 32)
+// One WARP per front (4 fronts per CTA), no block barriers: the front is
+// assembled in a per-warp shared-memory tile (zero, A entries, children's U^c
+// in ascending order), then lane i holds row i in registers and the k pivots
+// are eliminated right-looking with shuffles over the WHOLE front, which
+// yields L1, L2 and U^n = F22 - L2 L2^T together.  c2 (9-point 1000^2) has
+// ~230k such fronts.
+constexpr int kTinyF = 32, kTinyWarps = 4;
+template <int TF>
+__global__ void __launch_bounds__(32 * kTinyWarps, TF <= 16 ? 8 : 4)
+    k_tiny_fronts(DevPlan d, const int32_t *__restrict__ list, int count, const double *__restrict__ values) {
+    constexpr int kTinyLD = TF + 1;
+    __shared__ double Fs[kTinyWarps][TF * kTinyLD];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int idx = blockIdx.x * kTinyWarps + warp;
+    if (idx >= count) return;
+    double *F = Fs[warp];
+    const int s = list[idx];
+    const int k = d.sn_k[s], f = d.sn_f[s], m = f - k, first = d.sn_first[s];
+    if (lane < TF)
+        for (int c = 0; c < f; c++) F[lane + c * kTinyLD] = 0.0;
+    __syncwarp();
+    for (int j = 0; j < k; j++) {
+        const int64_t e0 = d.bcolptr[first + j], e1 = d.bcolptr[first + j + 1];
+        for (int64_t e = e0 + lane; e < e1; e += 32) F[d.blrow[e] + j * kTinyLD] = sum_values(d, values, e);
+    }
+    __syncwarp();
+    for (int q = d.child_ptr[s]; q < d.child_ptr[s + 1]; q++) {
+        const int c = d.child_list[q];
+        const int mc = d.sn_f[c] - d.sn_k[c];
+        const int32_t *__restrict__ rel = d.relmap + d.relmap_ptr[c];
+        const double *__restrict__ Uc = d.U + d.U_off[c];
+        const int myrel = lane < mc ? rel[lane] : 0;
+        for (int qq = 0; qq < mc; qq++) {
+            const int dc = __shfl_sync(0xffffffffu, myrel, qq);
+            if (lane >= qq && lane < mc) F[myrel + dc * kTinyLD] += Uc[lane + qq * mc];
+        }
+        __syncwarp();
+    }
+    double a[TF];
+#pragma unroll
+    for (int c = 0; c < TF; c++) a[c] = lane < TF ? F[lane + c * kTinyLD] : 0.0;
+#pragma unroll
+    for (int j = 0; j < TF; j++) {
+        if (j < k) {
+            const double dj = __shfl_sync(0xffffffffu, a[j], j);
+            const double inv = rsqrt(dj);
+            if (lane == j) {
+                note_pivot(d, dj, first + j);
+                a[j] = dj * inv;
+            } else if (lane > j) {
+                a[j] *= inv;
+            }
+#pragma unroll
+            for (int c = j + 1; c < TF; c++) {
+                const double lc = __shfl_sync(0xffffffffu, a[j], c);
+                if (lane >= c && c < f) a[c] -= a[j] * lc;
+            }
+        }
+    }
+    if (lane < f) {
+        double *__restrict__ P = d.L + d.L_off[s];
+        const int ld = d.sn_ld[s];
+#pragma unroll
+        for (int j = 0; j < TF; j++)
+            if (j < k) P[lane + (int64_t)j * ld] = lane >= j ? a[j] : 0.0;
+        if (m > 0) {
+            double *__restrict__ Us = d.U + d.U_off[s] - k - (int64_t)k * m;   // Us[(i-k) + (c-k) m]
+#pragma unroll
+            for (int c = 0; c < TF; c++)
+                if (c >= k && c < f && lane >= c) Us[lane + (int64_t)c * m] = a[c];
+        }
+    }
+}
+
 int small_front_smem_ok(int fmax) { return (size_t)(fmax * fmax + fmax) * sizeof(double) <= 227 * 1024; }
 
 void launch_small_fronts(const DevPlan &d, const int32_t *list, int count, int fmax, const double *values,
                          cudaStream_t st) {
     if (count <= 0) return;
     const size_t smem = (size_t)(fmax * fmax + fmax) * sizeof(double);
-    if (fmax <= 32) {
+    if (fmax <= 16) {
+        k_tiny_fronts<16><<<(count + kTinyWarps - 1) / kTinyWarps, 32 * kTinyWarps, 0, st>>>(d, list, count, values);
+    } else if (fmax <= kTinyF) {
+        k_tiny_fronts<32><<<(count + kTinyWarps - 1) / kTinyWarps, 32 * kTinyWarps, 0, st>>>(d, list, count, values);
+    } else if (fmax <= 32) {
         k_small_front<64><<<count, 64, smem, st>>>(d, list, values);
     } else if (fmax <= 64) {
         k_small_front<128><<<count, 128, smem, st>>>(d, list, values);

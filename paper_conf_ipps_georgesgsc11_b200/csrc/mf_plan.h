@@ -147,7 +147,7 @@ struct Plan {
 constexpr int kTileM = 64, kTileN = 64;
 constexpr int kAsmCols = 16;
 constexpr int kTrsmRows = 128;
-constexpr int kSmallClasses = 3;
+constexpr int kSmallClasses = 4;
 constexpr int kSolveRows = 256;
 
 int build_plan(const Symbolic &S, const Options &opt, Plan &P);

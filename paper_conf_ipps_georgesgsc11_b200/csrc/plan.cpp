@@ -286,7 +286,9 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         for (int32_t s = 0; s < ns; s++) P.level_list[fill[P.sn_level[s]]++] = s;
     }
     // small-front classes: f <= small_max/4, <= small_max/2, <= small_max
-    P.small_class_fmax = {std::max(8, P.small_max / 4), std::max(16, P.small_max / 2), P.small_max};
+    // (<= 16 and <= 32: one warp per front; <= 64 and <= small_max: one CTA per front)
+    P.small_class_fmax = {std::min(16, P.small_max), std::min(32, P.small_max), std::min(64, P.small_max),
+                          P.small_max};
     const int w = P.w;
     // algorithmic bytes of assembling front s: its A entries (value + index), the
     // children's U^c lower triangles and relative maps (read once)
