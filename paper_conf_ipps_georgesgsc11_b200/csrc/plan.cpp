@@ -23,14 +23,19 @@
 
 namespace mf {
 
+// Tiles are emitted in bands of kTileBand tile columns, row-major inside a band,
+// so the CTAs resident at one time cover a squarish block of the output and
+// share both operand row panels in L2.
+constexpr int32_t kTileBand = 16;
 static void add_tiles(Plan &P, int32_t prob, int32_t M, int32_t N) {
     const int32_t tm = (M + kTileM - 1) / kTileM, tn = (N + kTileN - 1) / kTileN;
-    for (int32_t tj = 0; tj < tn; tj++)
-        for (int32_t ti = 0; ti < tm; ti++) {
-            // lower-trapezoid: skip tiles entirely above the diagonal (i < j everywhere)
-            if ((int64_t)(ti + 1) * kTileM - 1 < (int64_t)tj * kTileN) continue;
-            P.tiles.push_back({prob, (ti << 16) | tj});
-        }
+    for (int32_t tj0 = 0; tj0 < tn; tj0 += kTileBand)
+        for (int32_t ti = 0; ti < tm; ti++)
+            for (int32_t tj = tj0; tj < std::min(tn, tj0 + kTileBand); tj++) {
+                // lower-trapezoid: skip tiles entirely above the diagonal (i < j everywhere)
+                if ((int64_t)(ti + 1) * kTileM - 1 < (int64_t)tj * kTileN) continue;
+                P.tiles.push_back({prob, (ti << 16) | tj});
+            }
 }
 
 // Solve program: per level, small supernodes in one batched launch; large ones
