@@ -50,8 +50,8 @@ struct mf_ctx {
     int64_t launches = 0;
     bool profiling = false;
     bool use_graph = true;
-    cudaGraph_t graph = nullptr, graph_top = nullptr;
-    cudaGraphExec_t graph_exec = nullptr, graph_top_exec = nullptr;
+    cudaGraph_t graph = nullptr, graph_top = nullptr, solve_graph = nullptr;
+    cudaGraphExec_t graph_exec = nullptr, graph_top_exec = nullptr, solve_exec = nullptr;
     mf_exchange_fn xfn = nullptr;
     void *xuser = nullptr;
     double *d_ytmp = nullptr;
@@ -103,6 +103,10 @@ void drop_graph(mf_ctx *c) {
     c->graph = nullptr;
     c->graph_top_exec = nullptr;
     c->graph_top = nullptr;
+    if (c->solve_exec) cudaGraphExecDestroy(c->solve_exec);
+    if (c->solve_graph) cudaGraphDestroy(c->solve_graph);
+    c->solve_exec = nullptr;
+    c->solve_graph = nullptr;
 }
 
 void free_device(mf_ctx *c) {
@@ -554,6 +558,36 @@ int mf_solve(mf_ctx *c, const double *b, double *x) {
     const bool multi = P.nranks > 1;
     CK(cudaEventRecord(c->ev0, st));
     const bool bdev = is_device_ptr(b), xdev = is_device_ptr(x);
+    if (!multi && c->use_graph) {
+        // single GPU: the whole solve is one CUDA graph over the ctx buffers
+        // (b -> d_bx, permute, forward, backward, permute back into d_bx -> x)
+        CK(cudaMemcpyAsync(c->d_bx, b, n * sizeof(double), bdev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice,
+                           st));
+        if (!c->solve_exec) {
+            CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
+            launch_permute_in(d, c->d_bx, c->d_y, n, st);
+            cudaError_t e1 = cudaMemsetAsync(c->d_counters, 0, (P.sb_groups.size() / 2 + 1) * sizeof(int), st);
+            run_solve_program(c, P.fsolve);
+            run_solve_program(c, P.bsolve);
+            launch_permute_out(d, c->d_y, c->d_bx, n, st);
+            cudaGraph_t g = nullptr;
+            cudaError_t e2 = cudaStreamEndCapture(st, &g);
+            CK(e1);
+            CK(e2);
+            c->solve_graph = g;
+            CK(cudaGraphInstantiate(&c->solve_exec, g, 0));
+        }
+        CK(cudaGraphLaunch(c->solve_exec, st));
+        CK(cudaMemcpyAsync(x, c->d_bx, n * sizeof(double), xdev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
+                           st));
+        CK(cudaGetLastError());
+        CK(cudaEventRecord(c->ev1, st));
+        CK(cudaStreamSynchronize(st));
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, c->ev0, c->ev1);
+        c->info.t_solve = ms * 1e-3;
+        return MF_OK;
+    }
     const double *bd = b;
     if (!bdev) {
         CK(cudaMemcpyAsync(c->d_bx, b, n * sizeof(double), cudaMemcpyHostToDevice, st));
