@@ -43,9 +43,7 @@ struct mf_ctx {
     double *d_values = nullptr;
     double *d_y = nullptr, *d_bx = nullptr;
     int *d_failed = nullptr;
-    int32_t *d_solve_list = nullptr, *d_sf_tasks = nullptr, *d_sb_tasks = nullptr, *d_sb_groups = nullptr;
-    double *d_partials = nullptr;
-    int *d_counters = nullptr;
+    int32_t *d_solve_list = nullptr, *d_df_tasks = nullptr;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     int64_t launches = 0;
     bool profiling = false;
@@ -315,9 +313,10 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     UP(&c->d_probs, P.probs);
     UP(&c->d_tiles, P.tiles);
     UP(&c->d_solve_list, P.solve_list);
-    UP(&c->d_sf_tasks, P.sf_tasks);
-    UP(&c->d_sb_tasks, P.sb_tasks);
-    UP(&c->d_sb_groups, P.sb_groups);
+    UP(&c->d_df_tasks, P.df_tasks);
+    int64_t *df_blk_off = nullptr, *df_part_off = nullptr;
+    UP(&df_blk_off, P.df_blk_off);
+    UP(&df_part_off, P.df_part_off);
     UP(&c->d_top_list, P.top_list);
     UP(&c->d_own_list, P.own_list);
 #undef UP
@@ -337,6 +336,8 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     d.bvptr = bvptr;
     d.bvidx = bvidx;
     d.perm = perm_d;
+    d.df_blk_off = df_blk_off;
+    d.df_part_off = df_part_off;
     void *p;
     if ((r = dev_alloc(c, &p, P.L_words * sizeof(double))) != MF_OK) return r;
     d.L = (double *)p;
@@ -346,12 +347,14 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     d.fv = (double *)p;
     if ((r = dev_alloc(c, &p, sizeof(int) * 4)) != MF_OK) return r;
     c->d_failed = (int *)p;
-    if ((r = dev_alloc(c, &p, (P.sb_tasks.size() / 3 + 1) * 64 * sizeof(double))) != MF_OK) return r;
-    c->d_partials = (double *)p;
-    if ((r = dev_alloc(c, &p, (P.sb_groups.size() / 2 + 1) * sizeof(int))) != MF_OK) return r;
-    c->d_counters = (int *)p;
+    if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.df_nparts, 1) * sizeof(double))) != MF_OK) return r;
+    d.df_parts = (double *)p;
+    if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.df_nflags, 1) * sizeof(unsigned))) != MF_OK) return r;
+    d.df_flags = (unsigned *)p;
+    CK(cudaMemsetAsync(d.df_flags, 0, (size_t)std::max<int64_t>(P.df_nflags, 1) * sizeof(unsigned), c->stream));
     d.failed = c->d_failed;
     d.epoch = reinterpret_cast<const unsigned *>(c->d_failed + 1);
+    d.solve_epoch = reinterpret_cast<unsigned *>(c->d_failed + 2);
     if ((r = dev_alloc(c, &p, std::max<int32_t>(P.nsuper, 1) * sizeof(unsigned))) != MF_OK) return r;
     d.leaf_flag = (unsigned *)p;
     CK(cudaMemsetAsync(d.leaf_flag, 0, std::max<int32_t>(P.nsuper, 1) * sizeof(unsigned), c->stream));
@@ -531,17 +534,14 @@ void run_solve_program(mf_ctx *c, const std::vector<SolveLaunch> &prog) {
         switch (L.kind) {
             case SK_SMALL_F: launch_fwd_solve(d, c->d_solve_list + L.off, (int)L.count, c->d_y, st); break;
             case SK_INIT_F: launch_fsolve_init(d, c->d_solve_list + L.off, (int)L.count, c->d_y, st); break;
-            case SK_WAVE_F: launch_fsolve_wave(d, c->d_sf_tasks + 3 * L.off, L.count, L.j0, P.w, c->d_y, st); break;
+            case SK_DF_F: launch_fsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, c->d_y, st); break;
             case SK_SMALL_B:
                 launch_bwd_solve(d, c->d_solve_list + L.off, (int)L.count, c->d_y, c->d_sn_rows, c->d_sn_rowptr, st);
                 break;
             case SK_INIT_B:
                 launch_bsolve_init(d, c->d_solve_list + L.off, (int)L.count, c->d_y, c->d_sn_rows, c->d_sn_rowptr, st);
                 break;
-            case SK_WAVE_B:
-                launch_bsolve_wave(d, c->d_sb_tasks + 3 * L.off, L.off, L.count, c->d_sb_groups, L.j0, P.w, c->d_y,
-                                   c->d_partials, c->d_counters, st);
-                break;
+            case SK_DF_B: launch_bsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, c->d_y, st); break;
         }
     }
 }
@@ -566,13 +566,11 @@ int mf_solve(mf_ctx *c, const double *b, double *x) {
         if (!c->solve_exec) {
             CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
             launch_permute_in(d, c->d_bx, c->d_y, n, st);
-            cudaError_t e1 = cudaMemsetAsync(c->d_counters, 0, (P.sb_groups.size() / 2 + 1) * sizeof(int), st);
             run_solve_program(c, P.fsolve);
             run_solve_program(c, P.bsolve);
             launch_permute_out(d, c->d_y, c->d_bx, n, st);
             cudaGraph_t g = nullptr;
             cudaError_t e2 = cudaStreamEndCapture(st, &g);
-            CK(e1);
             CK(e2);
             c->solve_graph = g;
             CK(cudaGraphInstantiate(&c->solve_exec, g, 0));
@@ -594,7 +592,6 @@ int mf_solve(mf_ctx *c, const double *b, double *x) {
         bd = c->d_bx;
     }
     launch_permute_in(d, bd, c->d_y, n, st);
-    CK(cudaMemsetAsync(c->d_counters, 0, (P.sb_groups.size() / 2 + 1) * sizeof(int), st));
     int r;
     run_solve_program(c, P.fsolve);                  // forward, own subtrees
     if (multi) {

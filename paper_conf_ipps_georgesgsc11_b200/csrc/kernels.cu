@@ -731,7 +731,11 @@ void launch_export_diag(const DevPlan &d, int nsuper, double *out, cudaStream_t 
 // per-front update vectors that the parent gathers through the same relative
 // maps as the extend-add (deterministic, no atomics).
 __global__ void k_permute_in(const int32_t *__restrict__ perm, const double *__restrict__ b, double *__restrict__ y,
-                             int64_t n) {
+                             int64_t n, unsigned *solve_epoch) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) {   // 20 bits (backward flags carry a 12-bit block counter); never 0
+        const unsigned e = (*solve_epoch + 1) & 0xfffffu;
+        *solve_epoch = e ? e : 1u;
+    }
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         y[i] = b[perm[i]];
 }
@@ -741,7 +745,7 @@ __global__ void k_permute_out(const int32_t *__restrict__ perm, const double *__
         x[perm[i]] = xf[i];
 }
 void launch_permute_in(const DevPlan &d, const double *b, double *y, int64_t n, cudaStream_t st) {
-    if (n > 0) k_permute_in<<<(unsigned)((n + 255) / 256 < 4096 ? (n + 255) / 256 : 4096), 256, 0, st>>>(d.perm, b, y, n);
+    if (n > 0) k_permute_in<<<(unsigned)((n + 255) / 256 < 4096 ? (n + 255) / 256 : 4096), 256, 0, st>>>(d.perm, b, y, n, d.solve_epoch);
 }
 void launch_permute_out(const DevPlan &d, const double *xf, double *x, int64_t n, cudaStream_t st) {
     if (n > 0) k_permute_out<<<(unsigned)((n + 255) / 256 < 4096 ? (n + 255) / 256 : 4096), 256, 0, st>>>(d.perm, xf, x, n);
@@ -826,44 +830,6 @@ __global__ void __launch_bounds__(kSolveThreads) k_fsolve_init(DevPlan d, const 
 
 constexpr int kSW = 64, kSLD = 65;   // solve block width and smem leading dimension
 
-__device__ __forceinline__ void load_diag_block(const double *__restrict__ P, int ld, int j0, int we,
-                                                double *__restrict__ Lb) {
-    for (int c = threadIdx.x >> 6; c < we; c += kSolveThreads / 64) {
-        const int r = threadIdx.x & 63;
-        if (r < we && r >= c) Lb[r + c * kSLD] = P[(j0 + r) + (int64_t)(j0 + c) * ld];
-    }
-}
-
-__global__ void __launch_bounds__(kSolveThreads) k_fsolve_wave(DevPlan d, const int32_t *__restrict__ tasks, int j0,
-                                                               int w, double *__restrict__ y) {
-    __shared__ double Lb[kSW * kSLD];
-    __shared__ double xs[kSW];
-    const int s = tasks[3 * blockIdx.x], row0 = tasks[3 * blockIdx.x + 1], writer = tasks[3 * blockIdx.x + 2];
-    const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
-    const int we = min(w, k - j0);
-    const double *__restrict__ P = d.L + d.L_off[s];
-    double *__restrict__ v = d.fv + d.fv_off[s];
-    const int tid = threadIdx.x, lane = tid & 31;
-    load_diag_block(P, ld, j0, we, Lb);
-    __syncthreads();
-    if (tid < 32) {   // L11 x = v[j0:j0+we], right-looking, two entries per lane
-        double a0 = lane < we ? v[j0 + lane] : 0.0, a1 = lane + 32 < we ? v[j0 + lane + 32] : 0.0;
-        for (int c = 0; c < we; c++) {
-            const double xc = __shfl_sync(0xffffffffu, c < 32 ? a0 : a1, c & 31) / Lb[c + c * kSLD];
-            if (lane == 0) xs[c] = xc;
-            if (lane > c && lane < we) a0 -= Lb[lane + c * kSLD] * xc;
-            if (lane + 32 > c && lane + 32 < we) a1 -= Lb[lane + 32 + c * kSLD] * xc;
-        }
-    }
-    __syncthreads();
-    if (writer && tid < we) y[first + j0 + tid] = xs[tid];
-    const int r = row0 + tid;
-    if (r < min(row0 + kSolveRows, f)) {
-        double acc = v[r];
-        for (int c = 0; c < we; c++) acc -= P[r + (int64_t)(j0 + c) * ld] * xs[c];
-        v[r] = acc;
-    }
-}
 
 __global__ void __launch_bounds__(kSolveThreads) k_bsolve_init(DevPlan d, const int32_t *__restrict__ list,
                                                                const double *__restrict__ y,
@@ -876,88 +842,247 @@ __global__ void __launch_bounds__(kSolveThreads) k_bsolve_init(DevPlan d, const 
     for (int i = k + threadIdx.x; i < f; i += kSolveThreads) v[i] = y[R[i]];
 }
 
-__global__ void __launch_bounds__(kSolveThreads) k_bsolve_wave(DevPlan d, const int32_t *__restrict__ tasks,
-                                                               int64_t task_base, const int32_t *__restrict__ groups,
-                                                               int j0, int w, double *__restrict__ y,
-                                                               double *__restrict__ partials, int *__restrict__ counters) {
-    __shared__ double red[kSolveThreads / 32][kSW];
+// ---- dataflow solves: one launch per level for all its large supernodes.  CTA =
+// one 256-row chunk of one front, one row per thread (value in a register).
+// Forward: for each 64-column block b in order, the chunk that holds the block's
+// rows solves its triangle and publishes x_b (flag = solve epoch); every chunk
+// below applies v -= L(rows, b) x_b.  Backward: for each block b in reverse, every
+// chunk below the block publishes its partial L(rows, b)^T x(rows); the owner
+// sums them in a fixed chunk order (deterministic) and solves L_bb^T x_b = t.
+// CTAs are ordered so that a chunk only waits on lower CTA ids.
+__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned *p) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_u32(unsigned *p, unsigned v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// Row r's 64 entries of the column block [j0, j0 + we), zero past we (independent
+// loads: the whole slab is in flight at once).
+__device__ __forceinline__ void load_row_block(const double *__restrict__ P, int64_t ld, int r, int j0, int we,
+                                               bool ok, double (&Lr)[kSW]) {
+    const double *__restrict__ col = P + (int64_t)j0 * ld + r;
+#pragma unroll
+    for (int q = 0; q < kSW; q++) Lr[q] = (ok && q < we) ? col[(int64_t)q * ld] : 0.0;
+}
+
+// Row i of the diagonal block (held in a row slab, entries q <= i) into shared
+// memory, its pivot's reciprocal into dinv, and xv into xs[i]; the slab row is
+// then zeroed so that the row takes no part in the block's off-diagonal product.
+__device__ __forceinline__ void stash_diag_row(double (&Lr)[kSW], int i, double xv, double *__restrict__ Lb,
+                                               double *__restrict__ dinv, double *__restrict__ xs) {
+    double dd = 1.0;
+#pragma unroll
+    for (int q = 0; q < kSW; q++) {
+        if (q <= i) Lb[i + q * kSLD] = Lr[q];
+        if (q == i) dd = Lr[q];
+        Lr[q] = 0.0;
+    }
+    dinv[i] = 1.0 / dd;
+    xs[i] = xv;
+}
+
+
+// One warp: x = L_bb^{-1} t (forward, right-looking) with t in (a0, a1) = entries
+// lane, lane + 32.
+__device__ __forceinline__ void warp_trsv_fwd(const double *__restrict__ Lb, const double *__restrict__ dinv, int we,
+                                              double &a0, double &a1) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll 8
+    for (int q = 0; q < we; q++) {
+        const double xq = __shfl_sync(0xffffffffu, q < 32 ? a0 : a1, q & 31) * dinv[q];
+        if (lane == (q & 31)) {
+            if (q < 32) a0 = xq; else a1 = xq;
+        }
+        if (lane > q && lane < we) a0 -= Lb[lane + q * kSLD] * xq;
+        if (lane + 32 > q && lane + 32 < we) a1 -= Lb[lane + 32 + q * kSLD] * xq;
+    }
+}
+// One warp: x = L_bb^{-T} t (backward, right-looking on the transpose).
+__device__ __forceinline__ void warp_trsv_bwd(const double *__restrict__ Lb, const double *__restrict__ dinv, int we,
+                                              double &a0, double &a1) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll 8
+    for (int q = we - 1; q >= 0; q--) {
+        const double xq = __shfl_sync(0xffffffffu, q < 32 ? a0 : a1, q & 31) * dinv[q];
+        if (lane == (q & 31)) {
+            if (q < 32) a0 = xq; else a1 = xq;
+        }
+        if (lane < q) a0 -= Lb[q + lane * kSLD] * xq;
+        if (lane + 32 < q) a1 -= Lb[q + (lane + 32) * kSLD] * xq;
+    }
+}
+
+__global__ void __launch_bounds__(kSolveThreads) k_fsolve_df(DevPlan d, const int32_t *__restrict__ tasks, int w,
+                                                             double *__restrict__ y) {
     __shared__ double Lb[kSW * kSLD];
-    __shared__ double tv[kSW];
-    __shared__ int is_last;
-    const int s = tasks[3 * blockIdx.x], row0 = tasks[3 * blockIdx.x + 1], grp = tasks[3 * blockIdx.x + 2];
+    __shared__ double xs[kSW], dinv[kSW];
+    const int s = tasks[2 * blockIdx.x], c = tasks[2 * blockIdx.x + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
-    const int we = min(w, k - j0);
     const double *__restrict__ P = d.L + d.L_off[s];
     double *__restrict__ v = d.fv + d.fv_off[s];
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    // partial (L2^T v)_c over this CTA's row chunk
-    const int r = row0 + tid;
-    const bool rok = r < min(row0 + kSolveRows, f);
-    const double rv = rok ? v[r] : 0.0;
-    for (int c = 0; c < we; c++) {
-        double p = rok ? P[r + (int64_t)(j0 + c) * ld] * rv : 0.0;
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) p += __shfl_xor_sync(0xffffffffu, p, o);
-        if (lane == 0) red[warp][c] = p;
-    }
-    __syncthreads();
-    if (tid < we) {
-        double t = 0.0;
-        for (int q = 0; q < kSolveThreads / 32; q++) t += red[q][tid];
-        partials[(task_base + blockIdx.x) * kSW + tid] = t;
-    }
-    __threadfence();
-    __syncthreads();
-    if (tid == 0) is_last = atomicAdd(&counters[grp], 1) == groups[2 * grp + 1] - 1;
-    __syncthreads();
-    if (!is_last) return;
-    __threadfence();
-    // the last CTA of the group reduces the partials in task order (deterministic) and solves L11^T x = t
-    load_diag_block(P, ld, j0, we, Lb);
-    if (tid < we) {
-        const int t0 = groups[2 * grp], nt = groups[2 * grp + 1];
-        double t = y[first + j0 + tid];
-        for (int q = 0; q < nt; q++) t -= __ldcg(&partials[(int64_t)(t0 + q) * kSW + tid]);
-        tv[tid] = t;
-    }
-    __syncthreads();
-    if (tid < 32) {
-        double a0 = lane < we ? tv[lane] : 0.0, a1 = lane + 32 < we ? tv[lane + 32] : 0.0;
-        for (int c = we - 1; c >= 0; c--) {
-            const double xc = __shfl_sync(0xffffffffu, c < 32 ? a0 : a1, c & 31) / Lb[c + c * kSLD];
-            if (lane == (c & 31)) {
-                if (c < 32) a0 = xc; else a1 = xc;
+    unsigned *__restrict__ bflag = d.df_flags + d.df_blk_off[s];
+    const unsigned epoch = *d.solve_epoch;
+    const int tid = threadIdx.x, lane = tid & 31;
+    const int c_lo = c * kSolveRows, c_hi = min(c_lo + kSolveRows, f);
+    const int r = c_lo + tid;
+    const bool rok = r < c_hi;
+    double vr = rok ? v[r] : 0.0;
+    const int nb = (k + w - 1) / w;
+    double Lr[kSW];
+    for (int b = 0; b < nb; b++) {
+        const int j0 = b * w, we = min(w, k - j0);
+        if (j0 >= c_hi) break;   // blocks below this chunk never update it
+        // this row's slab of the block (needs no x): issued before any wait; the
+        // owner's rows of the block carry the diagonal block itself
+        load_row_block(P, ld, r, j0, we, rok && r >= j0, Lr);
+        if (j0 >= c_lo) {        // this chunk owns the block: solve its triangle
+            const int i = r - j0;
+            if (rok && i >= 0 && i < we) stash_diag_row(Lr, i, vr, Lb, dinv, xs);
+            if (tid >= we && tid < kSW) xs[tid] = 0.0;
+            __syncthreads();
+            if (tid < 32) {
+                double a0 = xs[lane], a1 = xs[lane + 32];
+                warp_trsv_fwd(Lb, dinv, we, a0, a1);
+                xs[lane] = a0;
+                xs[lane + 32] = a1;
+                if (lane < we) y[first + j0 + lane] = a0;
+                if (lane + 32 < we) y[first + j0 + lane + 32] = a1;
+                __threadfence();
             }
-            if (lane < c) a0 -= Lb[c + lane * kSLD] * xc;
-            if (lane + 32 < c) a1 -= Lb[c + (lane + 32) * kSLD] * xc;
+            __syncthreads();
+            if (tid == 0) st_release_u32(bflag + b, epoch);
+            if (rok && i >= 0 && i < we) vr = xs[i];
+        } else {                 // a block above: wait for its solution
+            if (tid == 0)
+                while (ld_acquire_u32(bflag + b) != epoch) __nanosleep(32);
+            __syncthreads();
+            if (tid < kSW) xs[tid] = tid < we ? __ldcg(y + first + j0 + tid) : 0.0;   // (Lr = 0 past we; 0 * junk)
+            __syncthreads();
         }
-        if (lane < we) {
-            y[first + j0 + lane] = a0;
-            v[j0 + lane] = a0;
+        double a0 = 0.0, a1 = 0.0;
+#pragma unroll
+        for (int q = 0; q < kSW; q += 2) {
+            a0 += Lr[q] * xs[q];
+            a1 += Lr[q + 1] * xs[q + 1];
         }
-        if (lane + 32 < we) {
-            y[first + j0 + lane + 32] = a1;
-            v[j0 + lane + 32] = a1;
+        vr -= a0 + a1;           // rows not below the block have Lr = 0 (and xs past we is not read: Lr = 0)
+        __syncthreads();
+    }
+    if (rok && r >= k) v[r] = vr;   // the update vector the parent gathers
+}
+
+// Butterfly reduce-scatter over the warp: 64 values per lane in, lane l ends with
+// the warp sums of q = 2 l + {0, 1} in p[0], p[1] (62 shuffles).
+__device__ __forceinline__ void warp_reduce_scatter64(double (&p)[kSW]) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int st = 0; st < 5; st++) {
+        const int half = kSW >> (st + 1), off = 16 >> st;
+        const bool up = (lane & off) != 0;
+#pragma unroll
+        for (int i = 0; i < half; i++) {
+            const double send = up ? p[i] : p[i + half];
+            const double keep = up ? p[i + half] : p[i];
+            p[i] = keep + __shfl_xor_sync(0xffffffffu, send, off);
         }
+    }
+}
+
+__global__ void __launch_bounds__(kSolveThreads) k_bsolve_df(DevPlan d, const int32_t *__restrict__ tasks, int w,
+                                                             double *__restrict__ y) {
+    __shared__ double red[kSolveThreads / 32][kSW];
+    __shared__ double Lb[kSW * kSLD];
+    __shared__ double tv[kSW], dinv[kSW];
+    const int s = tasks[2 * blockIdx.x], c = tasks[2 * blockIdx.x + 1];
+    const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
+    const double *__restrict__ P = d.L + d.L_off[s];
+    double *__restrict__ v = d.fv + d.fv_off[s];
+    const int nb = (k + w - 1) / w, nc = (f + kSolveRows - 1) / kSolveRows;
+    unsigned *__restrict__ cflag = d.df_flags + d.df_blk_off[s] + nb;
+    double *__restrict__ part = d.df_parts + d.df_part_off[s];
+    const unsigned epoch = *d.solve_epoch;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int c_lo = c * kSolveRows, c_hi = min(c_lo + kSolveRows, f);
+    const int r = c_lo + tid;
+    const bool rok = r < c_hi;
+    const int qlane = 2 * lane;
+    double xr = (rok && r >= k) ? v[r] : 0.0;   // rows >= k: final (gathered from the ancestors)
+    double pr[kSW];
+    for (int b = nb - 1; b >= 0; b--) {
+        const int j0 = b * w, we = min(w, k - j0);
+        if (j0 >= c_hi) continue;                // block below this chunk: it contributes nothing
+        // partial L(rows, b)^T x(rows) over this chunk's rows below the block
+        load_row_block(P, ld, r, j0, we, rok && r >= j0, pr);
+        if (rok && r >= j0 && r < j0 + we) stash_diag_row(pr, r - j0, 0.0, Lb, dinv, tv);   // owner's block rows
+#pragma unroll
+        for (int q = 0; q < kSW; q++) pr[q] *= xr;
+        warp_reduce_scatter64(pr);
+        red[warp][qlane] = pr[0];
+        red[warp][qlane + 1] = pr[1];
+        __syncthreads();
+        double mine = 0.0;
+        if (tid < we)
+#pragma unroll
+            for (int q = 0; q < kSolveThreads / 32; q++) mine += red[q][tid];
+        if (j0 < c_lo) {                          // not the owner: publish the partial
+            if (tid < we) {
+                part[((int64_t)c * nb + b) * w + tid] = mine;
+                __threadfence();
+            }
+            __syncthreads();
+            if (tid == 0) st_release_u32(cflag + c, (epoch << 12) | (unsigned)(nb - b));
+            continue;
+        }
+        // owner: t = y_b - own partial - partials of every chunk below, in chunk order
+        if (warp == kSolveThreads / 32 - 1)   // poll every chunk below in parallel (its counter only grows)
+            for (int cc = c + 1 + lane; cc < nc; cc += 32)
+                for (;;) {
+                    const unsigned fl = ld_acquire_u32(cflag + cc);
+                    if ((fl >> 12) == epoch && (fl & 0xfffu) >= (unsigned)(nb - b)) break;
+                    __nanosleep(32);
+                }
+        __syncthreads();
+        if (tid < we) {
+            double t = y[first + j0 + tid] - mine;
+            const double *__restrict__ pc = part + (int64_t)b * w + tid;
+#pragma unroll 8
+            for (int cc = c + 1; cc < nc; cc++) t -= __ldcg(pc + (int64_t)cc * nb * w);
+            tv[tid] = t;
+        }
+        __syncthreads();
+        if (tid < 32) {
+            double a0 = lane < we ? tv[lane] : 0.0, a1 = lane + 32 < we ? tv[lane + 32] : 0.0;
+            warp_trsv_bwd(Lb, dinv, we, a0, a1);
+            if (lane < we) {
+                tv[lane] = a0;
+                y[first + j0 + lane] = a0;
+            }
+            if (lane + 32 < we) {
+                tv[lane + 32] = a1;
+                y[first + j0 + lane + 32] = a1;
+            }
+        }
+        __syncthreads();
+        if (rok && r >= j0 && r < j0 + we) xr = tv[r - j0];
+        __syncthreads();
     }
 }
 
 void launch_fsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, cudaStream_t st) {
     if (count > 0) k_fsolve_init<<<count, kSolveThreads, 0, st>>>(d, list, y);
 }
-void launch_fsolve_wave(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, double *y,
-                        cudaStream_t st) {
-    if (count > 0) k_fsolve_wave<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, j0, w, y);
+void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, cudaStream_t st) {
+    if (count > 0) k_fsolve_df<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, w, y);
 }
 void launch_bsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, const int32_t *sn_rows,
                         const int64_t *sn_rowptr, cudaStream_t st) {
     if (count > 0) k_bsolve_init<<<count, kSolveThreads, 0, st>>>(d, list, y, sn_rows, sn_rowptr);
 }
-void launch_bsolve_wave(const DevPlan &d, const int32_t *tasks, int64_t task_base, int64_t count, const int32_t *groups,
-                        int j0, int w, double *y, double *partials, int *counters, cudaStream_t st) {
-    if (count > 0)
-        k_bsolve_wave<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, task_base, groups, j0, w, y, partials,
-                                                                  counters);
+void launch_bsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, cudaStream_t st) {
+    if (count > 0) k_bsolve_df<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, w, y);
 }
 
 // dst[first_s + j] = src[first_s + j] for the columns of the listed supernodes

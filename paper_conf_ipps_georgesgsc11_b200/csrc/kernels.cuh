@@ -25,6 +25,10 @@ struct DevPlan {
     int *failed;             // min failing pivot column (final labels); INT_MAX = none
     const unsigned *epoch;   // factorization counter (= failed + 1), bumped by the init kernel
     unsigned *leaf_flag;     // per supernode: fused-leaf "diagonal block done" flag
+    unsigned *solve_epoch;   // solve counter (= failed + 2), bumped by the first solve kernel
+    unsigned *df_flags;      // dataflow solve flags (forward per block, backward per chunk)
+    double *df_parts;        // dataflow backward partial sums per (chunk, block)
+    const int64_t *df_blk_off, *df_part_off;
 };
 
 // launchers (all asynchronous on `st`)
@@ -43,12 +47,11 @@ void launch_fwd_solve(const DevPlan &d, const int32_t *list, int count, double *
 void launch_bwd_solve(const DevPlan &d, const int32_t *list, int count, double *y, const int32_t *sn_rows,
                       const int64_t *sn_rowptr, cudaStream_t st);
 void launch_fsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, cudaStream_t st);
-void launch_fsolve_wave(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, double *y,
-                        cudaStream_t st);
+void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, cudaStream_t st);
+void launch_bsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, cudaStream_t st);
 void launch_bsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, const int32_t *sn_rows,
                         const int64_t *sn_rowptr, cudaStream_t st);
-void launch_bsolve_wave(const DevPlan &d, const int32_t *tasks, int64_t task_base, int64_t count, const int32_t *groups,
-                        int j0, int w, double *y, double *partials, int *counters, cudaStream_t st);
+
 int small_front_smem_ok(int fmax);
 int kernels_init();
 void launch_copy_cols(const DevPlan &d, const int32_t *list, int count, const double *src, double *dst,

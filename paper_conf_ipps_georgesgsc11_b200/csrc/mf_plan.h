@@ -94,10 +94,10 @@ struct Launch {
 enum SolveKind : int32_t {
     SK_SMALL_F = 0,   // one CTA per small supernode: gather, trsv, gemv
     SK_INIT_F = 1,    // large supernodes: v = [y(cols); 0] + extend-add of children's update vectors
-    SK_WAVE_F = 2,    // one diagonal block: trsv (redundant per CTA) + gemv of a row chunk
+    SK_DF_F = 2,      // all large supernodes of a level, one launch: 256-row chunks, per-block flags
     SK_SMALL_B = 3,
     SK_INIT_B = 4,    // large supernodes: v(k:f) = x(R(k:f))
-    SK_WAVE_B = 5     // one diagonal block: partial L2^T v per row chunk, last CTA reduces + trsv
+    SK_DF_B = 5       // all large supernodes of a level, one launch: chunk partials, owner reduces + trsv
 };
 struct SolveLaunch {
     int32_t kind;
@@ -126,9 +126,9 @@ struct Plan {
     std::vector<Launch> program;
     // solve
     std::vector<int32_t> solve_list;                 // supernode lists (small / large) per launch
-    std::vector<int32_t> sf_tasks;                   // forward waves: (front, row0, writer)
-    std::vector<int32_t> sb_tasks;                   // backward waves: (front, row0, group)
-    std::vector<int32_t> sb_groups;                  // (first task, ntasks) per (front, block)
+    std::vector<int32_t> df_tasks;                   // dataflow solve: (front, chunk) pairs
+    std::vector<int64_t> df_blk_off, df_part_off;    // per supernode: block-flag and partial-sum bases
+    int64_t df_nflags = 0, df_nparts = 0;            // u32 flags / fp64 partial words
     std::vector<SolveLaunch> fsolve, bsolve;
     // ---- multi-GPU: subtree-to-GPU mapping.  Subtrees below a
     // frontier are factored by their owner; the supernodes above the frontier ("top")
@@ -148,7 +148,7 @@ constexpr int kTileM = 64, kTileN = 64;
 constexpr int kAsmCols = 16;
 constexpr int kTrsmRows = 128;
 constexpr int kSmallClasses = 4;
-constexpr int kSolveRows = 256;
+constexpr int kSolveRows = 256;   // dataflow solve: rows per chunk (a multiple of the 64-column block)
 
 int build_plan(const Symbolic &S, const Options &opt, Plan &P);
 

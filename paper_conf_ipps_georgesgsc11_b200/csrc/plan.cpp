@@ -60,59 +60,47 @@ static void build_solve_plan(const Symbolic &S, Plan &P, const std::vector<char>
         P.solve_list.insert(P.solve_list.end(), v.begin(), v.end());
         return off;
     };
+    // dataflow solve of the large supernodes: 256-row chunks; flags per 64-column
+    // block (forward) and per chunk (backward); partial sums per (chunk, block)
+    auto ensure_df = [&](int32_t s) {
+        if (P.df_blk_off[s] >= 0) return;
+        const int64_t nb = (P.sn_k[s] + w - 1) / w, nc = (P.sn_f[s] + kSolveRows - 1) / kSolveRows;
+        P.df_blk_off[s] = P.df_nflags;
+        P.df_nflags += nb + nc;   // nb forward block flags, then nc backward chunk flags
+        P.df_part_off[s] = P.df_nparts;
+        P.df_nparts += nc * nb * w;
+    };
     for (int32_t l = 0; l < P.nlevels; l++) {
         if (!small[l].empty()) fsolve.push_back({SK_SMALL_F, 0, push_list(small[l]), (int64_t)small[l].size()});
         if (large[l].empty()) continue;
         fsolve.push_back({SK_INIT_F, 0, push_list(large[l]), (int64_t)large[l].size()});
-        const int32_t kmax = P.sn_k[large[l][0]];
-        for (int32_t j0 = 0; j0 < kmax; j0 += w) {
-            const int64_t off = (int64_t)P.sf_tasks.size() / 3;
-            for (int32_t s : large[l]) {
-                const int32_t k = P.sn_k[s], f = P.sn_f[s];
-                if (k <= j0) break;
-                const int32_t r_begin = j0 + std::min(w, k - j0);
-                int32_t r0 = r_begin;
-                do {
-                    P.sf_tasks.push_back(s);
-                    P.sf_tasks.push_back(r0);
-                    P.sf_tasks.push_back(r0 == r_begin ? 1 : 0);
-                    r0 += kSolveRows;
-                } while (r0 < f);
+        const int64_t off = (int64_t)P.df_tasks.size() / 2;
+        for (int32_t s : large[l]) {   // chunks top-down: a chunk waits only on earlier blocks (lower CTA ids)
+            ensure_df(s);
+            for (int32_t c = 0; c * kSolveRows < P.sn_f[s]; c++) {
+                P.df_tasks.push_back(s);
+                P.df_tasks.push_back(c);
             }
-            fsolve.push_back({SK_WAVE_F, j0, off, (int64_t)P.sf_tasks.size() / 3 - off});
         }
+        fsolve.push_back({SK_DF_F, 0, off, (int64_t)P.df_tasks.size() / 2 - off});
     }
     for (int32_t l = P.nlevels - 1; l >= 0; l--) {
         if (!large[l].empty()) {
             bsolve.push_back({SK_INIT_B, 0, push_list(large[l]), (int64_t)large[l].size()});
-            const int32_t kmax = P.sn_k[large[l][0]];
-            const int32_t nb = (kmax + w - 1) / w;
-            for (int32_t b = nb - 1; b >= 0; b--) {
-                const int32_t j0 = b * w;
-                const int64_t off = (int64_t)P.sb_tasks.size() / 3;
-                for (int32_t s : large[l]) {
-                    const int32_t k = P.sn_k[s], f = P.sn_f[s];
-                    if (k <= j0) break;
-                    const int32_t grp = (int32_t)P.sb_groups.size() / 2;
-                    const int32_t first_task = (int32_t)(P.sb_tasks.size() / 3);
-                    const int32_t r_begin = j0 + std::min(w, k - j0);
-                    int32_t r0 = r_begin, nt = 0;
-                    do {
-                        P.sb_tasks.push_back(s);
-                        P.sb_tasks.push_back(r0);
-                        P.sb_tasks.push_back(grp);
-                        nt++;
-                        r0 += kSolveRows;
-                    } while (r0 < f);
-                    P.sb_groups.push_back(first_task);
-                    P.sb_groups.push_back(nt);
+            const int64_t off = (int64_t)P.df_tasks.size() / 2;
+            for (int32_t s : large[l]) {   // chunks bottom-up: a chunk waits only on chunks below (lower CTA ids)
+                ensure_df(s);
+                for (int32_t c = (P.sn_f[s] + kSolveRows - 1) / kSolveRows - 1; c >= 0; c--) {
+                    P.df_tasks.push_back(s);
+                    P.df_tasks.push_back(c);
                 }
-                bsolve.push_back({SK_WAVE_B, j0, off, (int64_t)P.sb_tasks.size() / 3 - off});
             }
+            bsolve.push_back({SK_DF_B, 0, off, (int64_t)P.df_tasks.size() / 2 - off});
         }
         if (!small[l].empty()) bsolve.push_back({SK_SMALL_B, 0, push_list(small[l]), (int64_t)small[l].size()});
     }
 }
+
 
 // Subtree-to-GPU mapping (proportional/LPT): start from the
 // tree roots as the frontier; repeatedly move the heaviest expandable frontier
@@ -474,6 +462,8 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         if (Ls.count) cur->push_back(Ls);
     }
     }   // pass
+    P.df_blk_off.assign(ns, -1);
+    P.df_part_off.assign(ns, -1);
     build_solve_plan(S, P, inc_local, P.fsolve, P.bsolve);
     build_solve_plan(S, P, inc_top, P.fsolve_top, P.bsolve_top);
     return MF_OK;
