@@ -234,10 +234,18 @@ def main():
     mapping = None
     if world > 1:
         _, top, load, top_load = S.mapping()
+        coop = S.cooperative()
+        sn = S.supernodes()
+        k = np.diff(sn["sn_first"]).astype(float)
+        m = np.diff(sn["sn_rowptr"]).astype(float) - k
+        fl = k * m * m + m * k * (k + 1) + k * (k + 1) * (2 * k + 1) / 6
         tot = float(load.sum() + top_load)
-        mapping = {"top_supernodes": int(top.sum()), "top_flop_share": top_load / tot,
-                   "max_rank_subtree_share": float(load.max()) / tot,
-                   "bound_speedup": tot / (float(load.max()) + top_load)}
+        # flop bound (no exchange cost): subtrees in parallel, then the shared top
+        # fronts split over the ranks and the replicated ones redundantly
+        top_time = float(fl[coop].sum()) / world + float(fl[top & ~coop].sum())
+        mapping = {"top_supernodes": int(top.sum()), "cooperative_top_supernodes": int(coop.sum()),
+                   "top_flop_share": top_load / tot, "max_rank_subtree_share": float(load.max()) / tot,
+                   "flop_bound_speedup": tot / (float(load.max()) + top_time)}
     vals_d = torch.from_numpy(A.values).cuda()
     torch.cuda.synchronize()
 

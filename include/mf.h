@@ -70,6 +70,10 @@ typedef struct {
     int32_t nranks;           /* GPUs (one process each) sharing the factorization (default 1)     */
     int32_t rank;             /* this process's rank in [0, nranks)                                 */
     void *stream;             /* cudaStream_t to run on (NULL = the ctx creates its own)           */
+    int32_t split_all;        /* multi-GPU mapping: 0 (default) = choose the frontier and which top
+                                 fronts are shared by the exchange-cost model; 1 = always split (a
+                                 frontier of >= nranks subtrees, every eligible top front shared),
+                                 e.g. to exercise the cooperative path on small problems           */
 } mf_options;
 
 typedef struct {
@@ -194,7 +198,10 @@ int mf_get_program(const mf_ctx *ctx, mf_launch_info *out, int64_t max, int64_t 
 int mf_set_exchange(mf_ctx *ctx, mf_exchange_fn fn, void *user);
 
 /* Subtree-to-GPU mapping of the analyzed pattern: owner[nsuper] (rank factoring
- * each supernode) and top[nsuper] (1 = factored by rank 0 after the exchange).
+ * each supernode) and top[nsuper] (0 = in a rank's subtree; 1 = top supernode,
+ * replicated and factored redundantly by every rank; 2 = top supernode factored
+ * cooperatively: pivot-column blocks block-cyclic over the ranks, broadcast by
+ * their owner, U^n all-gathered).
  * rank_load[nranks] = executed flops of each rank's subtrees; *top_load = flops
  * of the top.  Any pointer may be NULL. */
 int mf_get_mapping(const mf_ctx *ctx, int32_t *owner, int8_t *top, double *rank_load, double *top_load);

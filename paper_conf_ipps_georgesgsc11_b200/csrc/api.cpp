@@ -181,6 +181,7 @@ int mf_default_options(mf_options *o) {
     o->nranks = 1;
     o->rank = 0;
     o->stream = nullptr;
+    o->split_all = 0;
     return MF_OK;
 }
 
@@ -206,6 +207,7 @@ int mf_create(mf_ctx **out, const mf_options *o) {
         return MF_ERR_ARG;
     }
     c->opt.nranks = o->nranks;
+    c->opt.split_all = o->split_all;
     c->opt.rank = o->rank;
     c->host_only = o->host_only != 0;
     c->info.failed_col = -1;
@@ -383,14 +385,14 @@ namespace {
 // Run one launch program (the whole factorization for one rank, or rank 0's top
 // part) on the ctx stream: eagerly with per-launch events when profiling,
 // otherwise as a CUDA graph captured on first use.
-int run_program(mf_ctx *c, const std::vector<Launch> &prog, const double *vals, bool with_init, size_t ev_base,
-                cudaGraph_t *graph, cudaGraphExec_t *exec) {
+int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1, const double *vals, bool with_init,
+                size_t ev_base, cudaGraph_t *graph, cudaGraphExec_t *exec) {
     const Plan &P = c->P;
     const DevPlan &d = c->d;
     cudaStream_t st = c->stream;
     auto issue = [&](const double *v, bool with_events) -> int {
         if (with_init) launch_init_failed(c->d_failed, st);
-        for (size_t li = 0; li < prog.size(); li++) {
+        for (size_t li = i0; li < i1; li++) {
             const Launch &L = prog[li];
             if (with_events) CK(cudaEventRecord(c->prof_events[ev_base + 2 * li], st));
             switch (L.kind) {
@@ -402,13 +404,14 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, const double *vals, 
                 case KC_LEAF:
                     launch_leaf(d, c->d_large + L.off, (int)L.count, c->d_trsm + 2 * L.off2, L.count2, L.param, P.w, st);
                     break;
+                default: return MF_ERR_STATE;   // exchange points are handled by run_with_exchanges
             }
             if (with_events) CK(cudaEventRecord(c->prof_events[ev_base + 2 * li + 1], st));
         }
         return MF_OK;
     };
     if (c->profiling) return issue(vals, true);
-    if (!c->use_graph) return issue(vals, false);
+    if (!c->use_graph || !graph) return issue(vals, false);
     // the graph always reads the ctx's value buffer
     if (vals != c->d_values && c->S.nnz_in > 0 && with_init)
         CK(cudaMemcpyAsync(c->d_values, vals, c->S.nnz_in * sizeof(double), cudaMemcpyDeviceToDevice, st));
@@ -437,9 +440,34 @@ int exchange(mf_ctx *c, std::vector<mf_xfer> &ops) {
     return r ? MF_ERR_NCCL : MF_OK;
 }
 
+// A program with exchange points (the multi-GPU top): kernel segments run eagerly
+// on the ctx stream, each exchange point hands its transfer group (pointers into
+// the L / U arenas) to the callback.
+int run_with_exchanges(mf_ctx *c, const std::vector<Launch> &prog, const double *vals, size_t ev_base) {
+    const Plan &P = c->P;
+    size_t i0 = 0;
+    while (i0 < prog.size()) {
+        size_t i1 = i0;
+        while (i1 < prog.size() && prog[i1].kind != KC_EXCHANGE) i1++;
+        if (i1 > i0) {
+            const int r = run_program(c, prog, i0, i1, vals, false, ev_base, nullptr, nullptr);
+            if (r) return r;
+        }
+        if (i1 == prog.size()) break;
+        std::vector<mf_xfer> ops;
+        for (const XferSpec &x : P.xfers[prog[i1].param])
+            ops.push_back(mf_xfer{x.op, x.peer, (x.in_U ? c->d.U : c->d.L) + x.off, x.words * (int64_t)sizeof(double)});
+        const int r = exchange(c, ops);
+        if (r) return r;
+        i0 = i1 + 1;
+    }
+    return MF_OK;
+}
+
 void accumulate_stats(mf_ctx *c, const std::vector<Launch> &prog, size_t ev_base) {
     for (size_t li = 0; li < prog.size(); li++) {
         const Launch &L = prog[li];
+        if (L.kind < 0 || L.kind >= KC_COUNT) continue;
         float t = 0.f;
         cudaEventElapsedTime(&t, c->prof_events[ev_base + 2 * li], c->prof_events[ev_base + 2 * li + 1]);
         mf_kernel_stat &K = c->kstats[L.kind];
@@ -477,25 +505,25 @@ int mf_factor(mf_ctx *c, const double *values) {
             c->prof_events.push_back(e);
         }
     }
-    int r = run_program(c, P.program, vals, true, 0, &c->graph, &c->graph_exec);
+    int r = run_program(c, P.program, 0, P.program.size(), vals, true, 0, &c->graph, &c->graph_exec);
     if (r) return r;
     int64_t launches = 1 + (int64_t)P.program.size();
     if (multi) {
-        // (1) the frontier roots' update matrices travel to rank 0
+        // (1) the frontier roots' update matrices are broadcast by their owners: every
+        // rank holds a replica of the top fronts
         std::vector<mf_xfer> ops;
         for (int32_t root : P.frontier_roots) {
-            const int32_t own = P.owner[root], m = P.sn_f[root] - P.sn_k[root];
-            if (own == 0 || m <= 0) continue;
-            if (P.rank == own || P.rank == 0)
-                ops.push_back(mf_xfer{P.rank == own ? MF_XFER_SEND : MF_XFER_RECV, P.rank == own ? 0 : own,
-                                      c->d.U + P.U_off[root], (int64_t)m * m * (int64_t)sizeof(double)});
+            const int32_t m = P.sn_f[root] - P.sn_k[root];
+            if (m <= 0) continue;
+            ops.push_back(mf_xfer{MF_XFER_BCAST, P.owner[root], c->d.U + P.U_off[root],
+                                  (int64_t)m * m * (int64_t)sizeof(double)});
         }
         if ((r = exchange(c, ops))) return r;
-        // (2) rank 0 factors the top supernodes
+        // (2) every rank factors the top: replicated small fronts, cooperative large ones
         if (!P.program_top.empty()) {
-            r = run_program(c, P.program_top, vals, false, 2 * P.program.size(), &c->graph_top, &c->graph_top_exec);
+            r = run_with_exchanges(c, P.program_top, vals, 2 * P.program.size());
             if (r) return r;
-            launches += (int64_t)P.program_top.size();
+            for (const Launch &L : P.program_top) launches += L.kind != KC_EXCHANGE;
         }
         // (3) first failing pivot over all ranks
         std::vector<mf_xfer> red{mf_xfer{MF_XFER_ALLREDUCE_MIN_I32, 0, c->d_failed, (int64_t)sizeof(int)}};
@@ -705,7 +733,7 @@ int mf_get_mapping(const mf_ctx *c, int32_t *owner, int8_t *top, double *rank_lo
     const Plan &P = c->P;
     if (owner) std::memcpy(owner, P.owner.data(), P.owner.size() * sizeof(int32_t));
     if (top)
-        for (size_t i = 0; i < P.top.size(); i++) top[i] = P.top[i];
+        for (size_t i = 0; i < P.top.size(); i++) top[i] = P.top[i] ? (P.dist[i] ? 2 : 1) : 0;
     if (rank_load) std::memcpy(rank_load, P.rank_load.data(), P.rank_load.size() * sizeof(double));
     if (top_load) *top_load = P.top_load;
     return MF_OK;

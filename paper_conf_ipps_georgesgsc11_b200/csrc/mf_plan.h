@@ -21,6 +21,7 @@ struct Options {
     int panel_w = 64;
     int nranks = 1;   // GPUs sharing one factorization (one process per GPU)
     int rank = 0;
+    int split_all = 0;   // multi-GPU mapping ignores the exchange-cost model
 };
 
 // ---------------------------------------------------------------- symbolic
@@ -76,9 +77,19 @@ enum KernelClass : int32_t {
     KC_TRSM = 3,      // panel trsm below the diagonal block
     KC_UPDATE = 4,    // DMMA Schur update (panel trailing update and the syrk on U^n)
     KC_LEAF = 5,      // fused potrf + trsm of one diagonal block (few active fronts)
-    KC_COUNT = 6
+    KC_COUNT = 6,
+    KC_EXCHANGE = 16  // multi-GPU: hand the transfer group Plan::xfers[param] to the exchange callback
 };
 constexpr int kFuseLeafMaxFronts = 8;
+
+// One transfer of a multi-GPU exchange point, relative to the L or U arena.
+struct XferSpec {
+    int32_t op;         // MF_XFER_*
+    int32_t peer;       // root of a broadcast / peer of a send or receive
+    int32_t in_U;       // 0: L arena, 1: U arena
+    int64_t off, words; // fp64 words
+};
+constexpr int32_t kDistLeaves = 4;   // distribution block of a top front = kDistLeaves leaves of w columns
 
 struct Launch {
     int32_t kind;       // KernelClass
@@ -132,14 +143,18 @@ struct Plan {
     std::vector<SolveLaunch> fsolve, bsolve;
     // ---- multi-GPU: subtree-to-GPU mapping.  Subtrees below a
     // frontier are factored by their owner; the supernodes above the frontier ("top")
-    // are factored by rank 0 after the frontier roots' update matrices arrive.
-    int32_t nranks = 1, rank = 0;
+    // are replicated on every rank after the frontier roots' update matrices are
+    // broadcast, and the large ones are factored cooperatively (block-cyclic pivot
+    // columns, split trailing updates, all-gathered U^n).
+    int32_t nranks = 1, rank = 0, split_all = 0;
     std::vector<int32_t> owner;                      // rank factoring each supernode
-    std::vector<char> top;                           // above the frontier (rank 0)
+    std::vector<char> top;                           // above the frontier (replicated)
+    std::vector<char> dist;                          // top fronts factored cooperatively
     std::vector<int32_t> frontier_roots;             // subtree roots whose parent is top
     std::vector<double> rank_load;                   // executed flops per rank (subtrees)
     double top_load = 0;
-    std::vector<Launch> program_top;                 // rank 0: top supernodes
+    std::vector<Launch> program_top;                 // every rank: top supernodes, with exchange points
+    std::vector<std::vector<XferSpec>> xfers;        // transfer groups of the KC_EXCHANGE entries
     std::vector<SolveLaunch> fsolve_top, bsolve_top; // rank 0: top supernodes
     std::vector<int32_t> top_list, own_list;         // supernode lists (copy / mask kernels)
 };

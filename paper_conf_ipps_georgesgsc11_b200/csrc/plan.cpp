@@ -15,6 +15,7 @@
 //   * its update matrix U^s: m_s x m_s column-major (lower triangle used) in the
 //     U arena, written by the F-U of s and read by the extend-add of its parent.
 #include <algorithm>
+#include <cmath>
 #include <functional>
 #include <numeric>
 
@@ -27,15 +28,45 @@ namespace mf {
 // so the CTAs resident at one time cover a squarish block of the output and
 // share both operand row panels in L2.
 constexpr int32_t kTileBand = 16;
-static void add_tiles(Plan &P, int32_t prob, int32_t M, int32_t N) {
+template <class Keep>
+static void add_tiles(Plan &P, int32_t prob, int32_t M, int32_t N, Keep keep_col) {
     const int32_t tm = (M + kTileM - 1) / kTileM, tn = (N + kTileN - 1) / kTileN;
     for (int32_t tj0 = 0; tj0 < tn; tj0 += kTileBand)
         for (int32_t ti = 0; ti < tm; ti++)
             for (int32_t tj = tj0; tj < std::min(tn, tj0 + kTileBand); tj++) {
                 // lower-trapezoid: skip tiles entirely above the diagonal (i < j everywhere)
                 if ((int64_t)(ti + 1) * kTileM - 1 < (int64_t)tj * kTileN) continue;
+                if (!keep_col(tj)) continue;
                 P.tiles.push_back({prob, (ti << 16) | tj});
             }
+}
+static int64_t count_tiles(int32_t M, int32_t N) {
+    const int32_t tm = (M + kTileM - 1) / kTileM, tn = (N + kTileN - 1) / kTileN;
+    int64_t c = 0;
+    for (int32_t tj = 0; tj < tn; tj++) c += std::max<int64_t>(0, tm - ((int64_t)tj * kTileN) / kTileM);
+    return std::max<int64_t>(c, 1);
+}
+// Tile columns [tb[r], tb[r+1]) of an m x m lower syrk for rank r: contiguous
+// ranges with (nearly) equal numbers of tiles.
+static std::vector<int32_t> split_tile_columns(int32_t m, int R) {
+    const int32_t tn = (m + kTileN - 1) / kTileN;
+    std::vector<int64_t> w(tn);
+    int64_t tot = 0;
+    for (int32_t tj = 0; tj < tn; tj++) tot += (w[tj] = tn - tj);
+    std::vector<int32_t> tb(R + 1, tn);
+    tb[0] = 0;
+    int64_t acc = 0;
+    int r = 1;
+    for (int32_t tj = 0; tj < tn && r < R; tj++) {
+        acc += w[tj];
+        while (r < R && acc * R >= tot * r) tb[r++] = tj + 1;
+    }
+    return tb;
+}
+// A top front is distributed over the ranks when it takes the tiled path and has
+// at least two distribution blocks of pivot columns.
+static bool dist_eligible(const Plan &P, int32_t s) {
+    return P.sn_f[s] > P.small_max && P.sn_k[s] >= 2 * kDistLeaves * P.w;
 }
 
 // Solve program: per level, small supernodes in one batched launch; large ones
@@ -106,12 +137,26 @@ static void build_solve_plan(const Symbolic &S, Plan &P, const std::vector<char>
 // tree roots as the frontier; repeatedly move the heaviest expandable frontier
 // subtree's root into the "top" (its children join the frontier), assign the
 // frontier subtrees to ranks by LPT on executed flops, and keep the frontier
-// with the smallest makespan = max rank load + top load (rank 0 factors the top
-// after every frontier root's update matrix has arrived).
+// with the smallest makespan = max rank load + top load (the top starts after
+// every frontier root's update matrix has arrived; its large fronts are shared by
+// all ranks, the rest is replicated).
+// Cost model of a top front, in flop-equivalents at ~30 TF/s: replicated = its
+// flops; cooperative = flops / R + one exchange latency (~30 us) per distribution
+// block + its broadcast bytes (L panel and U^n, ~400 GB/s effective).
+constexpr double kXchgLatency = 9e8, kXchgPerByte = 75.0;
+static double coop_cost(const Plan &P, int32_t s, double load) {
+    if (!dist_eligible(P, s)) return 1e300;
+    if (P.split_all) return load / P.nranks;   // no exchange cost: every eligible top front is shared
+    const double k = P.sn_k[s], f = P.sn_f[s], m = f - k;
+    const double nb = std::ceil(k / (kDistLeaves * P.w));
+    return load / P.nranks + kXchgLatency * nb + kXchgPerByte * 8.0 * (f * k + m * m / 2);
+}
+
 static void map_subtrees(Plan &P, const std::vector<double> &front_load) {
     const int32_t ns = P.nsuper, R = P.nranks;
     P.owner.assign(ns, 0);
     P.top.assign(ns, 0);
+    P.dist.assign(ns, 0);
     P.frontier_roots.clear();
     P.rank_load.assign(R, 0.0);
     P.top_load = 0;
@@ -156,10 +201,17 @@ static void map_subtrees(Plan &P, const std::vector<double> &front_load) {
         const int32_t v = fr[pick];
         fr.erase(fr.begin() + pick);
         is_top[v] = 1;
-        topl += front_load[v];
+        topl += std::min(front_load[v], coop_cost(P, v, front_load[v]));   // cooperative or replicated
         for (int32_t q = P.child_ptr[v]; q < P.child_ptr[v + 1]; q++) fr.push_back(P.child_list[q]);
-        const double make = lpt(fr, assign, load) + topl;
-        if (make < best_make) {
+        double bc = 0;   // broadcast of the frontier roots' update matrices
+        for (int32_t r : fr) {
+            const double m = P.sn_f[r] - P.sn_k[r];
+            bc += kXchgLatency / 8 + kXchgPerByte * 8.0 * m * m;
+        }
+        const double make = lpt(fr, assign, load) + topl + bc;
+        // split_all: the first frontier with >= R subtrees wins, whatever the model says
+        const bool forced = P.split_all && (int)best_fr.size() < R && (int)fr.size() >= R;
+        if (forced || (make < best_make && !(P.split_all && (int)fr.size() < R && (int)best_fr.size() >= R))) {
             best_make = make;
             best_fr = fr;
             best_assign = assign;
@@ -170,7 +222,10 @@ static void map_subtrees(Plan &P, const std::vector<double> &front_load) {
     P.top = best_top;
     P.rank_load = best_load;
     for (int32_t s = 0; s < ns; s++)
-        if (P.top[s]) P.top_load += front_load[s];
+        if (P.top[s]) {
+            P.top_load += front_load[s];
+            P.dist[s] = coop_cost(P, s, front_load[s]) < front_load[s];
+        }
     // owner of every supernode below the frontier = owner of its frontier root
     for (size_t i = 0; i < best_fr.size(); i++) {
         const int32_t rt = best_fr[i];
@@ -194,6 +249,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     P.rank = opt.rank;
     P.w = opt.panel_w;
     P.small_max = opt.small_front_max;
+    P.split_all = opt.split_all;
     P.sn_k.resize(ns);
     P.sn_f.resize(ns);
     P.sn_ld.resize(ns);
@@ -310,24 +366,121 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         }
         map_subtrees(P, front_load);
     }
-    std::vector<char> inc_local(ns), inc_top(ns);
+    // Inclusion masks.  Local program: the supernodes of this rank's subtrees.  Top
+    // program (multi-GPU): EVERY rank holds a replica of every top front; the
+    // pivot-column blocks of the large top fronts are owned block-cyclically (the
+    // owner factors a block and broadcasts it), the trailing updates are split by
+    // owned column, and the syrk on U^n by contiguous column ranges (all-gathered
+    // by broadcasts), so the top's flops are divided over the ranks.
+    const int R = P.nranks;
+    const int32_t Wd = kDistLeaves * w;   // distribution block: kDistLeaves leaves of w columns
+    std::vector<char> inc_local(ns), inc_top(ns), inc_top_solve(ns);
     for (int32_t s = 0; s < ns; s++) {
         inc_local[s] = !P.top[s] && P.owner[s] == P.rank;
-        inc_top[s] = P.top[s] && P.rank == 0;
-        if (P.top[s]) P.top_list.push_back(s);                      // every rank: y columns broadcast by rank 0
-        if (inc_local[s] || inc_top[s]) P.own_list.push_back(s);   // columns this rank finalises
+        inc_top[s] = P.top[s] && R > 1;
+        inc_top_solve[s] = P.top[s] && P.rank == 0;   // the top solve stays on rank 0
+        if (P.top[s]) P.top_list.push_back(s);                            // every rank: y columns broadcast by rank 0
+        if (inc_local[s] || inc_top_solve[s]) P.own_list.push_back(s);   // columns this rank finalises in the solve
     }
+    auto blk_owner = [&](int32_t s, int32_t t) -> int32_t { return P.dist[s] ? (t + s) % R : -1; };
+    auto blk_mine = [&](int32_t s, int32_t t) { const int32_t o = blk_owner(s, t); return o < 0 || o == P.rank; };
     std::vector<Launch> *cur = &P.program;
-    const std::vector<char> *inc = &inc_local;
+    // the update of the pivot-column leaves [mid, b) by the factored leaves [a, mid)
+    // (units of w) for the fronts fl (sorted by k descending): one DMMA launch with
+    // inner dimension (mid - a) w; tiles of global column col only if keep(s, col)
+    auto rec_update = [&](const std::vector<int32_t> &fl, int32_t a, int32_t mid, int32_t b, int32_t l,
+                          const std::function<bool(int32_t, int32_t)> &keep) {
+        const int32_t c0 = mid * w, c_lo = a * w;
+        Launch Lu{KC_UPDATE, 0, (int64_t)P.tiles.size(), 0, 0.0, 0.0, l};
+        for (int32_t s : fl) {
+            const int32_t k = P.sn_k[s], f = P.sn_f[s], ld = P.sn_ld[s];
+            if (k <= c0) continue;
+            const int32_t M = f - c0, N = std::min(b * w, k) - c0, K = c0 - c_lo;
+            if (M <= 0 || N <= 0) continue;
+            GemmProb g;
+            g.a_off = P.L_off[s] + (int64_t)c_lo * ld + c0;
+            g.c_off = P.L_off[s] + (int64_t)c0 * ld + c0;
+            g.lda = ld;
+            g.ldc = ld;
+            g.M = M;
+            g.N = N;
+            g.K = K;
+            g.c_in_U = 0;
+            const int32_t pid = (int32_t)P.probs.size();
+            P.probs.push_back(g);
+            const int64_t t0 = (int64_t)P.tiles.size();
+            add_tiles(P, pid, M, N, [&](int32_t tj) { return keep(s, c0 + tj * kTileN); });
+            const int64_t nt = (int64_t)P.tiles.size() - t0;
+            if (nt == 0) {
+                P.probs.pop_back();
+                continue;
+            }
+            const double frac = (double)nt / (double)count_tiles(M, N);
+            Lu.flops += frac * upd_flops(M, N, K);
+            Lu.bytes += frac * upd_bytes(M, N, K);
+        }
+        Lu.count = (int64_t)P.tiles.size() - Lu.off;
+        if (Lu.count) cur->push_back(Lu);
+    };
+    auto keep_all = [](int32_t, int32_t) { return true; };
+    // the blocked factorization of the pivot-column leaves [a, b) (units of w) of the
+    // fronts fl (sorted by k descending, stored at P.large_list[loff..])
+    std::function<void(const std::vector<int32_t> &, int64_t, int32_t, int32_t, int32_t)> rec =
+        [&](const std::vector<int32_t> &fl, int64_t loff, int32_t a, int32_t b, int32_t l) {
+        if (b - a == 1) {
+            const int32_t j0 = a * w;
+            int32_t na = 0;   // fronts (prefix of fl) with k > j0
+            while (na < (int32_t)fl.size() && P.sn_k[fl[na]] > j0) na++;
+            if (na == 0) return;
+            Launch Lp{KC_POTRF, j0, loff, na, 0.0, 0.0, l};
+            Launch Lt{KC_TRSM, j0, (int64_t)P.trsm_tasks.size() / 2, 0, 0.0, 0.0, l};
+            for (int32_t q = 0; q < na; q++) {
+                const int32_t s = fl[q];
+                const int32_t k = P.sn_k[s], f = P.sn_f[s];
+                const int32_t we = std::min(w, k - j0);
+                Lp.flops += (double)we * (we + 1) * (2.0 * we + 1) / 6;
+                Lp.bytes += 8.0 * we * (we + 1);
+                for (int32_t r0 = j0 + we; r0 < f; r0 += kTrsmRows) {
+                    P.trsm_tasks.push_back(s);
+                    P.trsm_tasks.push_back(r0);
+                }
+                const double rows = f - j0 - we;
+                Lt.flops += rows * we * we;
+                Lt.bytes += 8.0 * (2 * rows * we + (double)we * (we + 1) / 2);
+            }
+            Lt.count = (int64_t)P.trsm_tasks.size() / 2 - Lt.off;
+            if (na <= kFuseLeafMaxFronts && Lt.count) {   // one launch: potrf CTAs + flag-waiting trsm CTAs
+                Launch Lf{KC_LEAF, j0, Lp.off, Lp.count, Lp.flops + Lt.flops, Lp.bytes + Lt.bytes, l};
+                Lf.off2 = Lt.off;
+                Lf.count2 = Lt.count;
+                cur->push_back(Lf);
+                return;
+            }
+            cur->push_back(Lp);
+            if (Lt.count) cur->push_back(Lt);
+            return;
+        }
+        const int32_t mid = a + (b - a + 1) / 2;
+        rec(fl, loff, a, mid, l);
+        rec_update(fl, a, mid, b, l, keep_all);
+        rec(fl, loff, mid, b, l);
+    };
+    auto push_large = [&](const std::vector<int32_t> &fl) {
+        const int64_t off = (int64_t)P.large_list.size();
+        P.large_list.insert(P.large_list.end(), fl.begin(), fl.end());
+        return off;
+    };
+    auto push_xfers = [&](std::vector<XferSpec> &&x, int32_t l) {
+        cur->push_back(Launch{KC_EXCHANGE, (int32_t)P.xfers.size(), 0, 0, 0.0, 0.0, l});
+        P.xfers.push_back(std::move(x));
+    };
     for (int pass = 0; pass < 2; pass++) {
-    if (pass == 1) {
-        cur = &P.program_top;
-        inc = &inc_top;
-    }
+    const std::vector<char> &inc = pass == 0 ? inc_local : inc_top;
+    if (pass == 1) cur = &P.program_top;
     for (int32_t l = 0; l < nlev; l++) {
         std::vector<int32_t> fronts;
         for (int32_t q = P.level_ptr[l]; q < P.level_ptr[l + 1]; q++)
-            if ((*inc)[P.level_list[q]]) fronts.push_back(P.level_list[q]);
+            if (inc[P.level_list[q]]) fronts.push_back(P.level_list[q]);
         for (int cls = 0; cls < kSmallClasses; cls++) {
             const int lo = cls == 0 ? 0 : P.small_class_fmax[cls - 1];
             Launch L{KC_SMALL, P.small_class_fmax[cls], (int64_t)P.small_list.size(), 0, 0.0, 0.0, l};
@@ -346,9 +499,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
             if (P.sn_f[s] > P.small_max) large.push_back(s);
         if (large.empty()) continue;
         std::stable_sort(large.begin(), large.end(), [&](int32_t a, int32_t b) { return P.sn_k[a] > P.sn_k[b]; });
-        const int64_t large_off = (int64_t)P.large_list.size();
-        P.large_list.insert(P.large_list.end(), large.begin(), large.end());
-        // assembly
+        // assembly (every rank assembles its replica of a top front)
         {
             Launch L{KC_ASSEMBLE, 0, (int64_t)P.asm_tasks.size() / 2, 0, 0.0, 0.0, l};
             for (int32_t s : large) {
@@ -370,76 +521,56 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         // right half), so most flops run with a long inner dimension instead of
         // w-wide right-looking steps.  A front whose k ends inside the range
         // simply drops out of the launches beyond its last block.
-        auto nactive_for = [&](int64_t col) {   // fronts (prefix of `large`) with k > col
-            int32_t na = 0;
-            while (na < (int32_t)large.size() && P.sn_k[large[na]] > col) na++;
-            return na;
-        };
-        std::function<void(int32_t, int32_t)> rec = [&](int32_t a, int32_t b) {
-            if (b - a == 1) {
-                const int32_t j0 = a * w;
-                const int32_t na = nactive_for(j0);
-                Launch Lp{KC_POTRF, j0, large_off, na, 0.0, 0.0, l};
-                Launch Lt{KC_TRSM, j0, (int64_t)P.trsm_tasks.size() / 2, 0, 0.0, 0.0, l};
-                for (int32_t q = 0; q < na; q++) {
-                    const int32_t s = large[q];
-                    const int32_t k = P.sn_k[s], f = P.sn_f[s];
-                    const int32_t we = std::min(w, k - j0);
-                    Lp.flops += (double)we * (we + 1) * (2.0 * we + 1) / 6;
-                    Lp.bytes += 8.0 * we * (we + 1);
-                    for (int32_t r0 = j0 + we; r0 < f; r0 += kTrsmRows) {
-                        P.trsm_tasks.push_back(s);
-                        P.trsm_tasks.push_back(r0);
+        const int32_t nbw = (P.sn_k[large[0]] + w - 1) / w;
+        bool any_dist = false;
+        for (int32_t s : large) any_dist = any_dist || P.dist[s];
+        if (!any_dist) {
+            rec(large, push_large(large), 0, nbw, l);
+        } else {
+            // distributed: the same recursion over blocks of Wd columns; a block (a
+            // "super-leaf") is factored by its owner alone (inner recursion over its
+            // leaves) and then broadcast; updates above the block level are split by
+            // owned column
+            const int32_t nbd = (P.sn_k[large[0]] + Wd - 1) / Wd;
+            std::function<void(int32_t, int32_t)> rec_d = [&](int32_t A, int32_t B) {
+                if (B - A == 1) {
+                    const int32_t t = A;
+                    std::vector<int32_t> fl;
+                    std::vector<XferSpec> x;
+                    for (int32_t s : large) {
+                        if (P.sn_k[s] <= t * Wd) continue;
+                        if (blk_mine(s, t)) fl.push_back(s);
+                        const int32_t o = blk_owner(s, t);
+                        if (o >= 0) {   // block columns [t Wd, min(k, (t+1) Wd)), rows t Wd .. f
+                            const int32_t ld = P.sn_ld[s], j0 = t * Wd, nc = std::min(P.sn_k[s], j0 + Wd) - j0;
+                            x.push_back(XferSpec{MF_XFER_BCAST, o, 0, P.L_off[s] + (int64_t)j0 * ld + j0,
+                                                 (int64_t)(nc - 1) * ld + (P.sn_f[s] - j0)});
+                        }
                     }
-                    const double rows = f - j0 - we;
-                    Lt.flops += rows * we * we;
-                    Lt.bytes += 8.0 * (2 * rows * we + (double)we * (we + 1) / 2);
-                }
-                Lt.count = (int64_t)P.trsm_tasks.size() / 2 - Lt.off;
-                if (na <= kFuseLeafMaxFronts && Lt.count) {   // one launch: potrf CTAs + flag-waiting trsm CTAs
-                    Launch Lf{KC_LEAF, j0, Lp.off, Lp.count, Lp.flops + Lt.flops, Lp.bytes + Lt.bytes, l};
-                    Lf.off2 = Lt.off;
-                    Lf.count2 = Lt.count;
-                    cur->push_back(Lf);
+                    if (!fl.empty())
+                        rec(fl, push_large(fl), t * kDistLeaves, std::min(nbw, (t + 1) * kDistLeaves), l);
+                    if (!x.empty()) push_xfers(std::move(x), l);
                     return;
                 }
-                cur->push_back(Lp);
-                if (Lt.count) cur->push_back(Lt);
-                return;
-            }
-            const int32_t mid = a + (b - a + 1) / 2;
-            rec(a, mid);
-            const int32_t c0 = mid * w, c_lo = a * w;
-            const int32_t na = nactive_for(c0);
-            Launch Lu{KC_UPDATE, 0, (int64_t)P.tiles.size(), 0, 0.0, 0.0, l};
-            for (int32_t q = 0; q < na; q++) {
-                const int32_t s = large[q];
-                const int32_t k = P.sn_k[s], f = P.sn_f[s], ld = P.sn_ld[s];
-                const int32_t M = f - c0, N = std::min(b * w, k) - c0, K = c0 - c_lo;
-                if (M <= 0 || N <= 0) continue;
-                GemmProb g;
-                g.a_off = P.L_off[s] + (int64_t)c_lo * ld + c0;
-                g.c_off = P.L_off[s] + (int64_t)c0 * ld + c0;
-                g.lda = ld;
-                g.ldc = ld;
-                g.M = M;
-                g.N = N;
-                g.K = K;
-                g.c_in_U = 0;
-                const int32_t pid = (int32_t)P.probs.size();
-                P.probs.push_back(g);
-                add_tiles(P, pid, M, N);
-                Lu.flops += upd_flops(M, N, K);
-                Lu.bytes += upd_bytes(M, N, K);
-            }
-            Lu.count = (int64_t)P.tiles.size() - Lu.off;
-            if (Lu.count) cur->push_back(Lu);
-            rec(mid, b);
-        };
-        const int32_t nb = (P.sn_k[large[0]] + w - 1) / w;
-        rec(0, nb);
-        // the syrk on U^n with inner dimension k (one launch for the level)
+                const int32_t mid = A + (B - A + 1) / 2;
+                rec_d(A, mid);
+                // the update of blocks [mid, B) by blocks [A, mid): the generic
+                // recursion's update step at leaf granularity, tiles of owned columns
+                std::vector<int32_t> fl;
+                for (int32_t s : large)
+                    if (P.sn_k[s] > mid * Wd) fl.push_back(s);
+                if (!fl.empty())
+                    rec_update(fl, A * kDistLeaves, mid * kDistLeaves, B * kDistLeaves, l,
+                               [&](int32_t s, int32_t col) { return blk_mine(s, col / Wd); });
+                rec_d(mid, B);
+            };
+            rec_d(0, nbd);
+        }
+        // the syrk on U^n with inner dimension k (one launch for the level); a
+        // distributed front's tile columns are split into contiguous ranges balanced
+        // by work, then every range is broadcast by the rank that computed it
         Launch Ls{KC_UPDATE, 1, (int64_t)P.tiles.size(), 0, 0.0, 0.0, l};
+        std::vector<XferSpec> ux;
         for (int32_t s : large) {
             const int32_t k = P.sn_k[s], f = P.sn_f[s], ld = P.sn_ld[s], m = f - k;
             if (m <= 0) continue;
@@ -454,18 +585,34 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
             g.c_in_U = 1;
             const int32_t pid = (int32_t)P.probs.size();
             P.probs.push_back(g);
-            add_tiles(P, pid, m, m);
-            Ls.flops += upd_flops(m, m, k);
-            Ls.bytes += upd_bytes(m, m, k);
+            if (!P.dist[s]) {
+                add_tiles(P, pid, m, m, [](int32_t) { return true; });
+                Ls.flops += upd_flops(m, m, k);
+                Ls.bytes += upd_bytes(m, m, k);
+                continue;
+            }
+            const std::vector<int32_t> tb = split_tile_columns(m, R);
+            const int64_t t0 = (int64_t)P.tiles.size();
+            add_tiles(P, pid, m, m, [&](int32_t tj) { return tj >= tb[P.rank] && tj < tb[P.rank + 1]; });
+            const double frac = (double)((int64_t)P.tiles.size() - t0) / std::max<int64_t>(1, count_tiles(m, m));
+            Ls.flops += frac * upd_flops(m, m, k);
+            Ls.bytes += frac * upd_bytes(m, m, k);
+            for (int r = 0; r < R; r++) {
+                const int32_t c0 = tb[r] * kTileN, c1 = std::min(m, tb[r + 1] * kTileN);
+                if (c1 <= c0) continue;
+                ux.push_back(XferSpec{MF_XFER_BCAST, r, 1, P.U_off[s] + (int64_t)c0 * m + c0,
+                                      (int64_t)(c1 - c0 - 1) * m + (m - c0)});
+            }
         }
         Ls.count = (int64_t)P.tiles.size() - Ls.off;
         if (Ls.count) cur->push_back(Ls);
+        if (!ux.empty()) push_xfers(std::move(ux), l);
     }
     }   // pass
     P.df_blk_off.assign(ns, -1);
     P.df_part_off.assign(ns, -1);
     build_solve_plan(S, P, inc_local, P.fsolve, P.bsolve);
-    build_solve_plan(S, P, inc_top, P.fsolve_top, P.bsolve_top);
+    build_solve_plan(S, P, inc_top_solve, P.fsolve_top, P.bsolve_top);
     return MF_OK;
 }
 

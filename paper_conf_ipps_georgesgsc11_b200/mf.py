@@ -34,7 +34,7 @@ class Options(ctypes.Structure):
         ("amalgamate", ctypes.c_int32), ("nrelax", ctypes.c_int32 * 3), ("zrelax", ctypes.c_double * 3),
         ("small_front_max", ctypes.c_int32), ("panel_w", ctypes.c_int32), ("device", ctypes.c_int32),
         ("host_only", ctypes.c_int32), ("nranks", ctypes.c_int32), ("rank", ctypes.c_int32),
-        ("stream", ctypes.c_void_p),
+        ("stream", ctypes.c_void_p), ("split_all", ctypes.c_int32),
     ]
 
 
@@ -147,7 +147,7 @@ class Solver:
 
     def __init__(self, amalgamate: bool = True, small_front_max: int | None = None, panel_w: int | None = None,
                  device: int = -1, stream: int | None = None, host_only: bool = False,
-                 nranks: int = 1, rank: int = 0, exchange=None):
+                 nranks: int = 1, rank: int = 0, exchange=None, split_all: bool = False):
         o = Options()
         lib.mf_default_options(ctypes.byref(o))
         o.amalgamate = int(amalgamate)
@@ -159,6 +159,7 @@ class Solver:
         o.host_only = int(host_only)
         o.nranks = nranks
         o.rank = rank
+        o.split_all = int(split_all)
         o.stream = stream
         h = ctypes.c_void_p()
         r = lib.mf_create(ctypes.byref(h), ctypes.byref(o))
@@ -193,7 +194,13 @@ class Solver:
         tl = ctypes.c_double()
         self._check(lib.mf_get_mapping(self._h, owner.ctypes.data, top.ctypes.data, load.ctypes.data,
                                        ctypes.byref(tl)), "mf_get_mapping")
+        self._top_kind = top
         return owner, top.astype(bool), load, tl.value
+
+    def cooperative(self) -> np.ndarray:
+        """Mask of the top supernodes factored cooperatively by all ranks."""
+        self.mapping()
+        return self._top_kind == 2
 
     def close(self):
         if getattr(self, "_h", None):

@@ -1,5 +1,7 @@
-"""Multi-GPU path: subtree-to-GPU mapping, exchange of the
-frontier roots' update matrices, rank 0 factors the top supernodes.
+"""Multi-GPU path: subtree-to-GPU mapping, broadcast of the
+frontier roots' update matrices, every rank holds the top supernodes and factors
+the large ones cooperatively (block-cyclic pivot-column blocks broadcast by their
+owner, trailing updates split by owned column, U^n all-gathered).
 
 CPU (not gpu): the mapping is a partition consistent across ranks (checked in
 two gloo processes, world size 2), and the exchange callback moves the right
@@ -20,8 +22,8 @@ from paper_conf_ipps_georgesgsc11_b200 import mf as mfmod
 from tests._grids import grid
 
 
-def mapping_for(A, p, R, rank):
-    S = mf.Solver(host_only=True, nranks=R, rank=rank)
+def mapping_for(A, p, R, rank, split_all=True):
+    S = mf.Solver(host_only=True, nranks=R, rank=rank, split_all=split_all)
     S.analyze(A.n, A.colptr, A.rowind, p)
     owner, top, load, top_load = S.mapping()
     sn = S.supernodes()
@@ -30,11 +32,14 @@ def mapping_for(A, p, R, rank):
     return owner, top, load, top_load, sn, inf
 
 
+@pytest.mark.parametrize("split_all", [True, False])
 @pytest.mark.parametrize("R", [2, 3, 4, 8])
 @pytest.mark.parametrize("kind,dims", [("27pt", (20, 20, 20)), ("9pt", (60, 60, 1)), ("elast", (8, 8, 8))])
-def test_mapping_is_a_partition(kind, dims, R):
+def test_mapping_is_a_partition(kind, dims, R, split_all):
     A, p = grid(kind, dims)
-    owner, top, load, top_load, sn, inf = mapping_for(A, p, R, 0)
+    owner, top, load, top_load, sn, inf = mapping_for(A, p, R, 0, split_all)
+    if split_all:   # forced split: at least R subtrees below the top
+        assert top.any() and len(set(owner[~top])) == R
     par = sn["sn_parent"]
     ns = inf["nsuper"]
     # top is closed upward; below the frontier every supernode has its subtree's owner
@@ -54,7 +59,7 @@ def test_mapping_is_a_partition(kind, dims, R):
         assert load[r] == pytest.approx(fl[(~top) & (owner == r)].sum(), rel=1e-12)
     # every rank computes the same mapping
     for r in range(1, R):
-        o2, t2, l2, tl2, _, _ = mapping_for(A, p, R, r)
+        o2, t2, l2, tl2, _, _ = mapping_for(A, p, R, r, split_all)
         np.testing.assert_array_equal(o2, owner)
         np.testing.assert_array_equal(t2, top)
 
@@ -112,10 +117,10 @@ def test_gloo_world2_mapping_and_exchange():
 
 
 # ---------------------------------------------------------------- GPU (loopback ranks)
-def run_loopback(A, perm, R, values=None, b=None):
+def run_loopback(A, perm, R, values=None, b=None, split_all=True, **opts):
     from paper_conf_ipps_georgesgsc11_b200.exchange import LoopbackHub
     hub = LoopbackHub(R)
-    solvers = [mf.Solver(nranks=R, rank=r, exchange=hub.for_rank(r)) for r in range(R)]
+    solvers = [mf.Solver(nranks=R, rank=r, exchange=hub.for_rank(r), split_all=split_all, **opts) for r in range(R)]
     for S in solvers:
         S.analyze(A.n, A.colptr, A.rowind, perm)
     vals = A.values if values is None else values
@@ -138,28 +143,36 @@ def run_loopback(A, perm, R, values=None, b=None):
     return solvers, xs
 
 
+LOOPBACK_CASES = [("27pt", (20, 20, 20), {}), ("7pt", (24, 24, 24), {}),
+                  ("27pt", (20, 20, 20), {"panel_w": 16}), ("27pt", (32, 32, 32), {})]
+
+
 @pytest.mark.gpu
 @pytest.mark.parametrize("R", [2, 3, 4])
-@pytest.mark.parametrize("kind,dims", [("27pt", (20, 20, 20)), ("7pt", (24, 24, 24))])
-def test_loopback_ranks_match_single(kind, dims, R):
+@pytest.mark.parametrize("kind,dims,opts", LOOPBACK_CASES)
+def test_loopback_ranks_match_single(kind, dims, opts, R):
     from tests.test_gpu_parity import c11, spmv, backward_error
     from workloads import grids as G
     A, p = grid(kind, dims)
-    ref = mf.Solver()
+    ref = mf.Solver(**opts)
     ref.analyze(A.n, A.colptr, A.rowind, p)
     ref.factor(A.values)
     b = spmv(A, G.rhs(A.n, 0))
     xref = ref.solve(b)
-    solvers, xs = run_loopback(A, p, R, b=b)
+    solvers, xs = run_loopback(A, p, R, b=b, **opts)
     owner, top, load, _ = solvers[0].mapping()
+    coop = solvers[0].cooperative()
     assert top.any() and len(set(owner[~top])) == R
+    if opts or dims[0] >= 32:   # cases with fronts wide enough to be shared
+        assert coop.any()
     sn = ref.supernodes()
     worst = 0.0
     for s in range(ref.info()["nsuper"]):
         f = int(sn["sn_rowptr"][s + 1] - sn["sn_rowptr"][s])
         k = int(sn["sn_first"][s + 1] - sn["sn_first"][s])
-        r = 0 if top[s] else int(owner[s])
-        worst = max(worst, c11(solvers[r].panel(s, f, k), ref.panel(s, f, k)))
+        holders = range(R) if top[s] else [int(owner[s])]   # the top is replicated on every rank
+        for r in holders:
+            worst = max(worst, c11(solvers[r].panel(s, f, k), ref.panel(s, f, k)))
     assert worst <= 1e-12
     for r in range(R):
         np.testing.assert_allclose(xs[r], xref, rtol=1e-11, atol=1e-13)
@@ -169,24 +182,29 @@ def test_loopback_ranks_match_single(kind, dims, R):
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("R", [2, 4])
-def test_loopback_manufactured_bit_exact(R):
+@pytest.mark.parametrize("R", [2, 3, 4])
+@pytest.mark.parametrize("dims,opts", [((12, 12, 12), {}), ((16, 16, 16), {"panel_w": 16})])
+def test_loopback_manufactured_bit_exact(R, dims, opts):
+    """SURVEY.md Sec. 8(c) 'Multi-GPU' pin: the manufactured factor is reproduced
+    bitwise by every rank, whatever the split of the top fronts' work."""
     import oracle
     from workloads import grids as G
-    A0, p = grid("27pt", (12, 12, 12))
+    A0, p = grid("27pt", dims)
     s0 = oracle.symbolic(A0, p, keep_struct=True)
     A, Lx = G.manufactured(A0.n, s0.Lp, s0.Li, s0.perm, seed=1234)
-    ref = mf.Solver()
+    ref = mf.Solver(**opts)
     ref.analyze(A.n, A.colptr, A.rowind, s0.perm)
     ref.factor(A.values)
-    solvers, _ = run_loopback(A, s0.perm, R)
+    solvers, _ = run_loopback(A, s0.perm, R, **opts)
     owner, top, _, _ = solvers[0].mapping()
+    if opts:
+        assert solvers[0].cooperative().any()
     sn = ref.supernodes()
     for s in range(ref.info()["nsuper"]):
         f = int(sn["sn_rowptr"][s + 1] - sn["sn_rowptr"][s])
         k = int(sn["sn_first"][s + 1] - sn["sn_first"][s])
-        r = 0 if top[s] else int(owner[s])
-        np.testing.assert_array_equal(solvers[r].panel(s, f, k), ref.panel(s, f, k))
+        for r in (range(R) if top[s] else [int(owner[s])]):
+            np.testing.assert_array_equal(solvers[r].panel(s, f, k), ref.panel(s, f, k))
 
 
 @pytest.mark.gpu
@@ -200,7 +218,7 @@ def test_loopback_not_spd_reported_on_every_rank():
     from paper_conf_ipps_georgesgsc11_b200.exchange import LoopbackHub
     R = 3
     hub = LoopbackHub(R)
-    solvers = [mf.Solver(nranks=R, rank=r, exchange=hub.for_rank(r)) for r in range(R)]
+    solvers = [mf.Solver(nranks=R, rank=r, exchange=hub.for_rank(r), split_all=True) for r in range(R)]
     for S in solvers:
         S.analyze(A.n, A.colptr, A.rowind, p)
     cols = [None] * R
