@@ -14,8 +14,10 @@
 // STAGES-deep shared-memory ring; each warp owns a TM x TN sub-tile whose
 // accumulators start from C (loaded while the first stages are in flight) and
 // accumulate C - A B^T directly (A fragments negated), so the epilogue is a
-// masked store.  Columns are 16-byte aligned (lda even); problems whose first
-// row is odd are staged with 8-byte cp.async instead of 16-byte chunks.
+// masked store.  Columns are 16-byte aligned (lda even) and every problem's
+// first row is even: the planner shifts a problem whose first row is odd (the
+// syrk on U^n of a supernode with odd k) one row up, computes the extra leading
+// row / column of the shifted space and masks it out here (flag bit 1).
 #pragma once
 #include <cstdint>
 
@@ -51,15 +53,13 @@ struct UpdCfg {
     static constexpr int TM = BM / WARPS_M, TN = BN / WARPS_N;   // warp tile
     static constexpr int MB = TM / 8, NB = TN / 8;                // DMMA blocks per warp
     static constexpr int SA = BM + 4, SB = BN + 4;                // pad: stride % 16 == 4 (conflict-free fragments)
-    // operand staging: 16-byte chunks (2 rows) when the problem's first row is
-    // even, 8-byte elements otherwise; every thread keeps a fixed row slot and
-    // walks the k dimension with a fixed stride, so there is no index math in
-    // the main loop.
+    // operand staging: 16-byte chunks (2 rows); every thread keeps a fixed row
+    // slot and walks the k dimension with a fixed stride, so there is no index
+    // math in the main loop.
     static constexpr int CPA = BM / 2, CPB = BN / 2;              // 16-byte chunks per column
-    static_assert(NT % CPA == 0 && NT % CPB == 0 && NT % BM == 0 && NT % BN == 0, "staging map");
-    static constexpr int PSA16 = NT / CPA, PSB16 = NT / CPB;      // k stride of a thread (16-byte path)
-    static constexpr int PSA8 = NT / BM, PSB8 = NT / BN;          // k stride of a thread (8-byte path)
-    static_assert(BK % PSA16 == 0 && BK % PSB16 == 0 && BK % PSA8 == 0 && BK % PSB8 == 0, "staging map");
+    static_assert(NT % CPA == 0 && NT % CPB == 0, "staging map");
+    static constexpr int PSA16 = NT / CPA, PSB16 = NT / CPB;      // k stride of a thread
+    static_assert(BK % PSA16 == 0 && BK % PSB16 == 0, "staging map");
     static constexpr int STAGE_WORDS = BK * (SA + SB);
     static constexpr size_t SMEM = (size_t)STAGES * STAGE_WORDS * sizeof(double);
     static_assert(SA % 16 == 4 && SB % 16 == 4, "bank-conflict-free fragment loads");
@@ -78,47 +78,31 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
     const GemmProb g = probs[t.prob];
     const int ti = t.tij >> 16, tj = t.tij & 0xffff;
     const int i0 = ti * BM, j0 = tj * BN;
-    const bool odd = (g.a_off & 1) != 0;   // columns are 16-byte aligned (even lda); rows may start odd
-    const double *__restrict__ A = Larena + g.a_off;
+    const double *__restrict__ A = Larena + g.a_off;   // a_off even: 16-byte aligned rows pairs
     const int lda = g.lda, K = g.K;
+    const int sh = (g.flags >> 1) & 1;                   // shifted problem: row / column 0 are padding
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int wm = warp % Cfg::WARPS_M, wn = warp / Cfg::WARPS_M;
     const int gq = lane >> 2, tq = lane & 3;
     // fixed staging slots of this thread
     const int ra16 = 2 * (tid % Cfg::CPA), pa16 = tid / Cfg::CPA;
     const int rb16 = 2 * (tid % Cfg::CPB), pb16 = tid / Cfg::CPB;
-    const int ra8 = tid % BM, pa8 = tid / BM;
-    const int rb8 = tid % BN, pb8 = tid / BN;
     const bool oka16 = i0 + ra16 < g.M, okb16 = j0 + rb16 < g.N;   // pair (r, r+1): r+1 may run past M: harmless
-    const bool oka8 = i0 + ra8 < g.M, okb8 = j0 + rb8 < g.N;
 
     auto load_stage = [&](int stage, int kt) {
         double *As = sm + stage * STAGE_WORDS;
         double *Bs = As + BK * SA;
         const int p0 = kt * BK;
         const double *__restrict__ Ak = A + (int64_t)p0 * lda;
-        if (!odd) {
 #pragma unroll
-            for (int p = pa16; p < BK; p += Cfg::PSA16) {
-                const bool ok = oka16 && (p0 + p < K);
-                cp_async16(As + p * SA + ra16, ok ? Ak + i0 + ra16 + (int64_t)p * lda : A, ok);
-            }
+        for (int p = pa16; p < BK; p += Cfg::PSA16) {
+            const bool ok = oka16 && (p0 + p < K);
+            cp_async16(As + p * SA + ra16, ok ? Ak + i0 + ra16 + (int64_t)p * lda : A, ok);
+        }
 #pragma unroll
-            for (int p = pb16; p < BK; p += Cfg::PSB16) {
-                const bool ok = okb16 && (p0 + p < K);
-                cp_async16(Bs + p * SB + rb16, ok ? Ak + j0 + rb16 + (int64_t)p * lda : A, ok);
-            }
-        } else {
-#pragma unroll
-            for (int p = pa8; p < BK; p += Cfg::PSA8) {
-                const bool ok = oka8 && (p0 + p < K);
-                cp_async8(As + p * SA + ra8, ok ? Ak + i0 + ra8 + (int64_t)p * lda : A, ok);
-            }
-#pragma unroll
-            for (int p = pb8; p < BK; p += Cfg::PSB8) {
-                const bool ok = okb8 && (p0 + p < K);
-                cp_async8(Bs + p * SB + rb8, ok ? Ak + j0 + rb8 + (int64_t)p * lda : A, ok);
-            }
+        for (int p = pb16; p < BK; p += Cfg::PSB16) {
+            const bool ok = okb16 && (p0 + p < K);
+            cp_async16(Bs + p * SB + rb16, ok ? Ak + j0 + rb16 + (int64_t)p * lda : A, ok);
         }
     };
 
@@ -128,7 +112,8 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
         if (st < KT) load_stage(st, st);
         cp_async_commit();
     }
-    double *__restrict__ C = (g.c_in_U ? Uarena : Larena) + g.c_off;
+    // C(i - sh, j - sh) for the (shifted) tile coordinates (i, j)
+    double *__restrict__ C = ((g.flags & 1) ? Uarena : Larena) + g.c_off;
     const int ldc = g.ldc;
     double acc[MB][NB][2];
 #pragma unroll
@@ -139,7 +124,8 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
 #pragma unroll
             for (int e = 0; e < 2; e++) {
                 const int j = j0 + wn * TN + nb * 8 + 2 * tq + e;
-                acc[mb][nb][e] = (i < g.M && j < g.N) ? C[i + (int64_t)j * ldc] : 0.0;
+                acc[mb][nb][e] =
+                    (i < g.M && j < g.N && i >= sh && j >= sh) ? C[(i - sh) + (int64_t)(j - sh) * ldc] : 0.0;
             }
     }
     for (int kt = 0; kt < KT; kt++) {
@@ -175,7 +161,7 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
 #pragma unroll
             for (int e = 0; e < 2; e++) {
                 const int j = j0 + wn * TN + nb * 8 + 2 * tq + e;
-                if (j < g.N && i >= j) C[i + (int64_t)j * ldc] = acc[mb][nb][e];
+                if (j < g.N && i >= j && j >= sh) C[(i - sh) + (int64_t)(j - sh) * ldc] = acc[mb][nb][e];
             }
     }
 }

@@ -53,13 +53,16 @@ int analyze_symbolic(int64_t n, const int64_t *colptr, const int32_t *rowind, co
 // A (lower-trapezoidal) Schur update problem:  C[i][j] -= sum_p A[i][p] * A[j][p]
 // for 0 <= j < N, j <= i < M (only entries with i >= j are written).
 // A: M x K, column-major, leading dim lda, inside the L arena.
-// C: column-major, leading dim ldc, inside the L arena (c_in_U = 0) or the U arena (1).
+// C: column-major, leading dim ldc, inside the L arena (flags bit 0 = 0) or the U
+// arena (1).  flags bit 1: the problem is shifted one row / column up-left so that
+// its first A row is even (16-byte staging); row / column 0 of the shifted space
+// are padding: C(i, j) of the kernel is C_orig(i - 1, j - 1).
 struct GemmProb {
     int64_t a_off;
     int64_t c_off;
     int32_t lda, ldc;
     int32_t M, N, K;
-    int32_t c_in_U;
+    int32_t flags;
 };
 static_assert(sizeof(GemmProb) == 40, "GemmProb layout");
 

@@ -405,7 +405,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
             g.M = M;
             g.N = N;
             g.K = K;
-            g.c_in_U = 0;
+            g.flags = 0;
             const int32_t pid = (int32_t)P.probs.size();
             P.probs.push_back(g);
             const int64_t t0 = (int64_t)P.tiles.size();
@@ -582,23 +582,29 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
             g.M = m;
             g.N = m;
             g.K = k;
-            g.c_in_U = 1;
+            g.flags = 1;
+            // odd first row (odd k): shift the problem one row / column up-left
+            const int32_t sh = (int32_t)(g.a_off & 1);
+            g.a_off -= sh;
+            g.M += sh;
+            g.N += sh;
+            g.flags |= sh << 1;
             const int32_t pid = (int32_t)P.probs.size();
             P.probs.push_back(g);
             if (!P.dist[s]) {
-                add_tiles(P, pid, m, m, [](int32_t) { return true; });
+                add_tiles(P, pid, g.M, g.N, [](int32_t) { return true; });
                 Ls.flops += upd_flops(m, m, k);
                 Ls.bytes += upd_bytes(m, m, k);
                 continue;
             }
-            const std::vector<int32_t> tb = split_tile_columns(m, R);
+            const std::vector<int32_t> tb = split_tile_columns(g.N, R);
             const int64_t t0 = (int64_t)P.tiles.size();
-            add_tiles(P, pid, m, m, [&](int32_t tj) { return tj >= tb[P.rank] && tj < tb[P.rank + 1]; });
-            const double frac = (double)((int64_t)P.tiles.size() - t0) / std::max<int64_t>(1, count_tiles(m, m));
+            add_tiles(P, pid, g.M, g.N, [&](int32_t tj) { return tj >= tb[P.rank] && tj < tb[P.rank + 1]; });
+            const double frac = (double)((int64_t)P.tiles.size() - t0) / (double)count_tiles(g.M, g.N);
             Ls.flops += frac * upd_flops(m, m, k);
             Ls.bytes += frac * upd_bytes(m, m, k);
-            for (int r = 0; r < R; r++) {
-                const int32_t c0 = tb[r] * kTileN, c1 = std::min(m, tb[r + 1] * kTileN);
+            for (int r = 0; r < R; r++) {   // original columns of rank r's shifted tile columns
+                const int32_t c0 = std::max(0, tb[r] * kTileN - sh), c1 = std::min(m, tb[r + 1] * kTileN - sh);
                 if (c1 <= c0) continue;
                 ux.push_back(XferSpec{MF_XFER_BCAST, r, 1, P.U_off[s] + (int64_t)c0 * m + c0,
                                       (int64_t)(c1 - c0 - 1) * m + (m - c0)});
@@ -609,6 +615,8 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         if (!ux.empty()) push_xfers(std::move(ux), l);
     }
     }   // pass
+    for (const GemmProb &g : P.probs)   // the DMMA kernel stages 16-byte row pairs
+        if ((g.a_off & 1) || (g.lda & 1)) return MF_ERR_STATE;
     P.df_blk_off.assign(ns, -1);
     P.df_part_off.assign(ns, -1);
     build_solve_plan(S, P, inc_local, P.fsolve, P.bsolve);
