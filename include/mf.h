@@ -74,6 +74,9 @@ typedef struct {
                                  fronts are shared by the exchange-cost model; 1 = always split (a
                                  frontier of >= nranks subtrees, every eligible top front shared),
                                  e.g. to exercise the cooperative path on small problems           */
+    int32_t nbranch;          /* single GPU: elimination subtrees are split into this many branches
+                                 that run concurrently (CUDA-graph branches on their own streams)
+                                 below the top fronts; 1 = one stream (default 4)                  */
 } mf_options;
 
 typedef struct {
@@ -108,7 +111,7 @@ typedef struct {
     double bytes;
 } mf_kernel_stat;
 
-#define MF_KERNEL_CLASSES 6
+#define MF_KERNEL_CLASSES 7
 
 /* Multi-GPU exchange.  With nranks > 1 every rank passes the
  * same n/colptr/rowind/perm/values/b; elimination subtrees are mapped to ranks and

@@ -36,6 +36,7 @@ struct mf_ctx {
     DevPlan d{};
     // device copies of schedule arrays
     int32_t *d_small = nullptr, *d_large = nullptr, *d_asm = nullptr, *d_trsm = nullptr, *d_levels = nullptr;
+    int32_t *d_panel = nullptr;
     int32_t *d_sn_rows = nullptr;
     int64_t *d_sn_rowptr = nullptr;
     GemmProb *d_probs = nullptr;
@@ -55,6 +56,9 @@ struct mf_ctx {
     double *d_ytmp = nullptr;
     int32_t *d_top_list = nullptr, *d_own_list = nullptr;
     std::vector<cudaEvent_t> prof_events;
+    // single GPU: one stream per subtree branch, forked from / joined into `stream`
+    std::vector<cudaStream_t> bstreams;
+    std::vector<cudaEvent_t> bevents;   // [0] fork, [1 + b] join of branch b
     mf_kernel_stat kstats[KC_COUNT];
     int64_t prof_factors = 0;
 };
@@ -182,6 +186,7 @@ int mf_default_options(mf_options *o) {
     o->rank = 0;
     o->stream = nullptr;
     o->split_all = 0;
+    o->nbranch = d.nbranch;
     return MF_OK;
 }
 
@@ -208,6 +213,11 @@ int mf_create(mf_ctx **out, const mf_options *o) {
     }
     c->opt.nranks = o->nranks;
     c->opt.split_all = o->split_all;
+    if (o->nbranch < 1 || o->nbranch > 64) {
+        delete c;
+        return MF_ERR_ARG;
+    }
+    c->opt.nbranch = o->nbranch;
     c->opt.rank = o->rank;
     c->host_only = o->host_only != 0;
     c->info.failed_col = -1;
@@ -255,6 +265,8 @@ void mf_destroy(mf_ctx *c) {
     if (c->stream) cudaStreamSynchronize(c->stream);
     free_device(c);
     for (cudaEvent_t e : c->prof_events) cudaEventDestroy(e);
+    for (cudaEvent_t e : c->bevents) cudaEventDestroy(e);
+    for (cudaStream_t bs : c->bstreams) cudaStreamDestroy(bs);
     if (c->ev0) cudaEventDestroy(c->ev0);
     if (c->ev1) cudaEventDestroy(c->ev1);
     if (c->own_stream) cudaStreamDestroy(c->stream);
@@ -309,6 +321,7 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     UP(&c->d_large, P.large_list);
     UP(&c->d_asm, P.asm_tasks);
     UP(&c->d_trsm, P.trsm_tasks);
+    UP(&c->d_panel, P.panel_tasks);
     UP(&c->d_levels, P.level_list);
     UP(&c->d_sn_rows, S.sn_rows);
     UP(&c->d_sn_rowptr, S.sn_rowptr);
@@ -360,6 +373,12 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     if ((r = dev_alloc(c, &p, std::max<int32_t>(P.nsuper, 1) * sizeof(unsigned))) != MF_OK) return r;
     d.leaf_flag = (unsigned *)p;
     CK(cudaMemsetAsync(d.leaf_flag, 0, std::max<int32_t>(P.nsuper, 1) * sizeof(unsigned), c->stream));
+    {
+        const size_t nf = (size_t)std::max<int32_t>(P.nsuper, 1) * kPanelFlags;
+        if ((r = dev_alloc(c, &p, nf * sizeof(unsigned))) != MF_OK) return r;
+        d.panel_flag = (unsigned *)p;
+        CK(cudaMemsetAsync(d.panel_flag, 0, nf * sizeof(unsigned), c->stream));
+    }
     CK(cudaMemsetAsync(c->d_failed, 0, sizeof(int) * 4, c->stream));
     if ((r = dev_alloc(c, &p, std::max<int64_t>(S.nnz_in, 1) * sizeof(double))) != MF_OK) return r;
     c->d_values = (double *)p;
@@ -369,6 +388,17 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     c->d_ytmp = (double *)p;
     if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(n, 1) * sizeof(double))) != MF_OK) return r;
     c->d_bx = (double *)p;
+    // subtree-branch streams (single GPU), created once per ctx
+    while ((int)c->bstreams.size() < P.nbranch) {
+        cudaStream_t bs;
+        CK(cudaStreamCreateWithFlags(&bs, cudaStreamNonBlocking));
+        c->bstreams.push_back(bs);
+    }
+    while ((int)c->bevents.size() < 1 + P.nbranch) {
+        cudaEvent_t e;
+        CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        c->bevents.push_back(e);
+    }
     // the L arena starts zeroed once so that never-written padding words are defined
     CK(cudaMemsetAsync(d.L, 0, P.L_words * sizeof(double), c->stream));
     CK(cudaStreamSynchronize(c->stream));
@@ -392,8 +422,32 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
     cudaStream_t st = c->stream;
     auto issue = [&](const double *v, bool with_events) -> int {
         if (with_init) launch_init_failed(c->d_failed, st);
+        // subtree branches run on their own streams (forked after the init launch,
+        // joined before the first top launch); profiled runs stay on one stream
+        const bool branches = !with_events && P.nbranch > 1 && (int)c->bstreams.size() >= P.nbranch;
+        bool forked = false, joined = false;
+        auto join = [&]() -> int {
+            for (int b = 0; b < P.nbranch; b++) {
+                CK(cudaEventRecord(c->bevents[1 + b], c->bstreams[b]));
+                CK(cudaStreamWaitEvent(st, c->bevents[1 + b], 0));
+            }
+            joined = true;
+            return MF_OK;
+        };
         for (size_t li = i0; li < i1; li++) {
             const Launch &L = prog[li];
+            cudaStream_t ls = st;
+            if (branches && L.stream >= 0) {
+                if (!forked) {
+                    CK(cudaEventRecord(c->bevents[0], st));
+                    for (int b = 0; b < P.nbranch; b++) CK(cudaStreamWaitEvent(c->bstreams[b], c->bevents[0], 0));
+                    forked = true;
+                }
+                ls = c->bstreams[L.stream];
+            } else if (branches && forked && !joined) {
+                if (int r = join()) return r;
+            }
+            auto launch = [&](cudaStream_t st) -> int {
             if (with_events) CK(cudaEventRecord(c->prof_events[ev_base + 2 * li], st));
             switch (L.kind) {
                 case KC_SMALL: launch_small_fronts(d, c->d_small + L.off, (int)L.count, L.param, v, st); break;
@@ -401,12 +455,19 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
                 case KC_POTRF: launch_potrf_diag(d, c->d_large + L.off, (int)L.count, L.param, P.w, st); break;
                 case KC_TRSM: launch_trsm_panel(d, c->d_trsm + 2 * L.off, L.count, L.param, P.w, st); break;
                 case KC_UPDATE: launch_update(d, c->d_probs, c->d_tiles + L.off, L.count, st); break;
+                case KC_PANEL: launch_panel(d, c->d_panel + 2 * L.off, L.count, L.param, (int)L.count2, st); break;
                 case KC_LEAF:
                     launch_leaf(d, c->d_large + L.off, (int)L.count, c->d_trsm + 2 * L.off2, L.count2, L.param, P.w, st);
                     break;
                 default: return MF_ERR_STATE;   // exchange points are handled by run_with_exchanges
             }
             if (with_events) CK(cudaEventRecord(c->prof_events[ev_base + 2 * li + 1], st));
+            return MF_OK;
+            };
+            if (int r = launch(ls)) return r;
+        }
+        if (forked && !joined) {
+            if (int r = join()) return r;
         }
         return MF_OK;
     };
@@ -714,7 +775,8 @@ int mf_export_panel(const mf_ctx *c, int32_t s, double *out) {
 }
 
 static const char *kKernelNames[KC_COUNT] = {"small_front_fused", "assemble_extend_add", "potrf_diag",
-                                             "trsm_panel", "dmma_schur_update", "leaf_potrf_trsm"};
+                                             "trsm_panel", "dmma_schur_update", "leaf_potrf_trsm",
+                                             "dataflow_panel"};
 
 int mf_set_profiling(mf_ctx *c, int enable) {
     if (!c) return MF_ERR_ARG;

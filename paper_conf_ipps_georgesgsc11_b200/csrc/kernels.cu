@@ -681,6 +681,534 @@ void launch_leaf(const DevPlan &d, const int32_t *fronts, int npotrf, const int3
     k_leaf<<<(unsigned)(npotrf + ntrsm), kTrsmThreads, kTrsmSmem, st>>>(d, fronts, npotrf, tasks, j0, w);
 }
 
+// ============================================================ dataflow panel ("super-leaf")
+// The base case of the recursive blocked factorization of the large fronts
+// (Fig. 9: "a light-weight GPU kernel performing potrf on a w x w
+// matrix", trsm on the rows below, the trailing update of the panel) for up to
+// kPanelMaxBlocks blocks of 64 pivot columns [j0, j0 + 64 nbk), in ONE launch.
+// A task is one 64-row tile row c (rows j0 + 64c ...) of one front; the tiles
+// (c, b), b <= c, of that row are produced in order b = 0, 1, ...:
+//   off-diagonal (b < c): X(c,b) -= sum_{b' < b} X(c,b') X(b,b')^T  (DMMA, K = 64 b,
+//       operands from L2), wait for the diagonal tile (b,b), X(c,b) <- X(c,b) L_bb^-T
+//       (substitution), store;
+//   diagonal (b = c, the "band" tiles c < nb): the row's own products
+//       X(c,b) X(c,b)^T are subtracted as each X(c,b) is finished (registers),
+//       then potrf in shared memory, store, publish.
+// Tiles publish epoch-tagged flags (band tiles (c,b) and the diagonal tiles);
+// a task only waits on tasks of the same front with a smaller row index, which
+// have smaller block indices (tasks are ordered row-major over the fronts), so
+// the launch cannot deadlock.  This replaces, per panel of 4 blocks, 4 fused
+// leaf launches and 3 narrow update launches whose latency serialised the
+// factorization of the top fronts.
+constexpr int kPanelThreads = 128;
+constexpr int kPLD = 68;   // 64-row tiles in shared memory: stride = 4 mod 16 (conflict-free fragments), even (16-byte cp.async)
+constexpr int kPanelRingWords = 3 * 16 * (2 * kPLD);   // 3-stage cp.async ring of 16-wide A / B slices
+constexpr size_t kPanelSmem = (size_t)(kPanelRingWords + 64 * kPLD + 64) * sizeof(double);
+static_assert(64 * kPLD <= kPanelRingWords, "the L_bb tile aliases the staging ring");
+
+__device__ __forceinline__ int panel_tri(int c, int b) { return c * (c + 1) / 2 + b; }
+
+// Optional device-side timeline of the panel tasks (tools/ubench/panel_bench.cu
+// compiles this file with -DMF_PANEL_TRACE); compiled out of libmf.
+#ifdef MF_PANEL_TRACE
+__device__ unsigned long long g_panel_trace[4096][32];
+__device__ __forceinline__ void panel_mark(int ev) {
+    if (threadIdx.x == 0 && blockIdx.x < 4096 && ev < 32) {
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        g_panel_trace[blockIdx.x][ev] = t;
+    }
+}
+#define PANEL_MARK(ev) panel_mark(ev)
+#else
+#define PANEL_MARK(ev)
+#endif
+
+// acc(64 x 64 tile; this warp's 32 x 32 fragment) -= A B^T with A = rows [ra0, ra0+64),
+// B = rows [rb0, rb0+64), columns [kc0, kc0 + K) of the panel Pn (column-major, ld);
+// rows >= arows / brows read as zero.  K is a multiple of 16.
+__device__ __forceinline__ void panel_tile_mma(double (&acc)[4][4][2], double *ring, const double *__restrict__ Pn,
+                                               int ld, int ra0, int arows, int rb0, int brows, int kc0, int K) {
+    constexpr int BK = 16, STAGES = 3, STW = BK * 2 * kPLD;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int wm = warp & 1, wn = warp >> 1, gq = lane >> 2, tq = lane & 3;
+    const int rr = 2 * lane, pt = warp;   // staging slot: row pair rr, k offsets pt + 4 i
+    const bool oka = rr < arows, okb = rr < brows;
+    auto load_stage = [&](int stage, int kt) {
+        double *As = ring + stage * STW, *Bs = As + BK * kPLD;
+        const double *__restrict__ Ak = Pn + (int64_t)(kc0 + kt * BK) * ld;
+#pragma unroll
+        for (int i = 0; i < 4; i++) {
+            const int p = pt + 4 * i;
+            cp_async16(As + p * kPLD + rr, oka ? Ak + (int64_t)p * ld + ra0 + rr : Pn, oka);
+            cp_async16(Bs + p * kPLD + rr, okb ? Ak + (int64_t)p * ld + rb0 + rr : Pn, okb);
+        }
+    };
+    const int KT = K / BK;
+#pragma unroll
+    for (int st = 0; st < STAGES - 1; st++) {
+        if (st < KT) load_stage(st, st);
+        cp_async_commit();
+    }
+    for (int kt = 0; kt < KT; kt++) {
+        cp_async_wait<STAGES - 2>();
+        __syncthreads();
+        {
+            const int nk = kt + STAGES - 1;
+            if (nk < KT) load_stage(nk % STAGES, nk);
+            cp_async_commit();
+        }
+        const double *As = ring + (kt % STAGES) * STW + wm * 32 + gq;
+        const double *Bs = ring + (kt % STAGES) * STW + BK * kPLD + wn * 32 + gq;
+#pragma unroll
+        for (int kk = 0; kk < BK / 4; kk++) {
+            double a[4], b[4];
+#pragma unroll
+            for (int mb = 0; mb < 4; mb++) a[mb] = -As[(kk * 4 + tq) * kPLD + mb * 8];
+#pragma unroll
+            for (int nb = 0; nb < 4; nb++) b[nb] = Bs[(kk * 4 + tq) * kPLD + nb * 8];
+#pragma unroll
+            for (int mb = 0; mb < 4; mb++)
+#pragma unroll
+                for (int nb = 0; nb < 4; nb++) dmma(acc[mb][nb][0], acc[mb][nb][1], a[mb], b[nb]);
+        }
+    }
+    cp_async_wait<0>();
+    __syncthreads();   // the ring is reused by the caller
+}
+
+// tile (rows r0.., cols c0..) of the panel <-> fragment registers / shared memory
+__device__ __forceinline__ void panel_frag_load(double (&acc)[4][4][2], const double *__restrict__ Pn, int ld, int r0,
+                                                int rows, int c0, int cols) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, wm = warp & 1, wn = warp >> 1;
+#pragma unroll
+    for (int mb = 0; mb < 4; mb++) {
+        const int i = wm * 32 + mb * 8 + (lane >> 2);
+#pragma unroll
+        for (int nb = 0; nb < 4; nb++)
+#pragma unroll
+            for (int e = 0; e < 2; e++) {
+                const int j = wn * 32 + nb * 8 + 2 * (lane & 3) + e;
+                acc[mb][nb][e] = (i < rows && j < cols) ? Pn[(r0 + i) + (int64_t)(c0 + j) * ld] : 0.0;
+            }
+    }
+}
+__device__ __forceinline__ void panel_frag_to_smem(const double (&acc)[4][4][2], double *Xs) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, wm = warp & 1, wn = warp >> 1;
+#pragma unroll
+    for (int mb = 0; mb < 4; mb++) {
+        const int i = wm * 32 + mb * 8 + (lane >> 2);
+#pragma unroll
+        for (int nb = 0; nb < 4; nb++)
+#pragma unroll
+            for (int e = 0; e < 2; e++) Xs[i + (wn * 32 + nb * 8 + 2 * (lane & 3) + e) * kPLD] = acc[mb][nb][e];
+    }
+}
+
+// Factor the first `we` columns of the R x we panel A (shared memory, column-major,
+// stride kPLD; R <= 64 rows, the top we x we block is the diagonal block): the
+// algorithm of potrf_block, extended to rows below the diagonal block (the last
+// block of a front whose k ends inside a 64-row tile).
+__device__ __forceinline__ void panel_potrf(const DevPlan &d, double *A, double *sinv, int R, int we, int first_col) {
+    constexpr int SB = 8, G = kPanelThreads / 64;
+    const int tid = threadIdx.x;
+#pragma unroll 1
+    for (int s0 = 0; s0 < we; s0 += SB) {
+        const int nb = min(SB, we - s0);
+        if (tid == 0) {
+            double a[SB][SB];
+#pragma unroll
+            for (int c = 0; c < SB; c++)
+#pragma unroll
+                for (int r = c; r < SB; r++) a[r][c] = (r < nb) ? A[(s0 + c) * kPLD + s0 + r] : (r == c ? 1.0 : 0.0);
+#pragma unroll
+            for (int q = 0; q < SB; q++) {
+                if (q < nb) note_pivot(d, a[q][q], first_col + s0 + q);
+                const double inv = rsqrt(a[q][q]);
+                a[q][q] *= inv;
+                sinv[s0 + q] = inv;
+#pragma unroll
+                for (int r = q + 1; r < SB; r++) a[r][q] *= inv;
+#pragma unroll
+                for (int c = q + 1; c < SB; c++)
+#pragma unroll
+                    for (int r = c; r < SB; r++) a[r][c] = fma(-a[r][q], a[c][q], a[r][c]);
+            }
+#pragma unroll
+            for (int c = 0; c < SB; c++)
+#pragma unroll
+                for (int r = c; r < SB; r++)
+                    if (r < nb) A[(s0 + c) * kPLD + s0 + r] = a[r][c];
+        }
+        __syncthreads();
+        const int rb = s0 + nb;
+        if (rb >= R) break;
+        // rows [rb, R) against the sub-block (columns >= nb of a partial sub-block are padding)
+        if (tid < R - rb) {
+            const int r = rb + tid;
+            double x[SB];
+#pragma unroll
+            for (int q = 0; q < SB; q++) x[q] = (q < nb) ? A[(s0 + q) * kPLD + r] : 0.0;
+#pragma unroll
+            for (int q = 0; q < SB; q++) {
+                if (q < nb) {
+                    x[q] *= sinv[s0 + q];
+#pragma unroll
+                    for (int q2 = q + 1; q2 < SB; q2++)
+                        if (q2 < nb) x[q2] -= x[q] * A[(s0 + q) * kPLD + s0 + q2];
+                }
+            }
+#pragma unroll
+            for (int q = 0; q < SB; q++)
+                if (q < nb) A[(s0 + q) * kPLD + r] = x[q];
+        }
+        __syncthreads();
+        // trailing update of columns [rb, we), rows i >= column
+        if (rb < we) {
+            const int i = tid & 63, h = tid >> 6;
+            if (i >= rb && i < R) {
+                double li[SB];
+#pragma unroll
+                for (int q = 0; q < SB; q++) li[q] = A[(s0 + q) * kPLD + i];
+                const int cmax = min(i, we - 1);
+                for (int c = rb + h; c <= cmax; c += G) {
+                    double acc = A[c * kPLD + i];
+#pragma unroll
+                    for (int q = 0; q < SB; q++) acc -= li[q] * A[(s0 + q) * kPLD + c];
+                    A[c * kPLD + i] = acc;
+                }
+            }
+        }
+        __syncthreads();
+    }
+}
+
+// 1/sqrt(x): MUFU.RSQ64H seed + two Newton steps (exact 2^-p for x = 4^p, so the
+// manufactured integer factors stay exact; ~1 ulp otherwise, reading C9).
+// Non-positive / NaN pivots come out NaN and are flagged by the caller.
+__device__ __forceinline__ double rsqrt_nr(double x) {
+    double y;
+    asm("rsqrt.approx.ftz.f64 %0, %1;" : "=d"(y) : "d"(x));
+    double r = fma(-x * y, y, 1.0);
+    y = fma(0.5 * y, r, y);
+    r = fma(-x * y, y, 1.0);
+    return fma(0.5 * y, r, y);
+}
+
+// Factor the nb x nb (nb <= 8) pivot block at (s0, s0) of A (shared memory, stride
+// kPLD) in ONE thread's registers; 1/L_jj to sinv[s0 + j].  The pivot chain is
+// written first in each step; the first non-positive / NaN pivot is reported once
+// at the end (reading C8: only later columns can be contaminated).
+__device__ __forceinline__ void factor_diag8(const DevPlan &d, double *A, double *sinv, int s0, int nb, int first_col) {
+    constexpr int SB = 8;
+    double a[SB][SB];
+#pragma unroll
+    for (int c = 0; c < SB; c++)
+#pragma unroll
+        for (int r = c; r < SB; r++) a[r][c] = (r < nb) ? A[(s0 + c) * kPLD + s0 + r] : (r == c ? 1.0 : 0.0);
+    int bad = SB;
+#pragma unroll
+    for (int q = 0; q < SB; q++) {
+        const double dq = a[q][q];
+        if (!(dq > 0.0) && q < nb && bad == SB) bad = q;
+        const double inv = rsqrt_nr(dq);
+        if (q + 1 < SB) {   // the next pivot first
+            a[q + 1][q] *= inv;
+            a[q + 1][q + 1] = fma(-a[q + 1][q], a[q + 1][q], a[q + 1][q + 1]);
+        }
+        a[q][q] = dq * inv;
+        sinv[s0 + q] = inv;
+#pragma unroll
+        for (int r = q + 2; r < SB; r++) a[r][q] *= inv;
+#pragma unroll
+        for (int c = q + 1; c < SB; c++)
+#pragma unroll
+            for (int r = c; r < SB; r++)
+                if (r != q + 1) a[r][c] = fma(-a[r][q], a[c][q], a[r][c]);   // (q+1, q+1) was done first
+    }
+#pragma unroll
+    for (int c = 0; c < SB; c++)
+#pragma unroll
+        for (int r = c; r < SB; r++)
+            if (r < nb) A[(s0 + c) * kPLD + s0 + r] = a[r][c];
+    if (bad < SB) atomicMin(d.failed, first_col + s0 + bad);
+}
+
+// C_IJ -= L_I L_J^T for the 8 x 8 blocks (I, J) of A over the 8 columns [s0, s0+8)
+// (one warp, DMMA m8n8k4 twice)
+__device__ __forceinline__ void upd_block8(double *A, int I, int J, int s0) {
+    const int lane = threadIdx.x & 31, gq = lane >> 2, tq = lane & 3;
+    double *Ci = A + I * 8 + gq;
+    double c0 = Ci[(J * 8 + 2 * tq) * kPLD], c1 = Ci[(J * 8 + 2 * tq + 1) * kPLD];
+#pragma unroll
+    for (int kk = 0; kk < 2; kk++) {
+        const double av = -Ci[(s0 + kk * 4 + tq) * kPLD];
+        const double bv = A[J * 8 + gq + (s0 + kk * 4 + tq) * kPLD];
+        dmma(c0, c1, av, bv);
+    }
+    Ci[(J * 8 + 2 * tq) * kPLD] = c0;
+    Ci[(J * 8 + 2 * tq + 1) * kPLD] = c1;
+}
+
+// Same contract as panel_potrf, restructured for latency: per 8-column step the
+// 8 x 8 pivot block is factored by one thread in registers (factor_diag8), the
+// rows below solve it one thread per row, and the trailing lower 8 x 8 blocks are
+// updated with DMMA (K = 8).  Look-ahead: warp 0 updates the next block column
+// and its lane 0 factors the next pivot block while warps 1-3 update the rest.
+__device__ __forceinline__ void panel_potrf_dmma(const DevPlan &d, double *A, double *sinv, int R, int we,
+                                                 int first_col) {
+    constexpr int SB = 8;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int nrb = (R + 7) / 8, ncb = (we + 7) / 8;
+#ifdef MF_PANEL_TRACE
+    long long ta = 0, tb = 0, tc = 0, x1 = 0, x2 = 0;
+    x1 = clock64();
+#endif
+    if (tid == 0) factor_diag8(d, A, sinv, 0, min(SB, we), first_col);
+    __syncthreads();
+#ifdef MF_PANEL_TRACE
+    ta += clock64() - x1;
+#endif
+#pragma unroll 1
+    for (int st = 0; st < ncb; st++) {
+        const int s0 = st * SB, nb = min(SB, we - s0);
+        const int rb = s0 + nb;
+        if (rb >= R) break;
+#ifdef MF_PANEL_TRACE
+        x1 = clock64();
+#endif
+        // rows [rb, R) against the factored pivot block st
+        if (tid < R - rb) {
+            const int r = rb + tid;
+            double x[SB];
+#pragma unroll
+            for (int q = 0; q < SB; q++) x[q] = (q < nb) ? A[(s0 + q) * kPLD + r] : 0.0;
+#pragma unroll
+            for (int q = 0; q < SB; q++) {
+                if (q < nb) {
+                    x[q] *= sinv[s0 + q];
+#pragma unroll
+                    for (int q2 = q + 1; q2 < SB; q2++) x[q2] = fma(-x[q], A[(s0 + q) * kPLD + s0 + q2], x[q2]);
+                }
+            }
+#pragma unroll
+            for (int q = 0; q < SB; q++)
+                if (q < nb) A[(s0 + q) * kPLD + r] = x[q];
+        }
+        __syncthreads();
+#ifdef MF_PANEL_TRACE
+        x2 = clock64();
+        tb += x2 - x1;
+#endif
+        if (st + 1 < ncb) {
+            const int J1 = st + 1;
+            if (warp == 0) {
+                // the next pivot block only, then its factorization (the critical chain)
+                upd_block8(A, J1, J1, s0);
+                __syncwarp();
+                if (lane == 0) factor_diag8(d, A, sinv, J1 * SB, min(SB, we - J1 * SB), first_col);
+            } else {
+                int t = 0;
+                for (int J = J1; J < ncb; J++)
+                    for (int I = (J == J1 ? J + 1 : J); I < nrb; I++, t++)
+                        if (t % 3 == warp - 1) upd_block8(A, I, J, s0);
+            }
+        }
+        __syncthreads();
+#ifdef MF_PANEL_TRACE
+        tc += clock64() - x2;
+#endif
+    }
+#ifdef MF_PANEL_TRACE
+    if (threadIdx.x == 0 && blockIdx.x < 4096) {
+        g_panel_trace[blockIdx.x][25] = ta; g_panel_trace[blockIdx.x][26] = tb; g_panel_trace[blockIdx.x][27] = tc;
+    }
+#endif
+}
+
+// X <- X L^-T for the 64 rows of Xs over wb columns; Ls = the wb x wb lower factor
+// (identity-padded to a multiple of 8), inv = 1 / diag.  8-column blocks: one
+// thread per row solves the block (substitution), then the four warps apply it
+// to the remaining columns with DMMA (16 rows each).
+__device__ __forceinline__ void panel_trsm(double *Xs, const double *Ls, const double *inv, int wb) {
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, gq = lane >> 2, tq = lane & 3;
+    const int ncb = (wb + 7) / 8;
+#pragma unroll 1
+    for (int cb = 0; cb < ncb; cb++) {
+        const int c0 = cb * 8;
+        if (tid < 64) {
+            double xv[8];
+#pragma unroll
+            for (int q = 0; q < 8; q++) xv[q] = Xs[tid + (c0 + q) * kPLD];
+#pragma unroll
+            for (int q = 0; q < 8; q++) {
+                xv[q] *= inv[c0 + q];
+#pragma unroll
+                for (int q2 = q + 1; q2 < 8; q2++) xv[q2] -= xv[q] * Ls[(c0 + q2) + (c0 + q) * kPLD];
+            }
+#pragma unroll
+            for (int q = 0; q < 8; q++) Xs[tid + (c0 + q) * kPLD] = xv[q];
+        }
+        __syncthreads();
+        // X[:, nbk] -= X[:, cb] L[nbk, cb]^T for nbk > cb: this warp's 16 rows, all
+        // column blocks at once (static indices: loads batched ahead of the DMMAs)
+        {
+            double av[2][2];
+#pragma unroll
+            for (int mb = 0; mb < 2; mb++)
+#pragma unroll
+                for (int kk = 0; kk < 2; kk++) av[mb][kk] = -Xs[warp * 16 + mb * 8 + gq + (c0 + kk * 4 + tq) * kPLD];
+#pragma unroll
+            for (int nbk = 1; nbk < 8; nbk++) {
+                if (nbk <= cb || nbk >= ncb) continue;
+                const double b0 = Ls[(nbk * 8 + gq) + (c0 + tq) * kPLD], b1 = Ls[(nbk * 8 + gq) + (c0 + 4 + tq) * kPLD];
+#pragma unroll
+                for (int mb = 0; mb < 2; mb++) {
+                    double *xr = Xs + warp * 16 + mb * 8 + gq + (nbk * 8 + 2 * tq) * kPLD;
+                    double acc0 = xr[0], acc1 = xr[kPLD];
+                    dmma(acc0, acc1, av[mb][0], b0);
+                    dmma(acc0, acc1, av[mb][1], b1);
+                    xr[0] = acc0;
+                    xr[kPLD] = acc1;
+                }
+            }
+        }
+        __syncthreads();
+    }
+}
+
+__device__ __forceinline__ void panel_publish(unsigned *flag, unsigned tag) {
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(flag), "r"(tag) : "memory");
+}
+
+__global__ void __launch_bounds__(kPanelThreads, 2) k_panel(DevPlan d, const int32_t *__restrict__ tasks, int j0,
+                                                             int nbk) {
+    extern __shared__ __align__(16) double psm[];
+    double *ring = psm;                         // accumulate staging; the L_bb tile afterwards
+    double *Xs = psm + kPanelRingWords;         // the tile being finished
+    double *inv = Xs + 64 * kPLD;
+    const int s = tasks[2 * blockIdx.x], c = tasks[2 * blockIdx.x + 1];
+    const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s];
+    const int nb = min(nbk, (k - j0 + 63) / 64);
+    const int r0 = j0 + 64 * c, rows = min(64, f - r0);
+    double *__restrict__ Pn = d.L + d.L_off[s];
+    unsigned *F = d.panel_flag + (int64_t)s * kPanelFlags;
+    const unsigned tag = ((*d.epoch & 0x3fffffu) << 10) | (unsigned)(j0 / 64 + 1);
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, gq = lane >> 2, tq = lane & 3;
+    const bool band = c < nb;
+    // the diagonal tile's accumulator: its 36 lower 8 x 8 blocks, 9 per warp
+    // (block rows `warp` and 7 - warp), so the row's own products cost 144 DMMA per warp
+    double dacc[9][2];
+    PANEL_MARK(0);
+    if (band) {
+        const int cols = min(64, k - r0);
+#pragma unroll
+        for (int t = 0; t < 9; t++) {
+            const int I = t <= warp ? warp : 7 - warp, J = t <= warp ? t : t - warp - 1;
+            const int i = I * 8 + gq;
+#pragma unroll
+            for (int e = 0; e < 2; e++) {
+                const int j = J * 8 + 2 * tq + e;
+                dacc[t][e] = (i < rows && j < cols) ? Pn[(r0 + i) + (int64_t)(r0 + j) * ld] : 0.0;
+            }
+        }
+    }
+    const int nsteps = min(c, nb);
+#pragma unroll 1
+    for (int b = 0; b < nsteps; b++) {
+        const int cb0 = j0 + 64 * b, wb = min(64, k - cb0);
+        double acc[4][4][2];
+        panel_frag_load(acc, Pn, ld, r0, rows, cb0, wb);
+        if (b > 0) {
+            wait_flag(F + panel_tri(b, b - 1), tag);   // band tiles (b, 0..b-1) are final
+            PANEL_MARK(1 + 6 * b);
+            panel_tile_mma(acc, ring, Pn, ld, r0, rows, cb0, min(64, f - cb0), j0, 64 * b);
+        }
+        panel_frag_to_smem(acc, Xs);
+        PANEL_MARK(2 + 6 * b);
+        wait_flag(F + panel_tri(b, b), tag);           // L_bb is final
+        PANEL_MARK(3 + 6 * b);
+        {
+            const double *__restrict__ D = Pn + (int64_t)cb0 * ld + cb0;
+            for (int q = tid; q < 32 * 64; q += kPanelThreads) {
+                const int rr = 2 * (q & 31), cc = q >> 5;
+                const bool ok = cc < wb && rr < wb;
+                cp_async16(ring + rr + cc * kPLD, ok ? D + rr + (int64_t)cc * ld : D, ok);
+            }
+            cp_async_commit();
+            cp_async_wait<0>();
+            __syncthreads();
+            if (tid < 64) {
+                if (tid >= wb) {
+                    for (int cc = 0; cc < 64; cc++) ring[tid + cc * kPLD] = (cc == tid) ? 1.0 : 0.0;
+                } else {
+                    for (int cc = wb; cc < 64; cc++) ring[tid + cc * kPLD] = 0.0;
+                }
+            }
+            __syncthreads();
+            if (tid < 64) inv[tid] = __drcp_rn(ring[tid + tid * kPLD]);
+            __syncthreads();
+        }
+        PANEL_MARK(4 + 6 * b);
+        panel_trsm(Xs, ring, inv, wb);
+        PANEL_MARK(5 + 6 * b);
+        for (int q = tid; q < 64 * 64; q += kPanelThreads) {
+            const int i = q & 63, j = q >> 6;
+            if (i < rows && j < wb) Pn[(r0 + i) + (int64_t)(cb0 + j) * ld] = Xs[i + j * kPLD];
+        }
+        if (band) {
+            panel_publish(F + panel_tri(c, b), tag);   // X(c,b) is stored: band tile final
+            // the row's own product: dacc -= X(c,b) X(c,b)^T (b < c < nb, so wb = 64)
+            const double *Xg = Xs + gq;
+#pragma unroll 2
+            for (int kk = 0; kk < 16; kk++) {
+                const double *Xk = Xg + (kk * 4 + tq) * kPLD;
+                const double a0 = -Xk[warp * 8], a1 = -Xk[(7 - warp) * 8];
+                double bj[9];
+#pragma unroll
+                for (int t = 0; t < 9; t++) bj[t] = Xk[(t <= warp ? t : t - warp - 1) * 8];
+#pragma unroll
+                for (int t = 0; t < 9; t++) dmma(dacc[t][0], dacc[t][1], t <= warp ? a0 : a1, bj[t]);
+            }
+            __syncthreads();   // Xs / ring are rewritten by the next step
+            PANEL_MARK(6 + 6 * b);
+        } else {
+            __syncthreads();   // Xs / ring are rewritten by the next step
+        }
+    }
+    if (band) {
+        const int we = min(64, k - r0);
+        __syncthreads();
+#pragma unroll
+        for (int t = 0; t < 9; t++) {
+            const int I = t <= warp ? warp : 7 - warp, J = t <= warp ? t : t - warp - 1;
+#pragma unroll
+            for (int e = 0; e < 2; e++) Xs[I * 8 + gq + (J * 8 + 2 * tq + e) * kPLD] = dacc[t][e];
+        }
+        __syncthreads();
+        PANEL_MARK(28);
+#ifdef MF_PANEL_OLD_POTRF
+        panel_potrf(d, Xs, inv, rows, we, d.sn_first[s] + r0);
+#else
+        panel_potrf_dmma(d, Xs, inv, rows, we, d.sn_first[s] + r0);
+#endif
+        PANEL_MARK(29);
+        for (int q = tid; q < 64 * 64; q += kPanelThreads) {
+            const int i = q & 63, j = q >> 6;
+            if (i < rows && j < we && i >= j) Pn[(r0 + i) + (int64_t)(r0 + j) * ld] = Xs[i + j * kPLD];
+        }
+        panel_publish(F + panel_tri(c, c), tag);
+        PANEL_MARK(30);
+    }
+}
+
+void launch_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int nbk, cudaStream_t st) {
+    if (count <= 0) return;
+    k_panel<<<(unsigned)count, kPanelThreads, kPanelSmem, st>>>(d, tasks, j0, nbk);
+}
+
 void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, cudaStream_t st) {
     if (count <= 0) return;
     k_trsm_panel<<<(unsigned)count, kTrsmThreads, kTrsmSmem, st>>>(d, tasks, j0, w);
@@ -708,6 +1236,8 @@ int kernels_init() {
         e = cudaFuncSetAttribute(k_trsm_panel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTrsmSmem);
     if (e == cudaSuccess)
         e = cudaFuncSetAttribute(k_leaf, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTrsmSmem);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_panel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kPanelSmem);
     if (e == cudaSuccess)
         e = cudaFuncSetAttribute(k_update_t<UpdProd>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)UpdProd::SMEM);
     return e == cudaSuccess ? 0 : -1;

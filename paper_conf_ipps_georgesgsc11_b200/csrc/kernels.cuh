@@ -25,6 +25,7 @@ struct DevPlan {
     int *failed;             // min failing pivot column (final labels); INT_MAX = none
     const unsigned *epoch;   // factorization counter (= failed + 1), bumped by the init kernel
     unsigned *leaf_flag;     // per supernode: fused-leaf "diagonal block done" flag
+    unsigned *panel_flag;    // per supernode: kPanelFlags dataflow-panel tile flags
     unsigned *solve_epoch;   // solve counter (= failed + 2), bumped by the first solve kernel
     unsigned *df_flags;      // dataflow solve flags (forward per block, backward per chunk)
     double *df_parts;        // dataflow backward partial sums per (chunk, block)
@@ -38,6 +39,7 @@ void launch_small_fronts(const DevPlan &d, const int32_t *list, int count, int f
 void launch_assemble(const DevPlan &d, const int32_t *tasks, int64_t count, const double *values, cudaStream_t st);
 void launch_leaf(const DevPlan &d, const int32_t *fronts, int npotrf, const int32_t *tasks, int64_t ntrsm, int j0,
                  int w, cudaStream_t st);
+void launch_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int nbk, cudaStream_t st);
 void launch_potrf_diag(const DevPlan &d, const int32_t *fronts, int count, int j0, int w, cudaStream_t st);
 void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, cudaStream_t st);
 void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, cudaStream_t st);

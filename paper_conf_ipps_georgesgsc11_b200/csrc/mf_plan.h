@@ -22,6 +22,7 @@ struct Options {
     int nranks = 1;   // GPUs sharing one factorization (one process per GPU)
     int rank = 0;
     int split_all = 0;   // multi-GPU mapping ignores the exchange-cost model
+    int nbranch = 4;     // single GPU: concurrent subtree branches (graph branches on their own streams)
 };
 
 // ---------------------------------------------------------------- symbolic
@@ -80,10 +81,15 @@ enum KernelClass : int32_t {
     KC_TRSM = 3,      // panel trsm below the diagonal block
     KC_UPDATE = 4,    // DMMA Schur update (panel trailing update and the syrk on U^n)
     KC_LEAF = 5,      // fused potrf + trsm of one diagonal block (few active fronts)
-    KC_COUNT = 6,
+    KC_PANEL = 6,     // dataflow panel: potrf + trsm + inner updates of up to kPanelMaxBlocks blocks of 64 columns
+    KC_COUNT = 7,
     KC_EXCHANGE = 16  // multi-GPU: hand the transfer group Plan::xfers[param] to the exchange callback
 };
 constexpr int kFuseLeafMaxFronts = 8;
+// Dataflow panel (KC_PANEL, w = 64 only): base case of the recursive blocked
+// factorization; per front kPanelFlags epoch-tagged flags (band tiles + diagonal tiles).
+constexpr int kPanelMaxBlocks = 4;
+constexpr int kPanelFlags = kPanelMaxBlocks * (kPanelMaxBlocks + 1) / 2;
 
 // One transfer of a multi-GPU exchange point, relative to the L or U arena.
 struct XferSpec {
@@ -101,7 +107,8 @@ struct Launch {
     double flops;       // algorithmic flops of this launch
     double bytes;       // algorithmic HBM bytes of this launch
     int32_t level;
-    int64_t off2 = 0, count2 = 0;   // KC_LEAF: the trsm tasks (off/count = the fronts)
+    int64_t off2 = 0, count2 = 0;   // KC_LEAF: the trsm tasks (off/count = the fronts); KC_PANEL: count2 = blocks
+    int32_t stream = -1;            // single GPU: subtree branch (its own stream), -1 = the main stream
 };
 
 // Triangular-solve program (forward sweep bottom-up, backward sweep top-down).
@@ -135,6 +142,7 @@ struct Plan {
     std::vector<int32_t> large_list;
     std::vector<int32_t> asm_tasks;                  // pairs (front, c0)
     std::vector<int32_t> trsm_tasks;                 // pairs (front, row0)
+    std::vector<int32_t> panel_tasks;                // pairs (front, 64-row tile row), row-major over the fronts
     std::vector<GemmProb> probs;
     std::vector<TileTask> tiles;
     std::vector<Launch> program;
@@ -150,6 +158,8 @@ struct Plan {
     // broadcast, and the large ones are factored cooperatively (block-cyclic pivot
     // columns, split trailing updates, all-gathered U^n).
     int32_t nranks = 1, rank = 0, split_all = 0;
+    int32_t nbranch = 1;                             // single GPU: subtree branches actually used
+    std::vector<int32_t> branch;                     // per supernode: its branch, -1 = top (main stream)
     std::vector<int32_t> owner;                      // rank factoring each supernode
     std::vector<char> top;                           // above the frontier (replicated)
     std::vector<char> dist;                          // top fronts factored cooperatively

@@ -241,6 +241,57 @@ static void map_subtrees(Plan &P, const std::vector<double> &front_load) {
     std::sort(P.frontier_roots.begin(), P.frontier_roots.end());
 }
 
+// Single GPU: split the elimination tree into concurrent branches (the paper's
+// task parallelism over independent subtrees [PAPER.md L443, L797], here as CUDA-
+// graph branches on their own streams of ONE GPU).  The heaviest expandable
+// frontier subtree is moved into the "top" until the frontier holds >= B
+// subtrees; those are assigned to B branches by LPT on executed flops.  The top
+// fronts run on the main stream after every branch has finished.  While one
+// branch runs latency-bound work (pivot chains, small fronts, narrow updates,
+// assembly), the others keep the DMMA pipes busy.
+static void assign_branches(Plan &P, const std::vector<double> &front_load, int B) {
+    const int32_t ns = P.nsuper;
+    P.branch.assign(ns, -1);
+    P.nbranch = 1;
+    if (B <= 1 || ns == 0) return;
+    std::vector<double> sub(front_load);
+    std::vector<int32_t> parent(ns, -1);
+    for (int32_t s = 0; s < ns; s++)
+        for (int32_t q = P.child_ptr[s]; q < P.child_ptr[s + 1]; q++) {
+            sub[s] += sub[P.child_list[q]];
+            parent[P.child_list[q]] = s;
+        }
+    std::vector<int32_t> fr;
+    for (int32_t s = 0; s < ns; s++)
+        if (parent[s] < 0) fr.push_back(s);
+    while ((int)fr.size() < B) {
+        int32_t pick = -1;
+        for (size_t i = 0; i < fr.size(); i++)
+            if (P.child_ptr[fr[i] + 1] > P.child_ptr[fr[i]] && (pick < 0 || sub[fr[i]] > sub[fr[pick]]))
+                pick = (int32_t)i;
+        if (pick < 0) break;
+        const int32_t v = fr[pick];
+        fr.erase(fr.begin() + pick);
+        for (int32_t q = P.child_ptr[v]; q < P.child_ptr[v + 1]; q++) fr.push_back(P.child_list[q]);
+    }
+    if (fr.size() < 2) return;   // nothing to run concurrently: one stream
+    const int nb = std::min<int>(B, (int)fr.size());
+    std::stable_sort(fr.begin(), fr.end(), [&](int32_t a, int32_t b) { return sub[a] > sub[b]; });
+    std::vector<double> load(nb, 0.0);
+    for (int32_t rt : fr) {
+        const int b = (int)(std::min_element(load.begin(), load.end()) - load.begin());
+        load[b] += sub[rt];
+        std::vector<int32_t> stack{rt};
+        while (!stack.empty()) {
+            const int32_t v = stack.back();
+            stack.pop_back();
+            P.branch[v] = b;
+            for (int32_t q = P.child_ptr[v]; q < P.child_ptr[v + 1]; q++) stack.push_back(P.child_list[q]);
+        }
+    }
+    P.nbranch = nb;
+}
+
 int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     P = Plan();
     const int32_t ns = (int32_t)S.sn_parent.size();
@@ -365,6 +416,8 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
             front_load[s] = k * m * m + m * k * (k + 1) + k * (k + 1) * (2 * k + 1) / 6;
         }
         map_subtrees(P, front_load);
+        if (P.nranks == 1) assign_branches(P, front_load, opt.nbranch);
+        else P.branch.assign(ns, -1);
     }
     // Inclusion masks.  Local program: the supernodes of this rank's subtrees.  Top
     // program (multi-GPU): EVERY rank holds a replica of every top front; the
@@ -425,8 +478,44 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     auto keep_all = [](int32_t, int32_t) { return true; };
     // the blocked factorization of the pivot-column leaves [a, b) (units of w) of the
     // fronts fl (sorted by k descending, stored at P.large_list[loff..])
+    // the dataflow panel of the leaves [a, b) (b - a <= kPanelMaxBlocks, w = 64):
+    // tasks = 64-row tile rows from j0 down, row-major over the active fronts
+    auto emit_panel = [&](const std::vector<int32_t> &fl, int32_t a, int32_t b, int32_t l) {
+        const int32_t j0 = a * w, j1 = b * w;
+        std::vector<int32_t> act;
+        int32_t maxc = 0;
+        for (int32_t s : fl)
+            if (P.sn_k[s] > j0) {
+                act.push_back(s);
+                maxc = std::max(maxc, (P.sn_f[s] - j0 + 63) / 64);
+            }
+        if (act.empty()) return;
+        Launch Lp{KC_PANEL, j0, (int64_t)P.panel_tasks.size() / 2, 0, 0.0, 0.0, l};
+        Lp.count2 = b - a;
+        for (int32_t c = 0; c < maxc; c++)
+            for (int32_t s : act)
+                if (j0 + 64 * c < P.sn_f[s]) {
+                    P.panel_tasks.push_back(s);
+                    P.panel_tasks.push_back(c);
+                }
+        for (int32_t s : act) {
+            const double f = P.sn_f[s];
+            const int32_t je = std::min(P.sn_k[s], j1);
+            for (int32_t j = j0; j < je; j++) {   // column j: scale (f - j) entries, update columns j+1 .. je-1
+                Lp.flops += f - j;
+                for (int32_t cc = j + 1; cc < je; cc++) Lp.flops += 2.0 * (f - cc);
+            }
+            Lp.bytes += 16.0 * (f - j0) * (je - j0);
+        }
+        Lp.count = (int64_t)P.panel_tasks.size() / 2 - Lp.off;
+        cur->push_back(Lp);
+    };
     std::function<void(const std::vector<int32_t> &, int64_t, int32_t, int32_t, int32_t)> rec =
         [&](const std::vector<int32_t> &fl, int64_t loff, int32_t a, int32_t b, int32_t l) {
+        if (w == 64 && b - a <= kPanelMaxBlocks) {
+            emit_panel(fl, a, b, l);
+            return;
+        }
         if (b - a == 1) {
             const int32_t j0 = a * w;
             int32_t na = 0;   // fronts (prefix of fl) with k > j0
@@ -474,9 +563,25 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         cur->push_back(Launch{KC_EXCHANGE, (int32_t)P.xfers.size(), 0, 0, 0.0, 0.0, l});
         P.xfers.push_back(std::move(x));
     };
-    for (int pass = 0; pass < 2; pass++) {
-    const std::vector<char> &inc = pass == 0 ? inc_local : inc_top;
-    if (pass == 1) cur = &P.program_top;
+    // passes over the levels: single GPU = one per branch (stream b), then the top
+    // fronts (main stream); multi-GPU = this rank's subtrees, then the top program
+    struct Pass { std::vector<char> inc; std::vector<Launch> *prog; int32_t stream; };
+    std::vector<Pass> passes;
+    if (R == 1 && P.nbranch > 1) {
+        for (int32_t b = 0; b <= P.nbranch; b++) {
+            const int32_t want = b < P.nbranch ? b : -1;
+            std::vector<char> m(ns);
+            for (int32_t s = 0; s < ns; s++) m[s] = P.branch[s] == want;
+            passes.push_back({std::move(m), &P.program, want});
+        }
+    } else {
+        passes.push_back({inc_local, &P.program, -1});
+        passes.push_back({inc_top, &P.program_top, -1});
+    }
+    for (const Pass &pass : passes) {
+    const std::vector<char> &inc = pass.inc;
+    cur = pass.prog;
+    const size_t pass_begin = cur->size();
     for (int32_t l = 0; l < nlev; l++) {
         std::vector<int32_t> fronts;
         for (int32_t q = P.level_ptr[l]; q < P.level_ptr[l + 1]; q++)
@@ -614,6 +719,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         if (Ls.count) cur->push_back(Ls);
         if (!ux.empty()) push_xfers(std::move(ux), l);
     }
+    for (size_t i = pass_begin; i < cur->size(); i++) (*cur)[i].stream = pass.stream;
     }   // pass
     for (const GemmProb &g : P.probs)   // the DMMA kernel stages 16-byte row pairs
         if ((g.a_off & 1) || (g.lda & 1)) return MF_ERR_STATE;

@@ -34,7 +34,7 @@ class Options(ctypes.Structure):
         ("amalgamate", ctypes.c_int32), ("nrelax", ctypes.c_int32 * 3), ("zrelax", ctypes.c_double * 3),
         ("small_front_max", ctypes.c_int32), ("panel_w", ctypes.c_int32), ("device", ctypes.c_int32),
         ("host_only", ctypes.c_int32), ("nranks", ctypes.c_int32), ("rank", ctypes.c_int32),
-        ("stream", ctypes.c_void_p), ("split_all", ctypes.c_int32),
+        ("stream", ctypes.c_void_p), ("split_all", ctypes.c_int32), ("nbranch", ctypes.c_int32),
     ]
 
 
@@ -57,7 +57,7 @@ class KernelStat(ctypes.Structure):
                 ("flops", ctypes.c_double), ("bytes", ctypes.c_double)]
 
 
-MF_KERNEL_CLASSES = 6
+MF_KERNEL_CLASSES = 7
 
 MF_XFER_SEND, MF_XFER_RECV, MF_XFER_BCAST, MF_XFER_ALLREDUCE_SUM, MF_XFER_ALLREDUCE_MIN_I32 = 1, 2, 3, 4, 5
 
@@ -147,7 +147,8 @@ class Solver:
 
     def __init__(self, amalgamate: bool = True, small_front_max: int | None = None, panel_w: int | None = None,
                  device: int = -1, stream: int | None = None, host_only: bool = False,
-                 nranks: int = 1, rank: int = 0, exchange=None, split_all: bool = False):
+                 nranks: int = 1, rank: int = 0, exchange=None, split_all: bool = False,
+                 nbranch: int | None = None):
         o = Options()
         lib.mf_default_options(ctypes.byref(o))
         o.amalgamate = int(amalgamate)
@@ -160,6 +161,8 @@ class Solver:
         o.nranks = nranks
         o.rank = rank
         o.split_all = int(split_all)
+        if nbranch is not None:
+            o.nbranch = nbranch
         o.stream = stream
         h = ctypes.c_void_p()
         r = lib.mf_create(ctypes.byref(h), ctypes.byref(o))

@@ -23,7 +23,7 @@ S.analyze(A.n, A.colptr, A.rowind, p)
 prog = S.program()
 assert len(seq) == len(prog) + 1, (len(seq), len(prog))
 seq = seq[1:]
-names = {0: "small", 1: "assemble", 2: "potrf", 3: "trsm", 4: "update", 5: "leaf"}
+names = {0: "small", 1: "assemble", 2: "potrf", 3: "trsm", 4: "update", 5: "leaf", 6: "panel"}
 by = collections.defaultdict(lambda: [0, 0.0, 0.0])
 upd = []
 for (kn, us, grid), L in zip(seq, prog):

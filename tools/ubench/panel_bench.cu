@@ -1,0 +1,89 @@
+// Latency / timeline microbenchmark of the dataflow panel kernel (k_panel) on one
+// dense front: f rows, k pivot columns, panel of nbk blocks at j0 = 0.
+// Builds kernels.cu with -DMF_PANEL_TRACE and prints per-task globaltimer marks.
+//   nvcc -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -DMF_PANEL_TRACE \
+//        -I include -I paper_conf_ipps_georgesgsc11_b200/csrc tools/ubench/panel_bench.cu -o tools/ubench/panel_bench
+#include "../../paper_conf_ipps_georgesgsc11_b200/csrc/kernels.cu"
+
+#include <cstdlib>
+#include <vector>
+
+using namespace mf;
+
+int main(int argc, char **argv) {
+    const int f = argc > 1 ? atoi(argv[1]) : 8192, k = argc > 2 ? atoi(argv[2]) : 8192;
+    const int nbk = argc > 3 ? atoi(argv[3]) : 4;
+    const int ld = f + (f & 1);
+    std::vector<double> h((size_t)ld * k, 0.0);
+    srand(1);
+    for (int j = 0; j < k; j++)
+        for (int i = j; i < f; i++) h[i + (size_t)j * ld] = (i == j) ? 4.0 * f : (rand() / (double)RAND_MAX - 0.5);
+    double *L, *L0;
+    cudaMalloc(&L, (h.size() + 2) * 8);
+    cudaMalloc(&L0, (h.size() + 2) * 8);
+    cudaMemcpy(L0, h.data(), h.size() * 8, cudaMemcpyHostToDevice);
+    int32_t hs[4] = {0, k, f, ld};
+    int64_t hoff = 0;
+    int32_t *dfirst, *dk, *df, *dld;
+    int64_t *doff;
+    cudaMalloc(&dfirst, 4); cudaMemcpy(dfirst, &hs[0], 4, cudaMemcpyHostToDevice);
+    cudaMalloc(&dk, 4); cudaMemcpy(dk, &hs[1], 4, cudaMemcpyHostToDevice);
+    cudaMalloc(&df, 4); cudaMemcpy(df, &hs[2], 4, cudaMemcpyHostToDevice);
+    cudaMalloc(&dld, 4); cudaMemcpy(dld, &hs[3], 4, cudaMemcpyHostToDevice);
+    cudaMalloc(&doff, 8); cudaMemcpy(doff, &hoff, 8, cudaMemcpyHostToDevice);
+    int *failed; cudaMalloc(&failed, 16);
+    int hf[4] = {INT_MAX, 1, 0, 0};
+    cudaMemcpy(failed, hf, 16, cudaMemcpyHostToDevice);
+    unsigned *pflag; cudaMalloc(&pflag, kPanelFlags * 4);
+    DevPlan d{};
+    d.L = L; d.sn_first = dfirst; d.sn_k = dk; d.sn_f = df; d.sn_ld = dld; d.L_off = doff;
+    d.failed = failed; d.epoch = reinterpret_cast<const unsigned *>(failed + 1); d.panel_flag = pflag;
+    const int nch = (f + 63) / 64;
+    std::vector<int32_t> tasks;
+    for (int c = 0; c < nch; c++) { tasks.push_back(0); tasks.push_back(c); }
+    int32_t *dt; cudaMalloc(&dt, tasks.size() * 4);
+    cudaMemcpy(dt, tasks.data(), tasks.size() * 4, cudaMemcpyHostToDevice);
+    cudaFuncSetAttribute(k_panel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kPanelSmem);
+    cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+    float best = 1e9;
+    for (int rep = 0; rep < 10; rep++) {
+        cudaMemcpy(L, L0, h.size() * 8, cudaMemcpyDeviceToDevice);
+        cudaMemset(pflag, 0, kPanelFlags * 4);
+        cudaEventRecord(e0);
+        launch_panel(d, dt, nch, 0, nbk, 0);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        float ms; cudaEventElapsedTime(&ms, e0, e1);
+        if (ms < best) best = ms;
+    }
+    cudaError_t err = cudaGetLastError();
+    printf("f=%d k=%d nbk=%d tasks=%d: best %.2f us (%s)\n", f, k, nbk, nch, best * 1e3, cudaGetErrorString(err));
+    static unsigned long long tr[4096][32];
+    cudaMemcpyFromSymbol(tr, g_panel_trace, sizeof(tr));
+    unsigned long long t0 = ~0ull;
+    for (int c = 0; c < nch; c++) if (tr[c][0] && tr[c][0] < t0) t0 = tr[c][0];
+    auto show = [&](int c) {
+        printf("task %4d:", c);
+        printf(" [potrf clk a %llu b %llu c %llu]", tr[c][25], tr[c][26], tr[c][27]);
+        for (int e = 0; e < 31; e++)
+            if (e < 25 || e > 27) if (tr[c][e] >= t0 && tr[c][e] - t0 < 10000000ull) printf(" %d:%.1f", e, (tr[c][e] - t0) / 1e3);
+        printf("\n");
+    };
+    for (int c = 0; c < std::min(nch, nbk + 1); c++) show(c);
+    show(nch / 2);
+    show(nch - 1);
+    // check: the leading W x W block of L L^T reproduces A (W = 64 nbk), and the rows
+    // below: (L L^T)(i, j) = A(i, j) for j < W
+    std::vector<double> Lh(h.size());
+    cudaMemcpy(Lh.data(), L, h.size() * 8, cudaMemcpyDeviceToHost);
+    const int W = std::min(64 * nbk, k);
+    double maxerr = 0;
+    for (int j = 0; j < W; j++)
+        for (int i = j; i < f; i += (i < W ? 1 : 37)) {
+            double sum = 0;
+            for (int p = 0; p <= j; p++) sum += Lh[i + (size_t)p * ld] * Lh[j + (size_t)p * ld];
+            maxerr = std::max(maxerr, fabs(sum - h[i + (size_t)j * ld]) / (4.0 * f));
+        }
+    printf("max |L L^T - A| / |A|_max over the panel columns: %.3e\n", maxerr);
+    return 0;
+}
