@@ -48,6 +48,7 @@ def parse():
                     help="true GFLOP of the oracle sample (one whole subtree)")
     ap.add_argument("--small-front-max", type=int, default=None)
     ap.add_argument("--panel-w", type=int, default=None)
+    ap.add_argument("--nbranch", type=int, default=None, help="concurrent subtree branches (single GPU)")
     return ap.parse_args()
 
 
@@ -227,7 +228,7 @@ def main():
         from paper_conf_ipps_georgesgsc11_b200.exchange import TorchDistExchange
         exchange = TorchDistExchange()
     S = mf.Solver(device=local, stream=stream.cuda_stream, small_front_max=args.small_front_max,
-                  panel_w=args.panel_w, nranks=world, rank=rank, exchange=exchange)
+                  panel_w=args.panel_w, nranks=world, rank=rank, exchange=exchange, nbranch=args.nbranch)
     S.analyze(A.n, A.colptr, A.rowind, perm)
     info = S.info()
     flops = float(info["flops_true"])
@@ -343,7 +344,7 @@ def main():
                    "flops_true": flops, "flops_exec": float(info["flops_exec"]), "nsuper": info["nsuper"],
                    "max_front": info["max_front"],
                    "parallelism": (f"subtree-to-GPU x{world}, top supernodes on rank 0 (NCCL send/recv)"
-                                   if world > 1 else "1 GPU"),
+                                   if world > 1 else f"1 GPU, {info['nbranch']} concurrent subtree branches"),
                    "l2": "no flush: working set (L = %.1f GB) >> 126 MB L2" % (info["panel_words"] * 8 / 1e9)},
         "clocks": clocks,
         "mapping": mapping,

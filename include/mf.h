@@ -98,6 +98,7 @@ typedef struct {
     double t_analyze;         /* seconds (host wall) of the last mf_analyze */
     double t_factor;          /* seconds (device events) of the last mf_factor */
     double t_solve;           /* seconds (device events) of the last mf_solve */
+    int32_t nbranch;          /* concurrent subtree branches the factorization uses (single GPU)   */
 } mf_info;
 
 /* Per-kernel-class statistics of profiled factorizations (mf_set_profiling):
@@ -214,6 +215,32 @@ int mf_set_profiling(mf_ctx *ctx, int enable);
 
 /* out[MF_KERNEL_CLASSES]: accumulated stats since the last mf_set_profiling; *count = classes written. */
 int mf_get_kernel_stats(const mf_ctx *ctx, mf_kernel_stat *out, int32_t *count);
+
+/* Per-launch CUDA-event times (ms) of the last PROFILED factorization, in program
+ * order (mf_get_program; the local program only).  out may be NULL to query *count. */
+int mf_get_launch_times(const mf_ctx *ctx, double *out_ms, int64_t max, int64_t *count);
+
+/* Learned kernel-variant selector (Sec. VI, Eqs. 3-5).
+ * The paper picks a CPU/GPU policy per factor-update call with a cost-sensitive
+ * multinomial logistic classifier y(x) = argmax_j x . theta_j over front features
+ * x(m, k).  Here the classes are GPU kernel variants of a front:
+ *   0: one warp per front, f <= 16        1: one warp per front, f <= 32
+ *   2: one CTA per front in shared memory, f <= 64     3: ... f <= 96
+ *   4: ... f <= 128      5: ... f <= 160      6: tiled large-front path (any f)
+ * and x = [1, m/64, k/64, m/k, (m/64)^2, (m/64)(k/64), (k/64)^2, (k/64)^3, (m/64)(k/64)^2]
+ * (the paper's [m, k, m/k, m^2, mk, k^2, k^3, mk^2] after a constant, m and k in
+ * units of 64).  theta: MF_VARIANT_FEATURES x MF_VARIANTS row-major (theta[q * MF_VARIANTS
+ * + j] = weight of feature q for class j); NULL = the default front-order thresholds.
+ * force >= 0 forces class `force` wherever it is feasible (used to measure the
+ * per-class times the model is fitted to).  Call before mf_analyze; the choice is
+ * made once per pattern.  Returns MF_ERR_STATE after mf_analyze, MF_ERR_ARG for a
+ * bad class or size. */
+#define MF_VARIANTS 7
+#define MF_VARIANT_FEATURES 9
+int mf_set_variant_model(mf_ctx *ctx, const double *theta, int32_t nfeatures, int32_t nclasses, int32_t force);
+
+/* Kernel-variant class of every supernode of the analyzed pattern: out[nsuper]. */
+int mf_get_variants(const mf_ctx *ctx, int32_t *out);
 
 void mf_destroy(mf_ctx *ctx);
 

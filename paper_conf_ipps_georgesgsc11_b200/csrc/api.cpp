@@ -144,6 +144,7 @@ void fill_info(mf_ctx *c, int64_t n, int with_device) {
     I.nsuper = P.nsuper;
     I.nlevels = P.nlevels;
     I.max_front = P.max_front;
+    I.nbranch = P.nbranch;
     I.rows_total = P.rows_total;
     I.failed_col = -1;
     int64_t ws = 0;
@@ -809,6 +810,38 @@ int mf_get_program(const mf_ctx *c, mf_launch_info *out, int64_t max, int64_t *c
     if (out)
         for (int64_t i = 0; i < std::min<int64_t>(max, (int64_t)prog.size()); i++)
             out[i] = mf_launch_info{prog[i].kind, prog[i].level, prog[i].count, prog[i].flops, prog[i].bytes};
+    return MF_OK;
+}
+
+int mf_get_launch_times(const mf_ctx *c, double *out, int64_t max, int64_t *count) {
+    if (!c || !count) return MF_ERR_ARG;
+    const int64_t n = (int64_t)c->P.program.size();
+    *count = n;
+    if (!out) return MF_OK;
+    if (c->host_only || c->prof_factors == 0 || (int64_t)c->prof_events.size() < 2 * n) return MF_ERR_STATE;
+    for (int64_t i = 0; i < std::min(n, max); i++) {
+        float t = 0.f;
+        cudaEventElapsedTime(&t, c->prof_events[2 * i], c->prof_events[2 * i + 1]);
+        out[i] = t;
+    }
+    return MF_OK;
+}
+
+int mf_set_variant_model(mf_ctx *c, const double *theta, int32_t nfeatures, int32_t nclasses, int32_t force) {
+    if (!c) return MF_ERR_ARG;
+    if (c->state != 0) return MF_ERR_STATE;
+    if (force < -1 || force >= kVariants) return MF_ERR_ARG;
+    if (theta && (nfeatures != kVariantFeatures || nclasses != kVariants)) return MF_ERR_ARG;
+    c->opt.variant_theta.clear();
+    if (theta) c->opt.variant_theta.assign(theta, theta + kVariantFeatures * kVariants);
+    c->opt.force_variant = force;
+    return MF_OK;
+}
+
+int mf_get_variants(const mf_ctx *c, int32_t *out) {
+    if (!c || !out) return MF_ERR_ARG;
+    if (c->state < 1) return MF_ERR_STATE;
+    std::copy(c->P.variant.begin(), c->P.variant.end(), out);
     return MF_OK;
 }
 

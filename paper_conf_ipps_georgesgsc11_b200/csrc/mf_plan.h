@@ -23,7 +23,37 @@ struct Options {
     int rank = 0;
     int split_all = 0;   // multi-GPU mapping ignores the exchange-cost model
     int nbranch = 4;     // single GPU: concurrent subtree branches (graph branches on their own streams)
+    // learned kernel-variant selector (Sec. VI, Eqs. 3-5):
+    // theta is kVariantFeatures x kVariants (column j = class j); empty = the fixed
+    // front-order thresholds.  force_variant >= 0 forces that class wherever feasible.
+    std::vector<double> variant_theta;
+    int force_variant = -1;
 };
+
+// Kernel variants a front can be factored with (the GPU-only policy classes that
+// replace the paper's CPU/GPU policies P1-P4, Table VI): one warp per
+// front (f <= 16, f <= 32), one CTA per front with the front in shared memory
+// (f <= 64, 96, 128, 160), or the tiled large-front path.  kVariantFmax = the
+// largest front order a class accepts (0 = any: tiled).
+constexpr int kVariants = 7;
+constexpr int kVariantTiled = 6;
+constexpr int kVariantFmax[kVariants] = {16, 32, 64, 96, 128, 160, 0};
+// Features of a front (m off-diagonal rows, k pivot columns): the paper's
+// [m, k, m/k, m^2, mk, k^2, k^3, mk^2] after a constant 1, with
+// m and k measured in units of 64 (reading R3 in DESIGN.md).
+constexpr int kVariantFeatures = 9;
+inline void variant_features(double m, double k, double *x) {
+    const double a = m / 64.0, b = k / 64.0;
+    x[0] = 1.0;
+    x[1] = a;
+    x[2] = b;
+    x[3] = m / k;
+    x[4] = a * a;
+    x[5] = a * b;
+    x[6] = b * b;
+    x[7] = b * b * b;
+    x[8] = a * b * b;
+}
 
 // ---------------------------------------------------------------- symbolic
 struct Symbolic {
@@ -139,6 +169,7 @@ struct Plan {
     // schedule
     std::vector<int32_t> level_ptr, level_list;      // all supernodes by level (solve)
     std::vector<int32_t> small_list, small_class_fmax;
+    std::vector<int32_t> variant;                    // per supernode: kernel-variant class (kVariantFmax)
     std::vector<int32_t> large_list;
     std::vector<int32_t> asm_tasks;                  // pairs (front, c0)
     std::vector<int32_t> trsm_tasks;                 // pairs (front, row0)

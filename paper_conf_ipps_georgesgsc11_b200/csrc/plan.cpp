@@ -389,6 +389,53 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     // (<= 16 and <= 32: one warp per front; <= 64 and <= small_max: one CTA per front)
     P.small_class_fmax = {std::min(16, P.small_max), std::min(32, P.small_max), std::min(64, P.small_max),
                           P.small_max};
+    // kernel variant per front: the learned selector y(x) = argmax_j x . theta_j over
+    // the feasible classes (Eq. 5), a forced class, or the default
+    // front-order thresholds (the analogue of the paper's baseline P_BH, L401).
+    // front_fmax = the order bound of the class's shared-memory / warp kernel, 0 = tiled.
+    std::vector<int32_t> front_fmax(ns, 0);
+    P.variant.assign(ns, kVariantTiled);
+    for (int32_t s = 0; s < ns; s++) {
+        const int32_t f = P.sn_f[s], k = P.sn_k[s];
+        auto feasible = [&](int j) { return j == kVariantTiled || f <= kVariantFmax[j]; };
+        int v = -1;
+        if (opt.force_variant >= 0 && opt.force_variant < kVariants && feasible(opt.force_variant)) {
+            v = opt.force_variant;
+        } else if ((int)opt.variant_theta.size() == kVariantFeatures * kVariants) {
+            double x[kVariantFeatures], best = -1e300;
+            variant_features(f - k, k, x);
+            for (int j = 0; j < kVariants; j++) {
+                if (!feasible(j)) continue;
+                double sc = 0;
+                for (int q = 0; q < kVariantFeatures; q++) sc += x[q] * opt.variant_theta[q * kVariants + j];
+                if (sc > best) {
+                    best = sc;
+                    v = j;
+                }
+            }
+        }
+        if (v >= 0) {
+            P.variant[s] = v;
+            front_fmax[s] = kVariantFmax[v];
+        } else if (f <= P.small_max) {
+            for (int cls = 0; cls < kSmallClasses; cls++)
+                if (f <= P.small_class_fmax[cls]) {
+                    front_fmax[s] = P.small_class_fmax[cls];
+                    break;
+                }
+            P.variant[s] = kVariantTiled;
+            for (int j = 0; j < kVariantTiled; j++)
+                if (front_fmax[s] <= kVariantFmax[j]) {
+                    P.variant[s] = j;
+                    break;
+                }
+        }
+    }
+    std::vector<int32_t> fmax_classes;
+    for (int32_t s = 0; s < ns; s++)
+        if (front_fmax[s] > 0) fmax_classes.push_back(front_fmax[s]);
+    std::sort(fmax_classes.begin(), fmax_classes.end());
+    fmax_classes.erase(std::unique(fmax_classes.begin(), fmax_classes.end()), fmax_classes.end());
     const int w = P.w;
     // algorithmic bytes of assembling front s: its A entries (value + index), the
     // children's U^c lower triangles and relative maps (read once)
@@ -586,11 +633,10 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         std::vector<int32_t> fronts;
         for (int32_t q = P.level_ptr[l]; q < P.level_ptr[l + 1]; q++)
             if (inc[P.level_list[q]]) fronts.push_back(P.level_list[q]);
-        for (int cls = 0; cls < kSmallClasses; cls++) {
-            const int lo = cls == 0 ? 0 : P.small_class_fmax[cls - 1];
-            Launch L{KC_SMALL, P.small_class_fmax[cls], (int64_t)P.small_list.size(), 0, 0.0, 0.0, l};
+        for (int32_t fm : fmax_classes) {
+            Launch L{KC_SMALL, fm, (int64_t)P.small_list.size(), 0, 0.0, 0.0, l};
             for (int32_t s : fronts)
-                if (P.sn_f[s] > lo && P.sn_f[s] <= P.small_class_fmax[cls]) {
+                if (front_fmax[s] == fm) {
                     P.small_list.push_back(s);
                     const double k = P.sn_k[s], m = P.sn_f[s] - P.sn_k[s];
                     L.flops += k * m * m + m * k * (k + 1) + k * (k + 1) * (2 * k + 1) / 6;
@@ -601,7 +647,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         }
         std::vector<int32_t> large;
         for (int32_t s : fronts)
-            if (P.sn_f[s] > P.small_max) large.push_back(s);
+            if (front_fmax[s] == 0) large.push_back(s);
         if (large.empty()) continue;
         std::stable_sort(large.begin(), large.end(), [&](int32_t a, int32_t b) { return P.sn_k[a] > P.sn_k[b]; });
         // assembly (every rank assembles its replica of a top front)

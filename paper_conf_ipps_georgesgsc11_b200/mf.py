@@ -26,7 +26,10 @@ EXPORTED_SYMBOLS = (
     "mf_default_options", "mf_create", "mf_analyze", "mf_factor", "mf_solve", "mf_get_info",
     "mf_get_perm", "mf_get_etree", "mf_get_supernodes", "mf_export_panel", "mf_export_diag", "mf_export_L",
     "mf_get_program", "mf_set_profiling", "mf_get_kernel_stats", "mf_set_exchange", "mf_get_mapping", "mf_destroy", "mf_strerror",
+    "mf_get_launch_times", "mf_set_variant_model", "mf_get_variants",
 )
+MF_VARIANTS = 7
+MF_VARIANT_FEATURES = 9
 
 
 class Options(ctypes.Structure):
@@ -46,6 +49,7 @@ class Info(ctypes.Structure):
         ("nlevels", ctypes.c_int32), ("max_front", ctypes.c_int32), ("rows_total", ctypes.c_int64),
         ("failed_col", ctypes.c_int64), ("workspace_bytes", ctypes.c_int64), ("launches_factor", ctypes.c_int64),
         ("t_analyze", ctypes.c_double), ("t_factor", ctypes.c_double), ("t_solve", ctypes.c_double),
+        ("nbranch", ctypes.c_int32),
     ]
 
     def as_dict(self) -> dict:
@@ -104,6 +108,9 @@ def _load():
         "mf_get_kernel_stats": ([vp, ctypes.POINTER(KernelStat), ctypes.POINTER(i32)], ctypes.c_int),
         "mf_destroy": ([vp], None),
         "mf_strerror": ([ctypes.c_int], ctypes.c_char_p),
+        "mf_get_launch_times": ([vp, vp, i64, ctypes.POINTER(i64)], ctypes.c_int),
+        "mf_set_variant_model": ([vp, vp, i32, i32, i32], ctypes.c_int),
+        "mf_get_variants": ([vp, vp], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         fn = getattr(L, name)
@@ -284,6 +291,32 @@ class Solver:
         arr = (LaunchInfo * max(cnt.value, 1))()
         self._check(lib.mf_get_program(self._h, arr, cnt.value, ctypes.byref(cnt)), "mf_get_program")
         return [dict(kind=a.kind, level=a.level, count=a.count, flops=a.flops, bytes=a.bytes) for a in arr[:cnt.value]]
+
+    def launch_times(self) -> np.ndarray:
+        """CUDA-event ms of every launch of the last profiled factorization (program order)."""
+        cnt = ctypes.c_int64()
+        self._check(lib.mf_get_launch_times(self._h, None, 0, ctypes.byref(cnt)), "mf_get_launch_times")
+        out = np.zeros(max(cnt.value, 1), dtype=np.float64)
+        self._check(lib.mf_get_launch_times(self._h, out.ctypes.data, cnt.value, ctypes.byref(cnt)),
+                    "mf_get_launch_times")
+        return out[:cnt.value]
+
+    def set_variant_model(self, theta=None, force: int = -1):
+        """Kernel-variant selector (before analyze): theta (MF_VARIANT_FEATURES x MF_VARIANTS)
+        or None for the default thresholds; force >= 0 forces a class where feasible."""
+        if theta is None:
+            self._check(lib.mf_set_variant_model(self._h, None, 0, 0, int(force)), "mf_set_variant_model")
+            return
+        th = np.ascontiguousarray(theta, dtype=np.float64)
+        if th.shape != (MF_VARIANT_FEATURES, MF_VARIANTS):
+            raise ValueError(f"theta must be {MF_VARIANT_FEATURES} x {MF_VARIANTS}")
+        self._check(lib.mf_set_variant_model(self._h, th.ctypes.data, MF_VARIANT_FEATURES, MF_VARIANTS, int(force)),
+                    "mf_set_variant_model")
+
+    def variants(self) -> np.ndarray:
+        out = np.empty(max(self._info["nsuper"], 1), dtype=np.int32)
+        self._check(lib.mf_get_variants(self._h, out.ctypes.data), "mf_get_variants")
+        return out[:self._info["nsuper"]]
 
     def set_profiling(self, enable: bool = True):
         self._check(lib.mf_set_profiling(self._h, int(enable)), "mf_set_profiling")
