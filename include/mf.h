@@ -77,6 +77,12 @@ typedef struct {
     int32_t nbranch;          /* single GPU: elimination subtrees are split into this many branches
                                  that run concurrently (CUDA-graph branches on their own streams)
                                  below the top fronts; 1 = one stream (default 4)                  */
+    int32_t fuse_ea;          /* 1 (default) = the extend-add of the children's U^c into the U^s part
+                                 of a large front is fused into the prologue of its syrk (the Schur
+                                 update starts from the gathered sum 0 + U^c1 + U^c2 + ... instead of
+                                 a U^s assembled in HBM); 0 = the
+                                 assembly kernel builds the whole front.  Both give bit-identical
+                                 fronts (same summation order, reading C6).                         */
 } mf_options;
 
 typedef struct {

@@ -188,6 +188,7 @@ int mf_default_options(mf_options *o) {
     o->stream = nullptr;
     o->split_all = 0;
     o->nbranch = d.nbranch;
+    o->fuse_ea = d.fuse_ea;
     return MF_OK;
 }
 
@@ -219,6 +220,7 @@ int mf_create(mf_ctx **out, const mf_options *o) {
         return MF_ERR_ARG;
     }
     c->opt.nbranch = o->nbranch;
+    c->opt.fuse_ea = o->fuse_ea != 0;
     c->opt.rank = o->rank;
     c->host_only = o->host_only != 0;
     c->info.failed_col = -1;
@@ -333,6 +335,8 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     int64_t *df_blk_off = nullptr, *df_part_off = nullptr;
     UP(&df_blk_off, P.df_blk_off);
     UP(&df_part_off, P.df_part_off);
+    int32_t *ea_qs = nullptr;
+    UP(&ea_qs, P.ea_qs);
     UP(&c->d_top_list, P.top_list);
     UP(&c->d_own_list, P.own_list);
 #undef UP
@@ -354,6 +358,8 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     d.perm = perm_d;
     d.df_blk_off = df_blk_off;
     d.df_part_off = df_part_off;
+    d.ea_qs = ea_qs;
+    d.fuse_ea = P.fuse_ea;
     void *p;
     if ((r = dev_alloc(c, &p, P.L_words * sizeof(double))) != MF_OK) return r;
     d.L = (double *)p;

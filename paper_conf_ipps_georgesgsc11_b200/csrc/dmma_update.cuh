@@ -45,6 +45,17 @@ __device__ __forceinline__ void dmma(double &c0, double &c1, double a, double b)
                  : "d"(a), "d"(b));
 }
 
+// Fused extend-add (GemmProb flags bit 2): the syrk on U^s
+// starts from the children's contributions gathered through their relative maps
+// (F^s = A-part (+) U^c1 (+) U^c2 ...; the U^s part of F^s has no A
+// entries), summed per element in ascending child order from 0 -- the order of
+// the assembly kernel (reading C6), so U^s is bit-identical to the unfused path.
+struct UpdGather {
+    const int32_t *child_ptr, *child_list, *sn_k, *sn_f;
+    const int64_t *U_off, *relmap_ptr;
+    const int32_t *relmap, *qs;
+};
+
 template <int BM_, int BN_, int BK_, int STAGES_, int WARPS_M_, int WARPS_N_, int MINB_>
 struct UpdCfg {
     static constexpr int BM = BM_, BN = BN_, BK = BK_, STAGES = STAGES_;
@@ -61,7 +72,7 @@ struct UpdCfg {
     static constexpr int PSA16 = NT / CPA, PSB16 = NT / CPB;      // k stride of a thread
     static_assert(BK % PSA16 == 0 && BK % PSB16 == 0, "staging map");
     static constexpr int STAGE_WORDS = BK * (SA + SB);
-    static constexpr size_t SMEM = (size_t)STAGES * STAGE_WORDS * sizeof(double);
+    static constexpr size_t SMEM = (size_t)STAGES * STAGE_WORDS * sizeof(double) + (BM + BN) * sizeof(int);
     static_assert(SA % 16 == 4 && SB % 16 == 4, "bank-conflict-free fragment loads");
     static_assert(TM % 8 == 0 && TN % 8 == 0 && BK % 4 == 0, "tile shape");
 };
@@ -69,7 +80,7 @@ struct UpdCfg {
 template <class Cfg>
 __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
     k_update_t(double *__restrict__ Larena, double *__restrict__ Uarena, const GemmProb *__restrict__ probs,
-               const TileTask *__restrict__ tiles) {
+               const TileTask *__restrict__ tiles, const UpdGather gv) {
     constexpr int BM = Cfg::BM, BN = Cfg::BN, BK = Cfg::BK, STAGES = Cfg::STAGES, NT = Cfg::NT;
     constexpr int SA = Cfg::SA, SB = Cfg::SB, STAGE_WORDS = Cfg::STAGE_WORDS;
     constexpr int MB = Cfg::MB, NB = Cfg::NB, TM = Cfg::TM, TN = Cfg::TN;
@@ -116,17 +127,60 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
     double *__restrict__ C = ((g.flags & 1) ? Uarena : Larena) + g.c_off;
     const int ldc = g.ldc;
     double acc[MB][NB][2];
+    if (!(g.flags & 4)) {
 #pragma unroll
-    for (int mb = 0; mb < MB; mb++) {
-        const int i = i0 + wm * TM + mb * 8 + gq;
+        for (int mb = 0; mb < MB; mb++) {
+            const int i = i0 + wm * TM + mb * 8 + gq;
 #pragma unroll
-        for (int nb = 0; nb < NB; nb++)
+            for (int nb = 0; nb < NB; nb++)
 #pragma unroll
-            for (int e = 0; e < 2; e++) {
-                const int j = j0 + wn * TN + nb * 8 + 2 * tq + e;
-                acc[mb][nb][e] =
-                    (i < g.M && j < g.N && i >= sh && j >= sh) ? C[(i - sh) + (int64_t)(j - sh) * ldc] : 0.0;
+                for (int e = 0; e < 2; e++) {
+                    const int j = j0 + wn * TN + nb * 8 + 2 * tq + e;
+                    acc[mb][nb][e] =
+                        (i < g.M && j < g.N && i >= sh && j >= sh) ? C[(i - sh) + (int64_t)(j - sh) * ldc] : 0.0;
+                }
+        }
+    } else {
+        // C = 0 (+) U^c1 (+) U^c2 ... over this tile: per child, the rows landing in
+        // tile row ti / tile column tj are the contiguous ranges qs[ti..ti+1) /
+        // qs[tj..tj+1) of its U^c (precomputed); their positions in the tile go
+        // to shared maps, then every accumulator adds its element if both its row
+        // and its column come from the child (lower part only: rel is increasing).
+#pragma unroll
+        for (int mb = 0; mb < MB; mb++)
+#pragma unroll
+            for (int nb = 0; nb < NB; nb++) acc[mb][nb][0] = acc[mb][nb][1] = 0.0;
+        int *rq = reinterpret_cast<int *>(sm + STAGES * STAGE_WORDS), *cq = rq + BM;
+        const int q0 = gv.child_ptr[g.s], q1 = gv.child_ptr[g.s + 1], kp = gv.sn_k[g.s];
+        const int ntr1 = (g.M + BM - 1) / BM + 1;
+        for (int jc = 0; jc < q1 - q0; jc++) {
+            const int32_t *__restrict__ qs = gv.qs + g.qs_off + (int64_t)jc * ntr1;
+            const int ra = qs[ti], rb = qs[ti + 1], ca = qs[tj], cb = qs[tj + 1];
+            if (ra == rb || ca == cb) continue;   // uniform over the CTA
+            const int ch = gv.child_list[q0 + jc];
+            const int mc = gv.sn_f[ch] - gv.sn_k[ch];
+            const int32_t *__restrict__ rel = gv.relmap + gv.relmap_ptr[ch];
+            const double *__restrict__ Uc = Uarena + gv.U_off[ch];
+            __syncthreads();   // the previous child's maps are consumed
+            for (int x = tid; x < BM + BN; x += NT) rq[x] = -1;
+            __syncthreads();
+            // front row r >= kp sits at shifted U row r - kp + sh
+            for (int q = ra + tid; q < rb; q += NT) rq[__ldg(rel + q) - kp + sh - i0] = q;
+            for (int q = ca + tid; q < cb; q += NT) cq[__ldg(rel + q) - kp + sh - j0] = q;
+            __syncthreads();
+#pragma unroll
+            for (int mb = 0; mb < MB; mb++) {
+                const int qi = rq[wm * TM + mb * 8 + gq];
+                if (qi < 0) continue;
+#pragma unroll
+                for (int nb = 0; nb < NB; nb++)
+#pragma unroll
+                    for (int e = 0; e < 2; e++) {
+                        const int qj = cq[wn * TN + nb * 8 + 2 * tq + e];
+                        if (qj >= 0 && qi >= qj) acc[mb][nb][e] += __ldg(Uc + qi + (int64_t)qj * mc);
+                    }
             }
+        }
     }
     for (int kt = 0; kt < KT; kt++) {
         cp_async_wait<STAGES - 2>();
@@ -168,7 +222,7 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
 
 template <class Cfg>
 inline void launch_update_t(double *L, double *U, const GemmProb *probs, const TileTask *tiles, int64_t ntiles,
-                            cudaStream_t st) {
+                            cudaStream_t st, const UpdGather gv = UpdGather{}) {
     if (ntiles <= 0) return;
     if (Cfg::SMEM > 48 * 1024) {   // idempotent; libmf also sets it up front (kernels_init) before graph capture
         static bool attr = false;
@@ -177,7 +231,7 @@ inline void launch_update_t(double *L, double *U, const GemmProb *probs, const T
             attr = true;
         }
     }
-    k_update_t<Cfg><<<(unsigned)ntiles, Cfg::NT, Cfg::SMEM, st>>>(L, U, probs, tiles);
+    k_update_t<Cfg><<<(unsigned)ntiles, Cfg::NT, Cfg::SMEM, st>>>(L, U, probs, tiles, gv);
 }
 
 }  // namespace mf

@@ -308,7 +308,7 @@ __global__ void __launch_bounds__(kAsmThreads) k_assemble(DevPlan d, const int32
     __shared__ int s_cp[NW][kAsmMaxCh];           // per warp and child: next child row to add
     const int s = tasks[2 * blockIdx.x], c0 = tasks[2 * blockIdx.x + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], m = f - k, ld = d.sn_ld[s], first = d.sn_first[s];
-    const int c1 = min(c0 + kAsmCols, f);
+    const int c1 = min(c0 + kAsmCols, d.fuse_ea ? k : f);   // fused extend-add: U^s is gathered by the syrk
     double *__restrict__ P = d.L + d.L_off[s];
     double *__restrict__ Us = d.U + d.U_off[s];
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -1221,7 +1221,8 @@ using UpdProd = UpdCfg<kTileM, kTileN, 16, 3, 2, 2, 4>;   // 33.5 TF/s on M=N=81
 
 void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, cudaStream_t st) {
     if (ntiles <= 0) return;   // attributes were set by kernels_init()
-    k_update_t<UpdProd><<<(unsigned)ntiles, UpdProd::NT, UpdProd::SMEM, st>>>(d.L, d.U, probs, tiles);
+    const UpdGather gv{d.child_ptr, d.child_list, d.sn_k, d.sn_f, d.U_off, d.relmap_ptr, d.relmap, d.ea_qs};
+    k_update_t<UpdProd><<<(unsigned)ntiles, UpdProd::NT, UpdProd::SMEM, st>>>(d.L, d.U, probs, tiles, gv);
 }
 
 void launch_init_failed(int *failed, cudaStream_t st) { k_init_failed<<<1, 1, 0, st>>>(failed, reinterpret_cast<unsigned *>(failed + 1)); }

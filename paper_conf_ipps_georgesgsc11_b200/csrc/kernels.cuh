@@ -30,6 +30,8 @@ struct DevPlan {
     unsigned *df_flags;      // dataflow solve flags (forward per block, backward per chunk)
     double *df_parts;        // dataflow backward partial sums per (chunk, block)
     const int64_t *df_blk_off, *df_part_off;
+    const int32_t *ea_qs;    // fused extend-add: tile-row start tables of the syrk problems
+    int fuse_ea;             // 1: large-front assembly covers the panel columns only
 };
 
 // launchers (all asynchronous on `st`)

@@ -22,6 +22,7 @@ struct Options {
     int nranks = 1;   // GPUs sharing one factorization (one process per GPU)
     int rank = 0;
     int split_all = 0;   // multi-GPU mapping ignores the exchange-cost model
+    int fuse_ea = 1;     // extend-add into the U^s part fused into the syrk prologue (NEXT-1)
     int nbranch = 4;     // single GPU: concurrent subtree branches (graph branches on their own streams)
     // learned kernel-variant selector (Sec. VI, Eqs. 3-5):
     // theta is kVariantFeatures x kVariants (column j = class j); empty = the fixed
@@ -88,14 +89,22 @@ int analyze_symbolic(int64_t n, const int64_t *colptr, const int32_t *rowind, co
 // arena (1).  flags bit 1: the problem is shifted one row / column up-left so that
 // its first A row is even (16-byte staging); row / column 0 of the shifted space
 // are padding: C(i, j) of the kernel is C_orig(i - 1, j - 1).
+// flags bit 2 (the syrk on U^s with the extend-add fused into its prologue,
+// SURVEY.md NEXT-1): C starts from 0 + the children's U^c in ascending order,
+// gathered through their relative maps, instead of from a U^s assembled in HBM;
+// s = the front, ea_qs[qs_off + j (ntr + 1) + t] = first row of child j whose
+// parent row falls in tile row t or below (ntr = tile rows of the problem).
 struct GemmProb {
     int64_t a_off;
     int64_t c_off;
     int32_t lda, ldc;
     int32_t M, N, K;
     int32_t flags;
+    int32_t s = -1;
+    int32_t qs_off = 0;
 };
-static_assert(sizeof(GemmProb) == 40, "GemmProb layout");
+static_assert(sizeof(GemmProb) == 48, "GemmProb layout");
+constexpr int32_t kProbU = 1, kProbShift = 2, kProbGather = 4;
 
 struct TileTask {       // one kTileM x kTileN output tile of a GemmProb
     int32_t prob;
@@ -176,6 +185,8 @@ struct Plan {
     std::vector<int32_t> panel_tasks;                // pairs (front, 64-row tile row), row-major over the fronts
     std::vector<GemmProb> probs;
     std::vector<TileTask> tiles;
+    std::vector<int32_t> ea_qs;                      // fused extend-add: per (syrk problem, child) tile-row starts
+    int32_t fuse_ea = 0;
     std::vector<Launch> program;
     // solve
     std::vector<int32_t> solve_list;                 // supernode lists (small / large) per launch

@@ -449,6 +449,29 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         }
         return b;
     };
+    // fused extend-add: child c's relative map positions below the parent's pivot
+    // columns: np = #rows of U^c landing in panel columns (a prefix: rel is
+    // increasing); its lower entries in panel columns = np mc - np (np - 1) / 2
+    auto child_np = [&](int32_t c, int32_t kp) -> int64_t {
+        const int32_t *rel = P.relmap.data() + P.relmap_ptr[c];
+        const int32_t mc = P.sn_f[c] - P.sn_k[c];
+        return std::lower_bound(rel, rel + mc, kp) - rel;
+    };
+    auto child_panel_entries = [&](int32_t c, int32_t kp) {
+        const double np = (double)child_np(c, kp), mc = P.sn_f[c] - P.sn_k[c];
+        return np * mc - np * (np - 1) / 2;
+    };
+    // assembly bytes of the panel columns only (the U^s part is gathered by the syrk)
+    auto asm_bytes_panel = [&](int32_t s) {
+        const int64_t e0 = S.bcolptr[S.sn_first[s]], e1 = S.bcolptr[S.sn_first[s + 1]];
+        double b = (double)(e1 - e0) * (8 + 4);
+        for (int32_t q = P.child_ptr[s]; q < P.child_ptr[s + 1]; q++) {
+            const int32_t c = P.child_list[q];
+            b += 8.0 * child_panel_entries(c, P.sn_k[s]) + 4.0 * (P.sn_f[c] - P.sn_k[c]);
+        }
+        return b;
+    };
+    P.fuse_ea = opt.fuse_ea ? 1 : 0;
     auto panel_words = [&](int32_t s) {
         const double k = P.sn_k[s], m = P.sn_f[s] - P.sn_k[s];
         return k * (k + 1) / 2 + k * m;
@@ -654,12 +677,17 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         {
             Launch L{KC_ASSEMBLE, 0, (int64_t)P.asm_tasks.size() / 2, 0, 0.0, 0.0, l};
             for (int32_t s : large) {
-                for (int32_t c0 = 0; c0 < P.sn_f[s]; c0 += kAsmCols) {
+                // fused extend-add: only the panel columns (the syrk gathers U^s)
+                const int32_t cend = P.fuse_ea ? P.sn_k[s] : P.sn_f[s];
+                for (int32_t c0 = 0; c0 < cend; c0 += kAsmCols) {
                     P.asm_tasks.push_back(s);
                     P.asm_tasks.push_back(c0);
                 }
                 const double f = P.sn_f[s], k = P.sn_k[s], m = f - k;
-                L.bytes += asm_bytes(s) + 8.0 * (f * k + m * (m + 1) / 2);   // zero + write panel and U
+                if (P.fuse_ea)
+                    L.bytes += asm_bytes_panel(s) + 8.0 * f * k;                // write the panel
+                else
+                    L.bytes += asm_bytes(s) + 8.0 * (f * k + m * (m + 1) / 2);   // zero + write panel and U
             }
             L.count = (int64_t)P.asm_tasks.size() / 2 - L.off;
             cur->push_back(L);
@@ -740,12 +768,35 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
             g.M += sh;
             g.N += sh;
             g.flags |= sh << 1;
+            // syrk bytes: read the k columns of L2, write the lower U^s; fused
+            // extend-add: + the children's entries landing in U^s (and their maps)
+            // instead of reading an assembled U^s
+            double sbytes = upd_bytes(m, m, k);
+            if (P.fuse_ea) {
+                g.flags |= kProbGather;
+                g.s = s;
+                g.qs_off = (int32_t)P.ea_qs.size();
+                const int32_t ntr = (g.M + kTileM - 1) / kTileM;
+                sbytes = 8.0 * ((double)m * k + (double)m * (m + 1) / 2);
+                for (int32_t q = P.child_ptr[s]; q < P.child_ptr[s + 1]; q++) {
+                    const int32_t c = P.child_list[q], mc = P.sn_f[c] - P.sn_k[c];
+                    const int32_t *rel = P.relmap.data() + P.relmap_ptr[c];
+                    // first child row whose parent row is >= max(k, k - sh + 64 t)
+                    for (int32_t t = 0; t <= ntr; t++) {
+                        const int32_t key = std::max(k, k - sh + kTileM * t);
+                        P.ea_qs.push_back((int32_t)(std::lower_bound(rel, rel + mc, key) - rel));
+                    }
+                    const double mcd = mc;
+                    sbytes += 8.0 * (mcd * (mcd + 1) / 2 - child_panel_entries(c, k)) + 4.0 * mc;
+                }
+                if (P.ea_qs.size() > (size_t)INT32_MAX) return MF_ERR_NOMEM;
+            }
             const int32_t pid = (int32_t)P.probs.size();
             P.probs.push_back(g);
             if (!P.dist[s]) {
                 add_tiles(P, pid, g.M, g.N, [](int32_t) { return true; });
                 Ls.flops += upd_flops(m, m, k);
-                Ls.bytes += upd_bytes(m, m, k);
+                Ls.bytes += sbytes;
                 continue;
             }
             const std::vector<int32_t> tb = split_tile_columns(g.N, R);
@@ -753,7 +804,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
             add_tiles(P, pid, g.M, g.N, [&](int32_t tj) { return tj >= tb[P.rank] && tj < tb[P.rank + 1]; });
             const double frac = (double)((int64_t)P.tiles.size() - t0) / (double)count_tiles(g.M, g.N);
             Ls.flops += frac * upd_flops(m, m, k);
-            Ls.bytes += frac * upd_bytes(m, m, k);
+            Ls.bytes += frac * sbytes;
             for (int r = 0; r < R; r++) {   // original columns of rank r's shifted tile columns
                 const int32_t c0 = std::max(0, tb[r] * kTileN - sh), c1 = std::min(m, tb[r + 1] * kTileN - sh);
                 if (c1 <= c0) continue;

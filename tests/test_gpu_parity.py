@@ -221,6 +221,26 @@ def test_deterministic_bitwise(mf):
     assert all(np.array_equal(outs[0], o) for o in outs[1:])
 
 
+@pytest.mark.parametrize("kind,dims,small_max,w", [("27pt", (18, 18, 18), 128, 64), ("7pt", (24, 24, 24), 8, 64),
+                                                    ("elast", (9, 9, 9), 48, 32), ("9pt", (90, 70, 1), 8, 16)])
+def test_fused_extend_add_bit_identical(mf, kind, dims, small_max, w):
+    """the extend-add of the U^s part fused into the syrk prologue
+    sums 0 + U^c1 + U^c2 ... per element in the assembly kernel's order (reading
+    C6), so L is bit-identical with fuse_ea on and off (odd and even k, shifted
+    problems, small and tiled children) -- and both match the oracle."""
+    A, p = grid(kind, dims)
+    outs = []
+    for fuse in (False, True):
+        S = mf.Solver(fuse_ea=fuse, small_front_max=small_max, panel_w=w)
+        S.analyze(A.n, A.colptr, A.rowind, p)
+        inf = S.info()
+        S.factor(A.values)
+        outs.append(S.export_L(sum_panel_words(S, inf)))
+    np.testing.assert_array_equal(outs[0], outs[1])
+    sym = oracle.symbolic(A, p, keep_struct=True)
+    check_panels(S, sym, oracle.factor(A, sym))
+
+
 def sum_panel_words(S, inf):
     sn = S.supernodes()
     k = np.diff(sn["sn_first"]).astype(np.int64)
