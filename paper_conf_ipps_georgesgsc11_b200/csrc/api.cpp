@@ -361,7 +361,9 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     d.ea_qs = ea_qs;
     d.fuse_ea = P.fuse_ea;
     void *p;
-    if ((r = dev_alloc(c, &p, P.L_words * sizeof(double))) != MF_OK) return r;
+    // + kTileM words: the bulk-copy Schur update stages whole 64-row operand columns,
+    // so the last tile row of the last panel may read past its f rows
+    if ((r = dev_alloc(c, &p, (P.L_words + kTileM) * sizeof(double))) != MF_OK) return r;
     d.L = (double *)p;
     if ((r = dev_alloc(c, &p, P.U_words * sizeof(double))) != MF_OK) return r;
     d.U = (double *)p;
@@ -407,7 +409,7 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
         c->bevents.push_back(e);
     }
     // the L arena starts zeroed once so that never-written padding words are defined
-    CK(cudaMemsetAsync(d.L, 0, P.L_words * sizeof(double), c->stream));
+    CK(cudaMemsetAsync(d.L, 0, (P.L_words + kTileM) * sizeof(double), c->stream));
     CK(cudaStreamSynchronize(c->stream));
 
     fill_info(c, n, 1);
@@ -461,7 +463,10 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
                 case KC_ASSEMBLE: launch_assemble(d, c->d_asm + 2 * L.off, L.count, v, st); break;
                 case KC_POTRF: launch_potrf_diag(d, c->d_large + L.off, (int)L.count, L.param, P.w, st); break;
                 case KC_TRSM: launch_trsm_panel(d, c->d_trsm + 2 * L.off, L.count, L.param, P.w, st); break;
-                case KC_UPDATE: launch_update(d, c->d_probs, c->d_tiles + L.off, L.count, st); break;
+                case KC_UPDATE:   // long-K launches of many waves take the bulk-copy pipeline
+                    launch_update(d, c->d_probs, c->d_tiles + L.off, L.count,
+                                  L.count >= kBulkMinTiles && L.flops >= kBulkMinK * 2.0 * kTileM * kTileN * L.count, st);
+                    break;
                 case KC_PANEL: launch_panel(d, c->d_panel + 2 * L.off, L.count, L.param, (int)L.count2, st); break;
                 case KC_LEAF:
                     launch_leaf(d, c->d_large + L.off, (int)L.count, c->d_trsm + 2 * L.off2, L.count2, L.param, P.w, st);

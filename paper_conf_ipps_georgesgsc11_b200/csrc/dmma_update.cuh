@@ -45,6 +45,38 @@ __device__ __forceinline__ void dmma(double &c0, double &c1, double a, double b)
                  : "d"(a), "d"(b));
 }
 
+// mbarrier + bulk-copy pipeline (the BULK variant): warp 0 stages every operand
+// column of a k-tile with one cp.async.bulk per lane (rows i0 .. i0+BM of an A
+// column are contiguous: 512 bytes), completing on the stage's "full" mbarrier;
+// each warp waits on it, computes, and arrives on the stage's "empty" mbarrier,
+// so no CTA-wide barrier sits in the main loop and no thread issues per-16-byte
+// copies.  Rows past M / N are staged as they are (they only feed masked
+// outputs: a DMMA output row depends on its own A row); k columns past K are
+// zero-filled by the producer lanes.
+__device__ __forceinline__ unsigned smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t *b, unsigned count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(smem_u32(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint64_t *b, unsigned tx) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(smem_u32(b)), "r"(tx) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t *b) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *b, unsigned parity) {
+    asm volatile(
+        "{\n .reg .pred p;\n MBW_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra MBW_%=;\n}\n" ::"r"(
+            smem_u32(b)),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, unsigned bytes, uint64_t *b) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(b))
+                 : "memory");
+}
+
 // Fused extend-add (GemmProb flags bit 2): the syrk on U^s
 // starts from the children's contributions gathered through their relative maps
 // (F^s = A-part (+) U^c1 (+) U^c2 ...; the U^s part of F^s has no A
@@ -72,12 +104,13 @@ struct UpdCfg {
     static constexpr int PSA16 = NT / CPA, PSB16 = NT / CPB;      // k stride of a thread
     static_assert(BK % PSA16 == 0 && BK % PSB16 == 0, "staging map");
     static constexpr int STAGE_WORDS = BK * (SA + SB);
-    static constexpr size_t SMEM = (size_t)STAGES * STAGE_WORDS * sizeof(double) + (BM + BN) * sizeof(int);
+    static constexpr size_t SMEM =
+        (size_t)STAGES * STAGE_WORDS * sizeof(double) + 2 * STAGES * sizeof(uint64_t) + (BM + BN) * sizeof(int);
     static_assert(SA % 16 == 4 && SB % 16 == 4, "bank-conflict-free fragment loads");
     static_assert(TM % 8 == 0 && TN % 8 == 0 && BK % 4 == 0, "tile shape");
 };
 
-template <class Cfg>
+template <class Cfg, bool BULK = false>
 __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
     k_update_t(double *__restrict__ Larena, double *__restrict__ Uarena, const GemmProb *__restrict__ probs,
                const TileTask *__restrict__ tiles, const UpdGather gv) {
@@ -118,10 +151,52 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
     };
 
     const int KT = (K + BK - 1) / BK;
+    uint64_t *full = reinterpret_cast<uint64_t *>(sm + STAGES * STAGE_WORDS), *empty = full + STAGES;
+    // BULK: warp 0 stages k-tile kt into ring slot `stage` (lane c: A column c, B column c - BK)
+    auto issue_bulk = [&](int stage, int kt) {
+        double *As = sm + stage * STAGE_WORDS;
+        double *Bs = As + BK * SA;
+        const int p0 = kt * BK, nv = min(BK, K - p0);
+        if (nv < BK) {   // k columns past K: zeros (generic stores, published by the arrive below)
+            for (int c = lane; c < 2 * BK; c += 32) {
+                const int p = c < BK ? c : c - BK;
+                if (p >= nv) {
+                    double *dst = c < BK ? As + p * SA : Bs + p * SB;
+                    for (int r = 0; r < (c < BK ? BM : BN); r++) dst[r] = 0.0;
+                }
+            }
+        }
+        __syncwarp();
+        constexpr int ra = BM, rb = BN;
+        if (lane == 0) mbar_arrive_tx(full + stage, (unsigned)(nv * (ra + rb) * sizeof(double)));
+        __syncwarp();
+        const double *__restrict__ Ak = A + (int64_t)p0 * lda;
+        for (int c = lane; c < 2 * BK; c += 32) {
+            const int p = c < BK ? c : c - BK;
+            if (p < nv) {
+                if (c < BK) bulk_g2s(As + p * SA, Ak + (int64_t)p * lda + i0, ra * sizeof(double), full + stage);
+                else bulk_g2s(Bs + p * SB, Ak + (int64_t)p * lda + j0, rb * sizeof(double), full + stage);
+            }
+        }
+    };
+    if constexpr (BULK) {
+        static_assert(Cfg::SA * sizeof(double) % 16 == 0 && Cfg::SB * sizeof(double) % 16 == 0, "bulk dst alignment");
+        if (tid == 0) {
+            for (int st = 0; st < STAGES; st++) {
+                mbar_init(full + st, 1);
+                mbar_init(empty + st, NT / 32);
+            }
+            asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+        }
+        __syncthreads();
+        if (warp == 0)
+            for (int st = 0; st < STAGES && st < KT; st++) issue_bulk(st, st);
+    } else {
 #pragma unroll
-    for (int st = 0; st < STAGES - 1; st++) {
-        if (st < KT) load_stage(st, st);
-        cp_async_commit();
+        for (int st = 0; st < STAGES - 1; st++) {
+            if (st < KT) load_stage(st, st);
+            cp_async_commit();
+        }
     }
     // C(i - sh, j - sh) for the (shifted) tile coordinates (i, j)
     double *__restrict__ C = ((g.flags & 1) ? Uarena : Larena) + g.c_off;
@@ -150,7 +225,7 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
         for (int mb = 0; mb < MB; mb++)
 #pragma unroll
             for (int nb = 0; nb < NB; nb++) acc[mb][nb][0] = acc[mb][nb][1] = 0.0;
-        int *rq = reinterpret_cast<int *>(sm + STAGES * STAGE_WORDS), *cq = rq + BM;
+        int *rq = reinterpret_cast<int *>(empty + STAGES), *cq = rq + BM;
         const int q0 = gv.child_ptr[g.s], q1 = gv.child_ptr[g.s + 1], kp = gv.sn_k[g.s];
         const int ntr1 = (g.M + BM - 1) / BM + 1;
         for (int jc = 0; jc < q1 - q0; jc++) {
@@ -183,9 +258,27 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
         }
     }
     for (int kt = 0; kt < KT; kt++) {
-        cp_async_wait<STAGES - 2>();
-        __syncthreads();
-        {
+        if constexpr (BULK) {
+            mbar_wait(full + kt % STAGES, (kt / STAGES) & 1);
+            // release the PREVIOUS slot: its LDS reads were consumed by the DMMAs of
+            // iteration kt-1, all issued before the wait loop above (a basic-block
+            // boundary ptxas does not schedule across).  Releasing right after the
+            // DMMAs instead lets ptxas hoist the arrive above them while their LDS are
+            // still in flight, and the bulk refill (async proxy) then races those
+            // reads (seen as stale A rows in ~10% of runs); a proxy fence there
+            // costs a MEMBAR per k-tile.
+            if (kt > 0) {
+                const int ps = (kt - 1) % STAGES;
+                __syncwarp();
+                if (lane == 0) mbar_arrive(empty + ps);
+                if (warp == 0 && kt - 1 + STAGES < KT) {
+                    mbar_wait(empty + ps, ((kt - 1) / STAGES) & 1);
+                    issue_bulk(ps, kt - 1 + STAGES);
+                }
+            }
+        } else {
+            cp_async_wait<STAGES - 2>();
+            __syncthreads();
             const int nk = kt + STAGES - 1;
             if (nk < KT) load_stage(nk % STAGES, nk);
             cp_async_commit();
@@ -205,7 +298,7 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
                 for (int nb = 0; nb < NB; nb++) dmma(acc[mb][nb][0], acc[mb][nb][1], a[mb], b[nb]);
         }
     }
-    cp_async_wait<0>();
+    if constexpr (!BULK) cp_async_wait<0>();
 #pragma unroll
     for (int mb = 0; mb < MB; mb++) {
         const int i = i0 + wm * TM + mb * 8 + gq;
@@ -220,18 +313,18 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
     }
 }
 
-template <class Cfg>
+template <class Cfg, bool BULK = false>
 inline void launch_update_t(double *L, double *U, const GemmProb *probs, const TileTask *tiles, int64_t ntiles,
                             cudaStream_t st, const UpdGather gv = UpdGather{}) {
     if (ntiles <= 0) return;
     if (Cfg::SMEM > 48 * 1024) {   // idempotent; libmf also sets it up front (kernels_init) before graph capture
         static bool attr = false;
         if (!attr) {
-            cudaFuncSetAttribute(k_update_t<Cfg>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Cfg::SMEM);
+            cudaFuncSetAttribute(k_update_t<Cfg, BULK>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Cfg::SMEM);
             attr = true;
         }
     }
-    k_update_t<Cfg><<<(unsigned)ntiles, Cfg::NT, Cfg::SMEM, st>>>(L, U, probs, tiles, gv);
+    k_update_t<Cfg, BULK><<<(unsigned)ntiles, Cfg::NT, Cfg::SMEM, st>>>(L, U, probs, tiles, gv);
 }
 
 }  // namespace mf

@@ -12,6 +12,7 @@
 // Determinism: extend-add has no atomics; every destination entry receives
 // 0, then its A value, then the children's contributions in ascending child
 // order (reading C6) -- the same summation order as the oracle.
+#include <cstdlib>
 #include <climits>
 #include <cstdio>
 
@@ -1217,12 +1218,27 @@ void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, in
 // ============================================================ DMMA Schur update
 // The production tile shape (kTileM x kTileN in mf_plan.h); variants are
 // benchmarked in tools/ubench/update_variants.cu.
-using UpdProd = UpdCfg<kTileM, kTileN, 16, 3, 2, 2, 4>;   // 33.5 TF/s on M=N=8192,K=4096 (ubench, even rows)
+// 64 x 64 tiles, BK 16, 3 stages, 4 CTAs / SM; staged by per-thread 16-byte
+// cp.async (33.2 TF/s on M=N=8192, K=4096) or, for launches of many long-K waves,
+// by the mbarrier + bulk-copy pipeline (33.8 TF/s there)
+using UpdProd = UpdCfg<kTileM, kTileN, 16, 3, 2, 2, 4>;
 
-void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, cudaStream_t st) {
+void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, bool bulk,
+                   cudaStream_t st) {
     if (ntiles <= 0) return;   // attributes were set by kernels_init()
     const UpdGather gv{d.child_ptr, d.child_list, d.sn_k, d.sn_f, d.U_off, d.relmap_ptr, d.relmap, d.ea_qs};
-    k_update_t<UpdProd><<<(unsigned)ntiles, UpdProd::NT, UpdProd::SMEM, st>>>(d.L, d.U, probs, tiles, gv);
+    // MF_UPD_BULK (A/B checks): 0 = cp.async everywhere, 1 = bulk everywhere; unset = per launch
+    static const int mode = [] {
+        const char *e = getenv("MF_UPD_BULK");
+        return e ? atoi(e) : -1;
+    }();
+    if (mode >= 0) bulk = mode == 1;
+#define MF_UPD_LAUNCH(V) k_update_t<UpdProd, V><<<(unsigned)ntiles, UpdProd::NT, UpdProd::SMEM, st>>>(d.L, d.U, probs, tiles, gv)
+    if (bulk)
+        MF_UPD_LAUNCH(true);
+    else
+        MF_UPD_LAUNCH(false);
+#undef MF_UPD_LAUNCH
 }
 
 void launch_init_failed(int *failed, cudaStream_t st) { k_init_failed<<<1, 1, 0, st>>>(failed, reinterpret_cast<unsigned *>(failed + 1)); }
@@ -1240,7 +1256,9 @@ int kernels_init() {
     if (e == cudaSuccess)
         e = cudaFuncSetAttribute(k_panel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kPanelSmem);
     if (e == cudaSuccess)
-        e = cudaFuncSetAttribute(k_update_t<UpdProd>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)UpdProd::SMEM);
+        e = cudaFuncSetAttribute(k_update_t<UpdProd, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)UpdProd::SMEM);
+    for (auto fn : {k_update_t<UpdProd, true>})
+        if (e == cudaSuccess) e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)UpdProd::SMEM);
     return e == cudaSuccess ? 0 : -1;
 }
 

@@ -241,6 +241,43 @@ def test_fused_extend_add_bit_identical(mf, kind, dims, small_max, w):
     check_panels(S, sym, oracle.factor(A, sym))
 
 
+_BULK_CHILD = r'''
+import hashlib, sys
+sys.path.insert(0, ".")
+import numpy as np
+import paper_conf_ipps_georgesgsc11_b200 as mf
+from tests._grids import grid
+kind, dims, sm = sys.argv[1], tuple(int(x) for x in sys.argv[2].split(",")), int(sys.argv[3])
+A, p = grid(kind, dims)
+S = mf.Solver(small_front_max=sm, nbranch=1)
+S.analyze(A.n, A.colptr, A.rowind, p)
+S.factor(A.values)
+sn = S.supernodes()
+k = np.diff(sn["sn_first"]); f = np.diff(sn["sn_rowptr"])
+print(hashlib.sha256(S.export_L(int(np.sum((f + (f & 1)) * k)) + 2).tobytes()).hexdigest())
+'''
+
+
+@pytest.mark.parametrize("kind,dims,sm", [("27pt", (20, 20, 20), 8), ("7pt", (28, 28, 28), 128)])
+def test_bulk_staging_bit_identical(mf, kind, dims, sm):
+    """The DMMA update's two operand-staging pipelines (per-thread cp.async with
+    CTA barriers; warp-0 bulk copies with full/empty mbarriers) compute every
+    element in the same order, so L is bitwise equal with either forced on every
+    launch (MF_UPD_BULK=0/1; the default picks per launch).  Guards the
+    generic-read -> async-write hazard on the ring slots (DESIGN.md Sec. 7)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = []
+    for mode in ("0", "1", "1"):
+        r = subprocess.run([sys.executable, "-c", _BULK_CHILD, kind, ",".join(map(str, dims)), str(sm)], cwd=root,
+                           env=dict(os.environ, MF_UPD_BULK=mode), capture_output=True, text=True, timeout=600)
+        assert r.returncode == 0, r.stderr[-2000:]
+        out.append(r.stdout.strip().splitlines()[-1])
+    assert out[0] == out[1] == out[2]
+
+
 def sum_panel_words(S, inf):
     sn = S.supernodes()
     k = np.diff(sn["sn_first"]).astype(np.int64)

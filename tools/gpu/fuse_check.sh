@@ -1,4 +1,3 @@
 set -x
 timeout 1200 python -m pytest tests -x -q -m gpu > gpurun_out/pytest_gpu.log 2>&1; tail -5 gpurun_out/pytest_gpu.log
-for c in c5 c3 c2; do timeout 600 python bench.py --config $c --steps 5 --warmup 3 --no-cpu-baseline > gpurun_out/bench_$c.json 2> gpurun_out/bench_$c.err; tail -1 gpurun_out/bench_$c.err; python -c "import json;d=json.load(open('gpurun_out/bench_$c.json'));print('$c', round(d['ms_per_step'],3), 'ms', round(d['value']), 'e2e', round(d['e2e']['value']), [(k['name'], round(k['ms']/d['steps'],2)) for k in d['kernels']])"; done
-timeout 600 python tools/level_breakdown.py c5 1 > gpurun_out/levels_c5_fused.txt 2>&1; tail -3 gpurun_out/levels_c5_fused.txt
+for c in c5 c3 c2 c4; do timeout 600 python bench.py --config $c --steps 5 --warmup 3 --no-cpu-baseline > gpurun_out/bench_$c.json 2> gpurun_out/bench_$c.err; tail -1 gpurun_out/bench_$c.err; python -c "import json;d=json.load(open('gpurun_out/bench_$c.json'));print('$c', round(d['ms_per_step'],3), 'ms', round(d['value']), 'e2e', round(d['e2e']['value']), 'roof', round(d['roofline']['frac'],3), [(k['name'], round(k['ms']/d['steps'],2)) for k in d['kernels']])"; done

@@ -52,6 +52,9 @@ def main():
             parts.append(f"{name}:{n}x {ms:7.2f}ms {rate}")
         print(f"L{l:2d} " + " | ".join(parts))
     print("totals:", {k: round(v, 2) for k, v in tot.items()})
+    if os.environ.get("DUMP"):
+        import json
+        json.dump([dict(L, ms=float(ms)) for L, ms in zip(prog, t)], open(os.environ["DUMP"], "w"))
     sn = S.supernodes()
     first, par = sn["sn_first"], sn["sn_parent"]
     k = np.diff(first)

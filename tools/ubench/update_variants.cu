@@ -11,7 +11,7 @@
 
 using namespace mf;
 
-template <class Cfg>
+template <class Cfg, bool BULK = false>
 double run(const char *name, double *L, double *U, int M, int N, int K, int ld, std::vector<double> &out,
            int aoff = 0, int reps = 5) {
     std::vector<TileTask> tiles;
@@ -35,7 +35,7 @@ double run(const char *name, double *L, double *U, int M, int N, int K, int ld, 
     for (int r = 0; r < reps + 1; r++) {
         cudaMemset(U, 0, (size_t)M * M * sizeof(double));
         cudaEventRecord(e0);
-        launch_update_t<Cfg>(L, U, dp, dt, (int64_t)tiles.size(), 0);
+        launch_update_t<Cfg, BULK>(L, U, dp, dt, (int64_t)tiles.size(), 0);
         cudaEventRecord(e1);
         cudaEventSynchronize(e1);
         float ms;
@@ -61,28 +61,35 @@ double run(const char *name, double *L, double *U, int M, int N, int K, int ld, 
 }
 
 int main(int argc, char **argv) {
+    setvbuf(stdout, nullptr, _IONBF, 0);
     int M = 8192, K = 4096;
     if (argc > 1) M = atoi(argv[1]);
     if (argc > 2) K = atoi(argv[2]);
     const int N = M, ld = M + 2;   // odd shift exercised by a_off = 1
     double *L, *U;
-    cudaMalloc(&L, ((size_t)ld * K + 16) * sizeof(double));
+    cudaMalloc(&L, ((size_t)ld * K + 256) * sizeof(double));
     cudaMalloc(&U, (size_t)M * M * sizeof(double));
     std::vector<double> hA((size_t)ld * K + 16);
     srand(1);
     for (auto &x : hA) x = (double)(rand() % 17 - 8);   // small integers: exact sums, any order
     cudaMemcpy(L, hA.data(), hA.size() * sizeof(double), cudaMemcpyHostToDevice);
-    double *Lshift = L;   // a_off = 0 here; odd offsets covered by the GPU parity tests
+    double *Lshift = L;   // a_off = 0 here: the kernel requires even first rows (the planner shifts odd ones)
     std::vector<double> ref;
     printf("lower-trapezoid SYRK M=N=%d K=%d\n", M, K);
     std::vector<double> ref1;
     run<UpdCfg<64, 64, 16, 3, 2, 2, 4>>("64x64 bk16 s3 w2x2 m4", Lshift, U, M, N, K, ld, ref);
-    run<UpdCfg<64, 64, 16, 3, 2, 2, 4>>("64x64 bk16 s3 w2x2 m4", Lshift, U, M, N, K, ld, ref1, 1);
+    run<UpdCfg<64, 64, 16, 3, 2, 2, 4>, true>("BULK 64x64 bk16 s3 w2x2 m4", Lshift, U, M, N, K, ld, ref);
+    run<UpdCfg<64, 64, 8, 6, 2, 2, 4>, true>("BULK 64x64 bk8 s6 w2x2 m4", Lshift, U, M, N, K, ld, ref);
+    run<UpdCfg<64, 64, 8, 5, 2, 2, 4>, true>("BULK 64x64 bk8 s5 w2x2 m4", Lshift, U, M, N, K, ld, ref);
+    run<UpdCfg<64, 64, 32, 2, 2, 2, 3>, true>("BULK 64x64 bk32 s2 w2x2 m3", Lshift, U, M, N, K, ld, ref);
+    run<UpdCfg<64, 64, 16, 4, 2, 2, 3>, true>("BULK 64x64 bk16 s4 w2x2 m3", Lshift, U, M, N, K, ld, ref);
+    run<UpdCfg<128, 64, 16, 3, 2, 2, 2>, true>("BULK 128x64 bk16 s3 w2x2 (64x32) m2", Lshift, U, M, N, K, ld, ref);
     run<UpdCfg<64, 64, 16, 4, 2, 2, 3>>("64x64 bk16 s4 w2x2 m3", Lshift, U, M, N, K, ld, ref);
     run<UpdCfg<64, 64, 32, 2, 2, 2, 3>>("64x64 bk32 s2 w2x2 m3", Lshift, U, M, N, K, ld, ref);
     run<UpdCfg<64, 64, 32, 3, 2, 2, 2>>("64x64 bk32 s3 w2x2 m2", Lshift, U, M, N, K, ld, ref);
     run<UpdCfg<128, 64, 16, 4, 4, 2, 2>>("128x64 bk16 s4 w4x2 m2", Lshift, U, M, N, K, ld, ref);
-    run<UpdCfg<128, 64, 16, 4, 4, 2, 2>>("128x64 bk16 s4 w4x2 m2", Lshift, U, M, N, K, ld, ref1, 1);
+    run<UpdCfg<128, 64, 16, 3, 2, 2, 2>>("128x64 bk16 s3 w2x2 (64x32) m2", Lshift, U, M, N, K, ld, ref);
+    run<UpdCfg<64, 128, 16, 3, 2, 2, 2>>("64x128 bk16 s3 w2x2 (32x64) m2", Lshift, U, M, N, K, ld, ref);
     run<UpdCfg<128, 128, 16, 4, 4, 4, 1>>("128x128 bk16 s4 w4x4 m1", Lshift, U, M, N, K, ld, ref);
     run<UpdCfg<64, 128, 16, 3, 2, 4, 2>>("64x128 bk16 s3 w2x4 m2", Lshift, U, M, N, K, ld, ref);
     run<UpdCfg<128, 128, 16, 3, 2, 2, 1>>("128x128 bk16 s3 w2x2 (64x64) m1", Lshift, U, M, N, K, ld, ref);
