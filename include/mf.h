@@ -83,6 +83,13 @@ typedef struct {
                                  a U^s assembled in HBM); 0 = the
                                  assembly kernel builds the whole front.  Both give bit-identical
                                  fronts (same summation order, reading C6).                         */
+    int32_t lookahead;        /* 1 = single GPU, main stream: each trailing update of a
+                                 large front is split into the columns the next panel needs and the
+                                 rest, which runs on a low-priority side stream beside that panel
+                                 (the paper's overlap of CPU and GPU work [P:L325] as overlap of the
+                                 latency-bound panel with throughput-bound updates); 0 (default) =
+                                 one stream.  Same arithmetic either way (bit-identical L); measured
+                                 no faster on c3-c5 (the co-running update slows the panel chain). */
 } mf_options;
 
 typedef struct {

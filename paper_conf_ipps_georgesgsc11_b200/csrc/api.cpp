@@ -14,6 +14,7 @@
 #include <cstdio>
 #include <cstring>
 #include <new>
+#include <map>
 #include <vector>
 
 #include "kernels.cuh"
@@ -59,6 +60,10 @@ struct mf_ctx {
     // single GPU: one stream per subtree branch, forked from / joined into `stream`
     std::vector<cudaStream_t> bstreams;
     std::vector<cudaEvent_t> bevents;   // [0] fork, [1 + b] join of branch b
+    // look-ahead: the main path of the top fronts on a high-priority stream, the
+    // split-off trailing updates on a low-priority side stream
+    cudaStream_t la_hi = nullptr, la_side = nullptr;
+    cudaEvent_t la_ev[4] = {nullptr, nullptr, nullptr, nullptr};   // hi fork, side fork, side join, hi join
     mf_kernel_stat kstats[KC_COUNT];
     int64_t prof_factors = 0;
 };
@@ -189,6 +194,7 @@ int mf_default_options(mf_options *o) {
     o->split_all = 0;
     o->nbranch = d.nbranch;
     o->fuse_ea = d.fuse_ea;
+    o->lookahead = d.lookahead;
     return MF_OK;
 }
 
@@ -221,6 +227,7 @@ int mf_create(mf_ctx **out, const mf_options *o) {
     }
     c->opt.nbranch = o->nbranch;
     c->opt.fuse_ea = o->fuse_ea != 0;
+    c->opt.lookahead = o->lookahead != 0;
     c->opt.rank = o->rank;
     c->host_only = o->host_only != 0;
     c->info.failed_col = -1;
@@ -269,6 +276,10 @@ void mf_destroy(mf_ctx *c) {
     free_device(c);
     for (cudaEvent_t e : c->prof_events) cudaEventDestroy(e);
     for (cudaEvent_t e : c->bevents) cudaEventDestroy(e);
+    for (cudaEvent_t e : c->la_ev)
+        if (e) cudaEventDestroy(e);
+    if (c->la_hi) cudaStreamDestroy(c->la_hi);
+    if (c->la_side) cudaStreamDestroy(c->la_side);
     for (cudaStream_t bs : c->bstreams) cudaStreamDestroy(bs);
     if (c->ev0) cudaEventDestroy(c->ev0);
     if (c->ev1) cudaEventDestroy(c->ev1);
@@ -408,6 +419,13 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
         CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
         c->bevents.push_back(e);
     }
+    if (P.nside > 0 && !c->la_hi) {
+        int least = 0, greatest = 0;
+        CK(cudaDeviceGetStreamPriorityRange(&least, &greatest));
+        CK(cudaStreamCreateWithPriority(&c->la_hi, cudaStreamNonBlocking, greatest));
+        CK(cudaStreamCreateWithPriority(&c->la_side, cudaStreamNonBlocking, least));
+        for (cudaEvent_t &e : c->la_ev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    }
     // the L arena starts zeroed once so that never-written padding words are defined
     CK(cudaMemsetAsync(d.L, 0, (P.L_words + kTileM) * sizeof(double), c->stream));
     CK(cudaStreamSynchronize(c->stream));
@@ -443,6 +461,9 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
             joined = true;
             return MF_OK;
         };
+        // look-ahead streams (graph replay only; profiled runs stay on one stream)
+        const bool la = !with_events && c->la_hi != nullptr;
+        cudaStream_t mainst = st;
         for (size_t li = i0; li < i1; li++) {
             const Launch &L = prog[li];
             cudaStream_t ls = st;
@@ -455,6 +476,22 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
                 ls = c->bstreams[L.stream];
             } else if (branches && forked && !joined) {
                 if (int r = join()) return r;
+            }
+            if (la && L.stream < 0) {
+                if (mainst == st) {   // the main path moves to the high-priority stream
+                    CK(cudaEventRecord(c->la_ev[0], st));
+                    CK(cudaStreamWaitEvent(c->la_hi, c->la_ev[0], 0));
+                    mainst = c->la_hi;
+                }
+                ls = mainst;
+                if (L.side) {
+                    CK(cudaEventRecord(c->la_ev[1], mainst));
+                    CK(cudaStreamWaitEvent(c->la_side, c->la_ev[1], 0));
+                    ls = c->la_side;
+                } else if (L.join) {
+                    CK(cudaEventRecord(c->la_ev[2], c->la_side));
+                    CK(cudaStreamWaitEvent(mainst, c->la_ev[2], 0));
+                }
             }
             auto launch = [&](cudaStream_t st) -> int {
             if (with_events) CK(cudaEventRecord(c->prof_events[ev_base + 2 * li], st));
@@ -481,6 +518,10 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
         if (forked && !joined) {
             if (int r = join()) return r;
         }
+        if (mainst != st) {
+            CK(cudaEventRecord(c->la_ev[3], mainst));
+            CK(cudaStreamWaitEvent(st, c->la_ev[3], 0));
+        }
         return MF_OK;
     };
     if (c->profiling) return issue(vals, true);
@@ -496,7 +537,25 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
         if (r) return r;
         CK(e);
         *graph = g;
-        CK(cudaGraphInstantiate(exec, g, 0));
+        // node priorities (captured from the look-ahead streams) decide which ready
+        // kernel gets free SM slots first: the panel path before the side updates
+        if (getenv("MF_DEBUG_GRAPH")) {   // node priorities as captured (look-ahead check)
+            size_t nn = 0;
+            cudaGraphGetNodes(g, nullptr, &nn);
+            std::vector<cudaGraphNode_t> nodes(nn);
+            cudaGraphGetNodes(g, nodes.data(), &nn);
+            std::map<int, int> hist;
+            for (cudaGraphNode_t nd : nodes) {
+                cudaGraphNodeType t;
+                cudaGraphNodeGetType(nd, &t);
+                if (t != cudaGraphNodeTypeKernel) continue;
+                cudaLaunchAttributeValue v{};
+                if (cudaGraphKernelNodeGetAttribute(nd, cudaLaunchAttributePriority, &v) == cudaSuccess) hist[v.priority]++;
+                else hist[999]++;
+            }
+            for (auto &kv : hist) fprintf(stderr, "[libmf] graph kernel nodes with priority %d: %d\n", kv.first, kv.second);
+        }
+        CK(cudaGraphInstantiateWithFlags(exec, g, cudaGraphInstantiateFlagUseNodePriority));
     }
     CK(cudaGraphLaunch(*exec, st));
     return MF_OK;

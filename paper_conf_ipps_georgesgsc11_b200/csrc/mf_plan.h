@@ -24,6 +24,7 @@ struct Options {
     int split_all = 0;   // multi-GPU mapping ignores the exchange-cost model
     int fuse_ea = 1;     // extend-add into the U^s part fused into the syrk prologue (NEXT-1)
     int nbranch = 4;     // single GPU: concurrent subtree branches (graph branches on their own streams)
+    int lookahead = 0;   // single GPU, main stream: trailing update split so the next panel overlaps its rest (measured: no gain; off)
     // learned kernel-variant selector (Sec. VI, Eqs. 3-5):
     // theta is kVariantFeatures x kVariants (column j = class j); empty = the fixed
     // front-order thresholds.  force_variant >= 0 forces that class wherever feasible.
@@ -148,6 +149,10 @@ struct Launch {
     int32_t level;
     int64_t off2 = 0, count2 = 0;   // KC_LEAF: the trsm tasks (off/count = the fronts); KC_PANEL: count2 = blocks
     int32_t stream = -1;            // single GPU: subtree branch (its own stream), -1 = the main stream
+    // look-ahead (main stream only): side = 1 runs this launch on the low-priority
+    // side stream, forked from the main stream at this point; join = 1 makes the
+    // main stream wait for the side stream before this launch
+    int32_t side = 0, join = 0;
 };
 
 // Triangular-solve program (forward sweep bottom-up, backward sweep top-down).
@@ -187,6 +192,7 @@ struct Plan {
     std::vector<TileTask> tiles;
     std::vector<int32_t> ea_qs;                      // fused extend-add: per (syrk problem, child) tile-row starts
     int32_t fuse_ea = 0;
+    int32_t nside = 0;                               // look-ahead forks in the program
     std::vector<Launch> program;
     // solve
     std::vector<int32_t> solve_list;                 // supernode lists (small / large) per launch

@@ -511,14 +511,27 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     // the update of the pivot-column leaves [mid, b) by the factored leaves [a, mid)
     // (units of w) for the fronts fl (sorted by k descending): one DMMA launch with
     // inner dimension (mid - a) w; tiles of global column col only if keep(s, col)
-    auto rec_update = [&](const std::vector<int32_t> &fl, int32_t a, int32_t mid, int32_t b, int32_t l,
-                          const std::function<bool(int32_t, int32_t)> &keep) {
-        const int32_t c0 = mid * w, c_lo = a * w;
+    // look-ahead bookkeeping: the next main-stream launch after a panel that ran
+    // beside a side-stream update must join the side stream
+    bool need_join = false, join_armed = false;
+    auto push = [&](Launch L) {
+        if (join_armed && !L.side) {
+            L.join = 1;
+            join_armed = need_join = false;
+        }
+        cur->push_back(L);
+    };
+    // the update of the pivot-column leaves [jlo, b) (default jlo = mid) by the
+    // factored leaves [a, mid) (units of w)
+    auto rec_update_cols = [&](const std::vector<int32_t> &fl, int32_t a, int32_t mid, int32_t jlo, int32_t b,
+                               int32_t l, const std::function<bool(int32_t, int32_t)> &keep, int32_t side) {
+        const int32_t c0 = jlo * w, c_lo = a * w;
         Launch Lu{KC_UPDATE, 0, (int64_t)P.tiles.size(), 0, 0.0, 0.0, l};
+        Lu.side = side;
         for (int32_t s : fl) {
             const int32_t k = P.sn_k[s], f = P.sn_f[s], ld = P.sn_ld[s];
             if (k <= c0) continue;
-            const int32_t M = f - c0, N = std::min(b * w, k) - c0, K = c0 - c_lo;
+            const int32_t M = f - c0, N = std::min(b * w, k) - c0, K = mid * w - c_lo;
             if (M <= 0 || N <= 0) continue;
             GemmProb g;
             g.a_off = P.L_off[s] + (int64_t)c_lo * ld + c0;
@@ -543,8 +556,14 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
             Lu.bytes += frac * upd_bytes(M, N, K);
         }
         Lu.count = (int64_t)P.tiles.size() - Lu.off;
-        if (Lu.count) cur->push_back(Lu);
+        if (Lu.count) push(Lu);
+        return Lu.count > 0;
     };
+    auto rec_update = [&](const std::vector<int32_t> &fl, int32_t a, int32_t mid, int32_t b, int32_t l,
+                          const std::function<bool(int32_t, int32_t)> &keep) {
+        rec_update_cols(fl, a, mid, mid, b, l, keep, 0);
+    };
+    bool lookahead_pass = false;
     auto keep_all = [](int32_t, int32_t) { return true; };
     // the blocked factorization of the pivot-column leaves [a, b) (units of w) of the
     // fronts fl (sorted by k descending, stored at P.large_list[loff..])
@@ -578,7 +597,8 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
             Lp.bytes += 16.0 * (f - j0) * (je - j0);
         }
         Lp.count = (int64_t)P.panel_tasks.size() / 2 - Lp.off;
-        cur->push_back(Lp);
+        push(Lp);
+        if (need_join) join_armed = true;   // the side update must finish before the next main launch
     };
     std::function<void(const std::vector<int32_t> &, int64_t, int32_t, int32_t, int32_t)> rec =
         [&](const std::vector<int32_t> &fl, int64_t loff, int32_t a, int32_t b, int32_t l) {
@@ -612,16 +632,38 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
                 Launch Lf{KC_LEAF, j0, Lp.off, Lp.count, Lp.flops + Lt.flops, Lp.bytes + Lt.bytes, l};
                 Lf.off2 = Lt.off;
                 Lf.count2 = Lt.count;
-                cur->push_back(Lf);
+                push(Lf);
                 return;
             }
-            cur->push_back(Lp);
-            if (Lt.count) cur->push_back(Lt);
+            push(Lp);
+            if (Lt.count) push(Lt);
             return;
         }
         const int32_t mid = a + (b - a + 1) / 2;
         rec(fl, loff, a, mid, l);
-        rec_update(fl, a, mid, b, l, keep_all);
+        // look-ahead: the first panel of rec(mid, b) covers the leaves [mid, f1); only
+        // those columns of the update are on its critical path.  The rest [f1, b) runs
+        // on the side stream, beside that panel, and is joined before the next launch.
+        int32_t f1 = b;
+        if (lookahead_pass && w == 64 && !need_join) {
+            f1 = mid;
+            int32_t bb = b;
+            while (bb - f1 > kPanelMaxBlocks) bb = f1 + (bb - f1 + 1) / 2;
+            f1 = bb;
+        }
+        if (f1 < b) {
+            // the side part is forked AFTER the critical part: when that finishes, the
+            // panel (high priority) and the side update become ready together, and the
+            // panel's CTAs are placed first (the side's long-K tiles would otherwise
+            // hold every SM slot for up to a millisecond)
+            rec_update_cols(fl, a, mid, mid, f1, l, keep_all, 0);
+            if (rec_update_cols(fl, a, mid, f1, b, l, keep_all, 1)) {
+                need_join = true;
+                P.nside++;
+            }
+        } else {
+            rec_update(fl, a, mid, b, l, keep_all);
+        }
         rec(fl, loff, mid, b, l);
     };
     auto push_large = [&](const std::vector<int32_t> &fl) {
@@ -630,7 +672,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         return off;
     };
     auto push_xfers = [&](std::vector<XferSpec> &&x, int32_t l) {
-        cur->push_back(Launch{KC_EXCHANGE, (int32_t)P.xfers.size(), 0, 0, 0.0, 0.0, l});
+        push(Launch{KC_EXCHANGE, (int32_t)P.xfers.size(), 0, 0, 0.0, 0.0, l});
         P.xfers.push_back(std::move(x));
     };
     // passes over the levels: single GPU = one per branch (stream b), then the top
@@ -651,6 +693,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     for (const Pass &pass : passes) {
     const std::vector<char> &inc = pass.inc;
     cur = pass.prog;
+    lookahead_pass = opt.lookahead && R == 1 && pass.stream < 0;
     const size_t pass_begin = cur->size();
     for (int32_t l = 0; l < nlev; l++) {
         std::vector<int32_t> fronts;
@@ -666,7 +709,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
                     L.bytes += asm_bytes(s) + 8.0 * (panel_words(s) + m * (m + 1) / 2);
                 }
             L.count = (int64_t)P.small_list.size() - L.off;
-            if (L.count) cur->push_back(L);
+            if (L.count) push(L);
         }
         std::vector<int32_t> large;
         for (int32_t s : fronts)
@@ -690,7 +733,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
                     L.bytes += asm_bytes(s) + 8.0 * (f * k + m * (m + 1) / 2);   // zero + write panel and U
             }
             L.count = (int64_t)P.asm_tasks.size() / 2 - L.off;
-            cur->push_back(L);
+            push(L);
         }
         // Blocked factorization of the k pivot columns of every large front, in
         // lockstep over the level (Fig. 9: w x w potrf kernel, trsm
@@ -813,8 +856,11 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
             }
         }
         Ls.count = (int64_t)P.tiles.size() - Ls.off;
-        if (Ls.count) cur->push_back(Ls);
+        if (Ls.count) push(Ls);
         if (!ux.empty()) push_xfers(std::move(ux), l);
+    }
+    if (join_armed || need_join) {   // (cannot happen: every fork is followed by its panel and a launch)
+        return MF_ERR_STATE;
     }
     for (size_t i = pass_begin; i < cur->size(); i++) (*cur)[i].stream = pass.stream;
     }   // pass

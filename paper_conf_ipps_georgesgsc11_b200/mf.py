@@ -38,7 +38,7 @@ class Options(ctypes.Structure):
         ("small_front_max", ctypes.c_int32), ("panel_w", ctypes.c_int32), ("device", ctypes.c_int32),
         ("host_only", ctypes.c_int32), ("nranks", ctypes.c_int32), ("rank", ctypes.c_int32),
         ("stream", ctypes.c_void_p), ("split_all", ctypes.c_int32), ("nbranch", ctypes.c_int32),
-        ("fuse_ea", ctypes.c_int32),
+        ("fuse_ea", ctypes.c_int32), ("lookahead", ctypes.c_int32),
     ]
 
 
@@ -156,7 +156,7 @@ class Solver:
     def __init__(self, amalgamate: bool = True, small_front_max: int | None = None, panel_w: int | None = None,
                  device: int = -1, stream: int | None = None, host_only: bool = False,
                  nranks: int = 1, rank: int = 0, exchange=None, split_all: bool = False,
-                 nbranch: int | None = None, fuse_ea: bool | None = None):
+                 nbranch: int | None = None, fuse_ea: bool | None = None, lookahead: bool | None = None):
         o = Options()
         lib.mf_default_options(ctypes.byref(o))
         o.amalgamate = int(amalgamate)
@@ -173,6 +173,8 @@ class Solver:
             o.nbranch = nbranch
         if fuse_ea is not None:
             o.fuse_ea = int(fuse_ea)
+        if lookahead is not None:
+            o.lookahead = int(lookahead)
         o.stream = stream
         h = ctypes.c_void_p()
         r = lib.mf_create(ctypes.byref(h), ctypes.byref(o))

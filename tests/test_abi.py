@@ -37,7 +37,7 @@ def test_strerror_and_defaults():
     o = mf.Options()
     assert mf.lib.mf_default_options(ctypes.byref(o)) == 0
     assert list(o.nrelax) == [4, 16, 48] and list(o.zrelax) == [0.8, 0.1, 0.05]
-    assert o.fuse_ea == 1 and o.nbranch == 4
+    assert o.fuse_ea == 1 and o.nbranch == 4 and o.lookahead == 0
     assert mf.lib.mf_default_options(None) == mf.MF_ERR_ARG
 
 

@@ -241,6 +241,25 @@ def test_fused_extend_add_bit_identical(mf, kind, dims, small_max, w):
     check_panels(S, sym, oracle.factor(A, sym))
 
 
+@pytest.mark.parametrize("kind,dims,nb", [("27pt", (24, 24, 24), 1), ("7pt", (32, 32, 32), 4), ("elast", (10, 10, 10), 1)])
+def test_lookahead_bit_identical(mf, kind, dims, nb):
+    """Look-ahead (trailing updates split so the next panel runs beside the rest on
+    a side stream) changes only the schedule: L is bitwise equal with it on and
+    off, and matches the oracle."""
+    A, p = grid(kind, dims)
+    outs = []
+    for la in (False, True, True):
+        S = mf.Solver(lookahead=la, nbranch=nb)
+        S.analyze(A.n, A.colptr, A.rowind, p)
+        inf = S.info()
+        S.factor(A.values)
+        outs.append(S.export_L(sum_panel_words(S, inf)))
+    np.testing.assert_array_equal(outs[0], outs[1])
+    np.testing.assert_array_equal(outs[0], outs[2])
+    sym = oracle.symbolic(A, p, keep_struct=True)
+    check_panels(S, sym, oracle.factor(A, sym))
+
+
 _BULK_CHILD = r'''
 import hashlib, sys
 sys.path.insert(0, ".")
