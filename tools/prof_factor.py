@@ -13,7 +13,7 @@ from workloads import grids as G  # noqa: E402
 cfg = sys.argv[1] if len(sys.argv) > 1 else "c5"
 c = G.CONFIGS[cfg]
 A, p = G.make_config(c["kind"], c["N"])
-S = mf.Solver()
+S = mf.Solver(nbranch=int(os.environ.get("NB", "4")))
 S.analyze(A.n, A.colptr, A.rowind, p)
 v = torch.from_numpy(A.values).cuda()
 S.factor(v)
