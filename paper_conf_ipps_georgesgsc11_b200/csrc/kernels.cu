@@ -548,7 +548,7 @@ __device__ __forceinline__ void wait_flag(const unsigned *flag, unsigned expect)
         unsigned v;
         do {
             asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(flag) : "memory");
-            if (v != expect) __nanosleep(200);
+            if (v != expect) __nanosleep(32);
         } while (v != expect);
     }
     __syncthreads();
@@ -1028,19 +1028,22 @@ __device__ __forceinline__ void panel_potrf_dmma(const DevPlan &d, double *A, do
 }
 
 // X <- X L^-T for the 64 rows of Xs over wb columns; Ls = the wb x wb lower factor
-// (identity-padded to a multiple of 8), inv = 1 / diag.  8-column blocks: one
-// thread per row solves the block (substitution), then the four warps apply it
-// to the remaining columns with DMMA (16 rows each).
+// (identity-padded to a multiple of 8), inv = 1 / diag.  Each warp owns 16 rows:
+// per 8-column block, 16 of its lanes solve their rows over the block
+// (substitution), then the warp applies the block to its rows' remaining columns
+// with DMMA -- warps never share rows, so only warp-level synchronisation (the
+// 16 CTA barriers of a row-per-thread substitution cost ~half of the trsm).
 __device__ __forceinline__ void panel_trsm(double *Xs, const double *Ls, const double *inv, int wb) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, gq = lane >> 2, tq = lane & 3;
     const int ncb = (wb + 7) / 8;
+    const int row = warp * 16 + (lane & 15);
 #pragma unroll 1
     for (int cb = 0; cb < ncb; cb++) {
         const int c0 = cb * 8;
-        if (tid < 64) {
+        if (lane < 16) {
             double xv[8];
 #pragma unroll
-            for (int q = 0; q < 8; q++) xv[q] = Xs[tid + (c0 + q) * kPLD];
+            for (int q = 0; q < 8; q++) xv[q] = Xs[row + (c0 + q) * kPLD];
 #pragma unroll
             for (int q = 0; q < 8; q++) {
                 xv[q] *= inv[c0 + q];
@@ -1048,9 +1051,9 @@ __device__ __forceinline__ void panel_trsm(double *Xs, const double *Ls, const d
                 for (int q2 = q + 1; q2 < 8; q2++) xv[q2] -= xv[q] * Ls[(c0 + q2) + (c0 + q) * kPLD];
             }
 #pragma unroll
-            for (int q = 0; q < 8; q++) Xs[tid + (c0 + q) * kPLD] = xv[q];
+            for (int q = 0; q < 8; q++) Xs[row + (c0 + q) * kPLD] = xv[q];
         }
-        __syncthreads();
+        __syncwarp();
         // X[:, nbk] -= X[:, cb] L[nbk, cb]^T for nbk > cb: this warp's 16 rows, all
         // column blocks at once (static indices: loads batched ahead of the DMMAs)
         {
@@ -1074,8 +1077,9 @@ __device__ __forceinline__ void panel_trsm(double *Xs, const double *Ls, const d
                 }
             }
         }
-        __syncthreads();
+        __syncwarp();
     }
+    __syncthreads();   // callers read other warps' rows next
 }
 
 __device__ __forceinline__ void panel_publish(unsigned *flag, unsigned tag) {

@@ -223,7 +223,7 @@ struct Plan {
 constexpr int kTileM = 64, kTileN = 64;
 constexpr int kAsmCols = 16;
 constexpr int kTrsmRows = 128;
-constexpr int kSmallClasses = 4;
+constexpr int kSmallClasses = 5;
 constexpr int kSolveRows = 256;   // dataflow solve: rows per chunk (a multiple of the 64-column block)
 
 int build_plan(const Symbolic &S, const Options &opt, Plan &P);

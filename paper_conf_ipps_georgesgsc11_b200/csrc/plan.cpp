@@ -387,8 +387,10 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     }
     // small-front classes: f <= small_max/4, <= small_max/2, <= small_max
     // (<= 16 and <= 32: one warp per front; <= 64 and <= small_max: one CTA per front)
+    // (+ <= 96 when small_max > 96: 74 KB of shared memory, 3 CTAs / SM instead of
+    // the 1 that a 128-order front's 132 KB allows; c2 has ~4k such fronts per level)
     P.small_class_fmax = {std::min(16, P.small_max), std::min(32, P.small_max), std::min(64, P.small_max),
-                          P.small_max};
+                          std::min(96, P.small_max), P.small_max};
     // kernel variant per front: the learned selector y(x) = argmax_j x . theta_j over
     // the feasible classes (Eq. 5), a forced class, or the default
     // front-order thresholds (the analogue of the paper's baseline P_BH, L401).

@@ -134,13 +134,18 @@ def predict(theta: np.ndarray, X: np.ndarray, mask: np.ndarray) -> np.ndarray:
 
 def baseline_class(m, k, small_max: int = 128) -> np.ndarray:
     """The default front-order thresholds of plan.cpp (the analogue of the paper's
-    baseline hybrid P_BH): warp16 / warp32 / cta64 / cta128 / tiled."""
+    baseline hybrid P_BH): size classes f <= 16 / 32 / 64 / 96 /
+    small_max (each capped at small_max), each run by the first variant whose
+    order bound covers the class bound; larger fronts tiled."""
     f = np.asarray(m) + np.asarray(k)
-    out = np.full(f.shape, 6)
-    out[f <= small_max] = 4
-    out[f <= 64] = 2
-    out[f <= 32] = 1
-    out[f <= 16] = 0
+    out = np.full(f.shape, len(VARIANT_FMAX) - 1)
+
+    def cls(bound):
+        return next(j for j, fm in enumerate(VARIANT_FMAX) if fm == 0 or bound <= fm)
+
+    for bound in sorted({small_max, min(96, small_max), min(64, small_max), min(32, small_max),
+                         min(16, small_max)}, reverse=True):
+        out[f <= bound] = cls(bound)
     return out
 
 
