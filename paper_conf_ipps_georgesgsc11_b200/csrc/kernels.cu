@@ -703,7 +703,17 @@ void launch_leaf(const DevPlan &d, const int32_t *fronts, int npotrf, const int3
 // factorization of the top fronts.
 constexpr int kPanelThreads = 128;
 constexpr int kPLD = 68;   // 64-row tiles in shared memory: stride = 4 mod 16 (conflict-free fragments), even (16-byte cp.async)
-constexpr int kPanelRingWords = 3 * 16 * (2 * kPLD);   // 3-stage cp.async ring of 16-wide A / B slices
+#ifndef MF_PANEL_STAGES
+#define MF_PANEL_STAGES 2
+#endif
+#ifndef MF_PANEL_MINB
+#define MF_PANEL_MINB 3
+#endif
+// 2-stage cp.async ring of 16-wide A / B slices: 70 KB of shared memory and <= 168
+// registers give 3 CTAs / SM (3 stages: 87.5 KB, 255 registers, 2 CTAs / SM) --
+// the many-front levels' panels are throughput-bound on their non-band tasks
+constexpr int kPanelStages = MF_PANEL_STAGES;
+constexpr int kPanelRingWords = kPanelStages * 16 * (2 * kPLD);
 constexpr size_t kPanelSmem = (size_t)(kPanelRingWords + 64 * kPLD + 64) * sizeof(double);
 static_assert(64 * kPLD <= kPanelRingWords, "the L_bb tile aliases the staging ring");
 
@@ -730,7 +740,7 @@ __device__ __forceinline__ void panel_mark(int ev) {
 // rows >= arows / brows read as zero.  K is a multiple of 16.
 __device__ __forceinline__ void panel_tile_mma(double (&acc)[4][4][2], double *ring, const double *__restrict__ Pn,
                                                int ld, int ra0, int arows, int rb0, int brows, int kc0, int K) {
-    constexpr int BK = 16, STAGES = 3, STW = BK * 2 * kPLD;
+    constexpr int BK = 16, STAGES = kPanelStages, STW = BK * 2 * kPLD;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int wm = warp & 1, wn = warp >> 1, gq = lane >> 2, tq = lane & 3;
     const int rr = 2 * lane, pt = warp;   // staging slot: row pair rr, k offsets pt + 4 i
@@ -1088,7 +1098,7 @@ __device__ __forceinline__ void panel_publish(unsigned *flag, unsigned tag) {
     if (threadIdx.x == 0) asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(flag), "r"(tag) : "memory");
 }
 
-__global__ void __launch_bounds__(kPanelThreads, 2) k_panel(DevPlan d, const int32_t *__restrict__ tasks, int j0,
+__global__ void __launch_bounds__(kPanelThreads, MF_PANEL_MINB) k_panel(DevPlan d, const int32_t *__restrict__ tasks, int j0,
                                                              int nbk) {
     extern __shared__ __align__(16) double psm[];
     double *ring = psm;                         // accumulate staging; the L_bb tile afterwards
