@@ -79,8 +79,10 @@ int main(int argc, char **argv) {
     std::vector<double> ref1;
     run<UpdCfg<64, 64, 16, 3, 2, 2, 4>>("64x64 bk16 s3 w2x2 m4", Lshift, U, M, N, K, ld, ref);
     run<UpdCfg<64, 64, 16, 3, 2, 2, 4>, true>("BULK 64x64 bk16 s3 w2x2 m4", Lshift, U, M, N, K, ld, ref);
-    run<UpdCfg<64, 64, 8, 6, 2, 2, 4>, true>("BULK 64x64 bk8 s6 w2x2 m4", Lshift, U, M, N, K, ld, ref);
-    run<UpdCfg<64, 64, 8, 5, 2, 2, 4>, true>("BULK 64x64 bk8 s5 w2x2 m4", Lshift, U, M, N, K, ld, ref);
+    run<UpdCfg<128, 64, 16, 3, 4, 2, 2>, true>("BULK 128x64 bk16 s3 w4x2 m2", Lshift, U, M, N, K, ld, ref);
+    run<UpdCfg<128, 64, 16, 4, 4, 2, 2>, true>("BULK 128x64 bk16 s4 w4x2 m2", Lshift, U, M, N, K, ld, ref);
+    run<UpdCfg<64, 128, 16, 4, 2, 4, 2>, true>("BULK 64x128 bk16 s4 w2x4 m2", Lshift, U, M, N, K, ld, ref);
+    run<UpdCfg<128, 128, 16, 3, 4, 4, 1>, true>("BULK 128x128 bk16 s3 w4x4 m1", Lshift, U, M, N, K, ld, ref);
     run<UpdCfg<64, 64, 32, 2, 2, 2, 3>, true>("BULK 64x64 bk32 s2 w2x2 m3", Lshift, U, M, N, K, ld, ref);
     run<UpdCfg<64, 64, 16, 4, 2, 2, 3>, true>("BULK 64x64 bk16 s4 w2x2 m3", Lshift, U, M, N, K, ld, ref);
     run<UpdCfg<128, 64, 16, 3, 2, 2, 2>, true>("BULK 128x64 bk16 s3 w2x2 (64x32) m2", Lshift, U, M, N, K, ld, ref);
