@@ -502,7 +502,7 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
                 case KC_TRSM: launch_trsm_panel(d, c->d_trsm + 2 * L.off, L.count, L.param, P.w, st); break;
                 case KC_UPDATE:   // long-K launches of many waves take the bulk-copy pipeline
                     launch_update(d, c->d_probs, c->d_tiles + L.off, L.count,
-                                  L.count >= kBulkMinTiles && L.flops >= kBulkMinK * 2.0 * kTileM * kTileN * L.count, st);
+                                  L.count > 0 ? L.flops / (2.0 * kTileM * kTileN * L.count) : 0.0, st);
                     break;
                 case KC_PANEL: launch_panel(d, c->d_panel + 2 * L.off, L.count, L.param, (int)L.count2, st); break;
                 case KC_LEAF:

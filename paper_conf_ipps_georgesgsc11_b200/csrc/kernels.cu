@@ -1236,22 +1236,38 @@ void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, in
 // cp.async (33.2 TF/s on M=N=8192, K=4096) or, for launches of many long-K waves,
 // by the mbarrier + bulk-copy pipeline (33.8 TF/s there)
 using UpdProd = UpdCfg<kTileM, kTileN, 16, 3, 2, 2, 4>;
+// short-K launches: 2 stages (35 KB), 96 registers -> 5 CTAs / SM (20 warps) for
+// more loads in flight on the latency-bound C gather and U store
+using UpdLowK = UpdCfg<kTileM, kTileN, 16, 2, 2, 2, 5>;
 
-void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, bool bulk,
+void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, double kavg,
                    cudaStream_t st) {
     if (ntiles <= 0) return;   // attributes were set by kernels_init()
     const UpdGather gv{d.child_ptr, d.child_list, d.sn_k, d.sn_f, d.U_off, d.relmap_ptr, d.relmap, d.ea_qs};
-    // MF_UPD_BULK (A/B checks): 0 = cp.async everywhere, 1 = bulk everywhere; unset = per launch
+    // MF_UPD_BULK / MF_UPD_LOWK (A/B checks): 0 = never, 1 = every launch; unset = per launch
     static const int mode = [] {
         const char *e = getenv("MF_UPD_BULK");
         return e ? atoi(e) : -1;
     }();
+    static const int lowk_mode = [] {
+        const char *e = getenv("MF_UPD_LOWK");
+        return e ? atoi(e) : -1;
+    }();
+    bool bulk = ntiles >= kBulkMinTiles && kavg >= kBulkMinK;
     if (mode >= 0) bulk = mode == 1;
-#define MF_UPD_LAUNCH(V) k_update_t<UpdProd, V><<<(unsigned)ntiles, UpdProd::NT, UpdProd::SMEM, st>>>(d.L, d.U, probs, tiles, gv)
+    static const double lowk_max = [] {   // MF_UPD_LOWK_MAX: tuning override of kLowKMax
+        const char *e = getenv("MF_UPD_LOWK_MAX");
+        return e ? atof(e) : kLowKMax;
+    }();
+    bool lowk = !bulk && kavg < lowk_max;
+    if (lowk_mode >= 0) lowk = !bulk && lowk_mode == 1;
+#define MF_UPD_LAUNCH(C, V) k_update_t<C, V><<<(unsigned)ntiles, C::NT, C::SMEM, st>>>(d.L, d.U, probs, tiles, gv)
     if (bulk)
-        MF_UPD_LAUNCH(true);
+        MF_UPD_LAUNCH(UpdProd, true);
+    else if (lowk)
+        MF_UPD_LAUNCH(UpdLowK, false);
     else
-        MF_UPD_LAUNCH(false);
+        MF_UPD_LAUNCH(UpdProd, false);
 #undef MF_UPD_LAUNCH
 }
 
@@ -1273,6 +1289,9 @@ int kernels_init() {
         e = cudaFuncSetAttribute(k_update_t<UpdProd, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)UpdProd::SMEM);
     for (auto fn : {k_update_t<UpdProd, true>})
         if (e == cudaSuccess) e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)UpdProd::SMEM);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_update_t<UpdLowK, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)UpdLowK::SMEM);
     return e == cudaSuccess ? 0 : -1;
 }
 

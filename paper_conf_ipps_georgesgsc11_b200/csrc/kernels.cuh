@@ -44,12 +44,15 @@ void launch_leaf(const DevPlan &d, const int32_t *fronts, int npotrf, const int3
 void launch_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int nbk, cudaStream_t st);
 void launch_potrf_diag(const DevPlan &d, const int32_t *fronts, int count, int j0, int w, cudaStream_t st);
 void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, cudaStream_t st);
-// bulk = use the mbarrier + bulk-copy staging (pays off on many waves of long-K
-// tiles: c5 -4 ms; on short or few-wave launches the cp.async pipeline is faster,
-// measured per launch with tools/level_breakdown.py, MF_UPD_BULK=0/1)
+// kavg = the launch's average inner dimension.  Variant per launch (measured per
+// launch with tools/level_breakdown.py and MF_UPD_BULK / MF_UPD_LOWK = 0/1):
+//  * many waves of long-K tiles: mbarrier + bulk-copy staging (c5 -4 ms);
+//  * short K (latency-bound on the C gather / store): 2-stage ring, 5 CTAs/SM;
+//  * otherwise the 3-stage cp.async pipeline, 4 CTAs/SM.
 constexpr int64_t kBulkMinTiles = 4 * 592;   // 4 waves of 148 SMs x 4 CTAs
-constexpr double kBulkMinK = 512;            // average inner dimension of the launch's tiles
-void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, bool bulk,
+constexpr double kBulkMinK = 512;
+constexpr double kLowKMax = 128;
+void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, double kavg,
                    cudaStream_t st);
 void launch_permute_in(const DevPlan &d, const double *b, double *y, int64_t n, cudaStream_t st);
 void launch_permute_out(const DevPlan &d, const double *xf, double *x, int64_t n, cudaStream_t st);
