@@ -51,7 +51,7 @@ void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, in
 //  * otherwise the 3-stage cp.async pipeline, 4 CTAs/SM.
 constexpr int64_t kBulkMinTiles = 4 * 592;   // 4 waves of 148 SMs x 4 CTAs
 constexpr double kBulkMinK = 512;
-constexpr double kLowKMax = 128;
+constexpr double kLowKMax = 256;
 void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, double kavg,
                    cudaStream_t st);
 void launch_permute_in(const DevPlan &d, const double *b, double *y, int64_t n, cudaStream_t st);
