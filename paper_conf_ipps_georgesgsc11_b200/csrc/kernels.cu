@@ -1038,18 +1038,34 @@ __device__ __forceinline__ void panel_potrf_dmma(const DevPlan &d, double *A, do
 }
 
 // X <- X L^-T for the 64 rows of Xs over wb columns; Ls = the wb x wb lower factor
-// (identity-padded to a multiple of 8), inv = 1 / diag.  Each warp owns 16 rows:
-// per 8-column block, 16 of its lanes solve their rows over the block
-// (substitution), then the warp applies the block to its rows' remaining columns
-// with DMMA -- warps never share rows, so only warp-level synchronisation (the
-// 16 CTA barriers of a row-per-thread substitution cost ~half of the trsm).
+// (identity-padded to a multiple of 8), inv = 1 / diag.  Each warp owns 16 rows and
+// keeps them in registers as DMMA accumulators: per 8-column block, the block goes
+// to shared memory, 16 lanes solve their rows over it (substitution, written back),
+// and the warp applies it to the remaining column blocks with DMMA into the
+// registers -- no shared-memory round trip per block update, so the updates of
+// different blocks pipeline (same operations, same order per element as a
+// shared-memory-resident update).  Xs holds the solved X on return.
 __device__ __forceinline__ void panel_trsm(double *Xs, const double *Ls, const double *inv, int wb) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, gq = lane >> 2, tq = lane & 3;
     const int ncb = (wb + 7) / 8;
     const int row = warp * 16 + (lane & 15);
-#pragma unroll 1
-    for (int cb = 0; cb < ncb; cb++) {
+    double acc[2][8][2];
+#pragma unroll
+    for (int mb = 0; mb < 2; mb++)
+#pragma unroll
+        for (int nb = 0; nb < 8; nb++)
+#pragma unroll
+            for (int e = 0; e < 2; e++) acc[mb][nb][e] = Xs[warp * 16 + mb * 8 + gq + (nb * 8 + 2 * tq + e) * kPLD];
+#pragma unroll
+    for (int cb = 0; cb < 8; cb++) {
+        if (cb >= ncb) break;
         const int c0 = cb * 8;
+        // block cb of this warp's rows (updated by every earlier block) -> shared memory
+#pragma unroll
+        for (int mb = 0; mb < 2; mb++)
+#pragma unroll
+            for (int e = 0; e < 2; e++) Xs[warp * 16 + mb * 8 + gq + (c0 + 2 * tq + e) * kPLD] = acc[mb][cb][e];
+        __syncwarp();
         if (lane < 16) {
             double xv[8];
 #pragma unroll
@@ -1064,30 +1080,22 @@ __device__ __forceinline__ void panel_trsm(double *Xs, const double *Ls, const d
             for (int q = 0; q < 8; q++) Xs[row + (c0 + q) * kPLD] = xv[q];
         }
         __syncwarp();
-        // X[:, nbk] -= X[:, cb] L[nbk, cb]^T for nbk > cb: this warp's 16 rows, all
-        // column blocks at once (static indices: loads batched ahead of the DMMAs)
-        {
-            double av[2][2];
+        // X[:, nbk] -= X[:, cb] L[nbk, cb]^T for nbk > cb, in registers
+        double av[2][2];
 #pragma unroll
-            for (int mb = 0; mb < 2; mb++)
+        for (int mb = 0; mb < 2; mb++)
 #pragma unroll
-                for (int kk = 0; kk < 2; kk++) av[mb][kk] = -Xs[warp * 16 + mb * 8 + gq + (c0 + kk * 4 + tq) * kPLD];
+            for (int kk = 0; kk < 2; kk++) av[mb][kk] = -Xs[warp * 16 + mb * 8 + gq + (c0 + kk * 4 + tq) * kPLD];
 #pragma unroll
-            for (int nbk = 1; nbk < 8; nbk++) {
-                if (nbk <= cb || nbk >= ncb) continue;
-                const double b0 = Ls[(nbk * 8 + gq) + (c0 + tq) * kPLD], b1 = Ls[(nbk * 8 + gq) + (c0 + 4 + tq) * kPLD];
+        for (int nbk = 1; nbk < 8; nbk++) {
+            if (nbk <= cb || nbk >= ncb) continue;
+            const double b0 = Ls[(nbk * 8 + gq) + (c0 + tq) * kPLD], b1 = Ls[(nbk * 8 + gq) + (c0 + 4 + tq) * kPLD];
 #pragma unroll
-                for (int mb = 0; mb < 2; mb++) {
-                    double *xr = Xs + warp * 16 + mb * 8 + gq + (nbk * 8 + 2 * tq) * kPLD;
-                    double acc0 = xr[0], acc1 = xr[kPLD];
-                    dmma(acc0, acc1, av[mb][0], b0);
-                    dmma(acc0, acc1, av[mb][1], b1);
-                    xr[0] = acc0;
-                    xr[kPLD] = acc1;
-                }
+            for (int mb = 0; mb < 2; mb++) {
+                dmma(acc[mb][nbk][0], acc[mb][nbk][1], av[mb][0], b0);
+                dmma(acc[mb][nbk][0], acc[mb][nbk][1], av[mb][1], b1);
             }
         }
-        __syncwarp();
     }
     __syncthreads();   // callers read other warps' rows next
 }
