@@ -1182,8 +1182,9 @@ __global__ void __launch_bounds__(kPanelThreads, MF_PANEL_MINB) k_panel(DevPlan 
             if (i < rows && j < wb) Pn[(r0 + i) + (int64_t)(cb0 + j) * ld] = Xs[i + j * kPLD];
         }
         if (band) {
-            panel_publish(F + panel_tri(c, b), tag);   // X(c,b) is stored: band tile final
-            // the row's own product: dacc -= X(c,b) X(c,b)^T (b < c < nb, so wb = 64)
+            // the row's own product first: dacc -= X(c,b) X(c,b)^T (b < c < nb, so wb =
+            // 64), from shared memory, while the stores above drain -- so the fence of
+            // the publish below no longer waits for them (3.6 us -> the product's 2.4)
             const double *Xg = Xs + gq;
 #pragma unroll 2
             for (int kk = 0; kk < 16; kk++) {
@@ -1195,7 +1196,9 @@ __global__ void __launch_bounds__(kPanelThreads, MF_PANEL_MINB) k_panel(DevPlan 
 #pragma unroll
                 for (int t = 0; t < 9; t++) dmma(dacc[t][0], dacc[t][1], t <= warp ? a0 : a1, bj[t]);
             }
-            __syncthreads();   // Xs / ring are rewritten by the next step
+            PANEL_MARK(31);
+            panel_publish(F + panel_tri(c, b), tag);   // X(c,b) is stored: band tile final (+ CTA barrier:
+                                                       // Xs / ring are rewritten by the next step)
             PANEL_MARK(6 + 6 * b);
         } else {
             __syncthreads();   // Xs / ring are rewritten by the next step

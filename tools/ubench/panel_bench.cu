@@ -65,7 +65,7 @@ int main(int argc, char **argv) {
     auto show = [&](int c) {
         printf("task %4d:", c);
         printf(" [potrf clk a %llu b %llu c %llu]", tr[c][25], tr[c][26], tr[c][27]);
-        for (int e = 0; e < 31; e++)
+        for (int e = 0; e < 32; e++)
             if (e < 25 || e > 27) if (tr[c][e] >= t0 && tr[c][e] - t0 < 10000000ull) printf(" %d:%.1f", e, (tr[c][e] - t0) / 1e3);
         printf("\n");
     };
