@@ -343,8 +343,11 @@ def main():
         "config": {"workload": c["desc"] + f" [{args.config}]", "n": A.n, "nnz_lower": A.nnz,
                    "flops_true": flops, "flops_exec": float(info["flops_exec"]), "nsuper": info["nsuper"],
                    "max_front": info["max_front"],
-                   "parallelism": (f"subtree-to-GPU x{world}, top supernodes on rank 0 (NCCL send/recv)"
+                   "parallelism": (f"subtree-to-GPU x{world}, top fronts replicated and factored cooperatively "
+                                   "(NCCL broadcasts)"
                                    if world > 1 else f"1 GPU, {info['nbranch']} concurrent subtree branches"),
+                   "variant_selector": ("learned (PAPER Eqs. 3-5, " + os.path.basename(S.variant_model) + ")"
+                                        if S.variant_model else "front-order thresholds"),
                    "l2": "no flush: working set (L = %.1f GB) >> 126 MB L2" % (info["panel_words"] * 8 / 1e9)},
         "clocks": clocks,
         "mapping": mapping,

@@ -156,7 +156,11 @@ class Solver:
     def __init__(self, amalgamate: bool = True, small_front_max: int | None = None, panel_w: int | None = None,
                  device: int = -1, stream: int | None = None, host_only: bool = False,
                  nranks: int = 1, rank: int = 0, exchange=None, split_all: bool = False,
-                 nbranch: int | None = None, fuse_ea: bool | None = None, lookahead: bool | None = None):
+                 nbranch: int | None = None, fuse_ea: bool | None = None, lookahead: bool | None = None,
+                 variant_model="auto"):
+        """variant_model: "auto" = the fitted kernel-variant selector packaged with the
+        binding (selector.MODEL_PATH, Eqs. 3-5 fitted to B200 timings) when
+        present, None = libmf's fixed front-order thresholds, or a theta array."""
         o = Options()
         lib.mf_default_options(ctypes.byref(o))
         o.amalgamate = int(amalgamate)
@@ -184,6 +188,16 @@ class Solver:
         self.n = None
         self.nranks, self.rank = nranks, rank
         self._xcb = None
+        self.variant_model = None
+        if isinstance(variant_model, str) and variant_model == "auto":
+            from . import selector as _sel   # (lazy: selector imports this module)
+            th = _sel.load_model()
+            if th is not None:
+                self.set_variant_model(th)
+                self.variant_model = _sel.MODEL_PATH
+        elif variant_model is not None:
+            self.set_variant_model(variant_model)
+            self.variant_model = "caller theta"
         if exchange is not None:
             self.set_exchange(exchange)
 

@@ -192,3 +192,30 @@ def test_gpu_variants_parity(mode):
     assert worst <= 1e-10, (mode, worst, used)
     if mode.startswith("random"):
         assert len(used) >= 2, used
+
+
+def test_packaged_model_is_the_default_and_feasible():
+    """The fitted selector shipped with the binding (variant_model.json, fitted by
+    tools/fit_variant_model.py --relative on B200 timings) is loaded by default and
+    every class it picks can run its front (order bound >= f)."""
+    import paper_conf_ipps_georgesgsc11_b200 as mf
+    from paper_conf_ipps_georgesgsc11_b200 import selector as sel
+    th = sel.load_model()
+    assert th is not None and th.shape == (9, R)
+    A, p = grid("27pt", (12, 12, 12))
+    S = mf.Solver(host_only=True)
+    assert S.variant_model == sel.MODEL_PATH
+    S.analyze(A.n, A.colptr, A.rowind, p)
+    sn = S.supernodes()
+    k = np.diff(sn["sn_first"])
+    f = np.diff(sn["sn_rowptr"])
+    var = S.variants()
+    feas = sel.feasible(f - k, k)
+    assert feas[np.arange(len(var)), var].all()
+    # Eq. 5 over the feasible classes, as the planner evaluates it
+    np.testing.assert_array_equal(var, sel.predict(th, sel.features(f - k, k), feas))
+    S.close()
+    S = mf.Solver(host_only=True, variant_model=None)
+    S.analyze(A.n, A.colptr, A.rowind, p)
+    np.testing.assert_array_equal(S.variants(), sel.baseline_class(f - k, k))
+    S.close()

@@ -31,7 +31,11 @@ def main():
     d, m, k, T = load(path)
     X = sel.features(m, k)
     F = sel.feasible(m, k) & np.isfinite(T)
-    th = sel.fit(X, np.where(F, T, 0.0), F, reg=1e-6, verbose=False)
+    # --relative: each shape's times divided by its fastest variant (R5): the
+    # grid is not a workload sample, and in absolute time the cheap shapes (175k tiny
+    # fronts in c2) would not count at all
+    Tfit = T / np.nanmin(np.where(F, T, np.nan), axis=1, keepdims=True) if "--relative" in sys.argv else T
+    th = sel.fit(X, np.where(F, Tfit, 0.0), F, reg=1e-6, verbose=False)
     pm = sel.predict(th, X, F)
     pb = sel.baseline_class(m, k)
     pi = np.where(F, T, np.inf).argmin(axis=1)

@@ -15,7 +15,11 @@ v = torch.from_numpy(A.values).cuda()
 for val in vals.split(","):
     kw = {opt: int(val)}
     kw.update({k: int(x) for k, x in extra.items()})
+    model = kw.pop("model", 0)     # model=1: the fitted variant selector (selector.load_model)
     S = mf.Solver(**kw)
+    if model:
+        from paper_conf_ipps_georgesgsc11_b200 import selector as sel
+        S.set_variant_model(sel.load_model())
     S.analyze(A.n, A.colptr, A.rowind, p)
     for _ in range(3):
         S.factor(v)
