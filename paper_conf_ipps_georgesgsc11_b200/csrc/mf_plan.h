@@ -128,7 +128,7 @@ enum KernelClass : int32_t {
 constexpr int kFuseLeafMaxFronts = 8;
 // Dataflow panel (KC_PANEL, w = 64 only): base case of the recursive blocked
 // factorization; per front kPanelFlags epoch-tagged flags (band tiles + diagonal tiles).
-constexpr int kPanelMaxBlocks = 4;
+constexpr int kPanelMaxBlocks = 8;   // 8 x 64 columns per panel launch (A/B: 4 -> 8 c5 -0.6%, c3 -1.6%, c4 -1%; 16 worse on c2/c3)
 constexpr int kPanelFlags = kPanelMaxBlocks * (kPanelMaxBlocks + 1) / 2;
 
 // One transfer of a multi-GPU exchange point, relative to the L or U arena.
