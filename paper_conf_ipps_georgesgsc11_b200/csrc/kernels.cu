@@ -1264,7 +1264,15 @@ void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tile
         const char *e = getenv("MF_UPD_LOWK");
         return e ? atoi(e) : -1;
     }();
-    bool bulk = ntiles >= kBulkMinTiles && kavg >= kBulkMinK;
+    static const double bulk_min_tiles = [] {   // MF_UPD_BULK_TILES / MF_UPD_BULK_K: tuning overrides
+        const char *e = getenv("MF_UPD_BULK_TILES");
+        return e ? atof(e) : (double)kBulkMinTiles;
+    }();
+    static const double bulk_min_k = [] {
+        const char *e = getenv("MF_UPD_BULK_K");
+        return e ? atof(e) : kBulkMinK;
+    }();
+    bool bulk = (double)ntiles >= bulk_min_tiles && kavg >= bulk_min_k;
     if (mode >= 0) bulk = mode == 1;
     static const double lowk_max = [] {   // MF_UPD_LOWK_MAX: tuning override of kLowKMax
         const char *e = getenv("MF_UPD_LOWK_MAX");
