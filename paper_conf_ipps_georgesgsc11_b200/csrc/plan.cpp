@@ -15,6 +15,8 @@
 //   * its update matrix U^s: m_s x m_s column-major (lower triangle used) in the
 //     U arena, written by the F-U of s and read by the extend-add of its parent.
 #include <algorithm>
+#include <cstdlib>
+#include <map>
 #include <cmath>
 #include <functional>
 #include <numeric>
@@ -292,6 +294,98 @@ static void assign_branches(Plan &P, const std::vector<double> &front_load, int 
     P.nbranch = nb;
 }
 
+// U-arena liveness (single GPU): U^s is written at front s's level and read only
+// by its parent (assembly of the panel columns and the syrk prologue's gather, or
+// the parent's small-front kernel) at the parent's level, in the same stream or,
+// for a branch root, in the top pass after the branches joined.  Slots are
+// therefore recycled level by level with a first-fit allocator: each concurrent
+// branch in its own region (branches run concurrently), the top pass over the
+// whole arena minus the frontier roots' still-live slots.  Only offsets change.
+static void plan_u_reuse(Plan &P) {
+    const int32_t ns = P.nsuper;
+    auto words = [&](int32_t s) -> int64_t {
+        const int64_t m = P.sn_f[s] - P.sn_k[s], w = m * m;
+        return w + (w & 1);
+    };
+    std::vector<int64_t> off(ns, -1);
+    std::map<int64_t, int64_t> freel;   // offset -> length
+    int64_t hw = 0;                     // high-water mark of the current allocator
+    auto alloc = [&](int64_t len) -> int64_t {
+        for (auto it = freel.begin(); it != freel.end(); ++it)
+            if (it->second >= len) {
+                const int64_t o = it->first, rem = it->second - len;
+                freel.erase(it);
+                if (rem) freel[o + len] = rem;
+                return o;
+            }
+        const int64_t o = hw;
+        hw += len;
+        return o;
+    };
+    auto release = [&](int64_t o, int64_t len) {
+        auto it = freel.emplace(o, len).first;
+        auto nx = std::next(it);
+        if (nx != freel.end() && it->first + it->second == nx->first) {
+            it->second += nx->second;
+            freel.erase(nx);
+        }
+        if (it != freel.begin()) {
+            auto pv = std::prev(it);
+            if (pv->first + pv->second == it->first) {
+                pv->second += it->second;
+                freel.erase(it);
+            }
+        }
+    };
+    auto run_group = [&](int32_t g) {
+        for (int32_t l = 0; l < P.nlevels; l++) {
+            for (int32_t q = P.level_ptr[l]; q < P.level_ptr[l + 1]; q++) {
+                const int32_t s = P.level_list[q];
+                if (P.branch[s] != g) continue;
+                off[s] = words(s) > 0 ? alloc(words(s)) : 0;
+            }
+            for (int32_t q = P.level_ptr[l]; q < P.level_ptr[l + 1]; q++) {   // children consumed at level l
+                const int32_t s = P.level_list[q];
+                if (P.branch[s] != g) continue;
+                for (int32_t c = P.child_ptr[s]; c < P.child_ptr[s + 1]; c++) {
+                    const int32_t ch = P.child_list[c];
+                    if (words(ch) > 0 && off[ch] >= 0) release(off[ch], words(ch));
+                }
+            }
+        }
+    };
+    int64_t total = 0;
+    std::vector<std::pair<int64_t, int64_t>> live;   // branch roots' slots, live into the top pass
+    for (int32_t b = 0; b < (P.nbranch > 1 ? P.nbranch : 0); b++) {
+        freel.clear();
+        hw = 0;
+        run_group(b);
+        for (int32_t s = 0; s < ns; s++)   // shift the branch's region behind the previous ones
+            if (P.branch[s] == b && off[s] >= 0 && words(s) > 0) off[s] += total;
+        total += hw;
+    }
+    // top pass (or everything, without branches): the whole arena is free except
+    // the slots of branch fronts whose parent is a top front
+    freel.clear();
+    for (int32_t s = 0; s < ns; s++)
+        if (P.branch[s] < 0)
+            for (int32_t c = P.child_ptr[s]; c < P.child_ptr[s + 1]; c++) {
+                const int32_t ch = P.child_list[c];
+                if (P.branch[ch] >= 0 && words(ch) > 0) live.emplace_back(off[ch], words(ch));
+            }
+    std::sort(live.begin(), live.end());
+    int64_t cur = 0;
+    for (auto &iv : live) {
+        if (iv.first > cur) freel[cur] = iv.first - cur;
+        cur = std::max(cur, iv.first + iv.second);
+    }
+    if (total > cur) freel[cur] = total - cur;
+    hw = total;
+    run_group(-1);
+    for (int32_t s = 0; s < ns; s++) P.U_off[s] = off[s] >= 0 ? off[s] : 0;
+    P.U_words = hw + 2;
+}
+
 int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     P = Plan();
     const int32_t ns = (int32_t)S.sn_parent.size();
@@ -490,6 +584,12 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         map_subtrees(P, front_load);
         if (P.nranks == 1) assign_branches(P, front_load, opt.nbranch);
         else P.branch.assign(ns, -1);
+    }
+    // U-slot recycling (single GPU; multi-GPU exchanges address the U arena by
+    // supernode and keep disjoint slots).  MF_U_REUSE=0 disables it (A/B checks).
+    {
+        const char *e = getenv("MF_U_REUSE");
+        if (P.nranks == 1 && (!e || atoi(e) != 0)) plan_u_reuse(P);
     }
     // Inclusion masks.  Local program: the supernodes of this rank's subtrees.  Top
     // program (multi-GPU): EVERY rank holds a replica of every top front; the

@@ -291,7 +291,7 @@ def test_bulk_staging_bit_identical(mf, kind, dims, sm):
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     out = []
     envs = [dict(MF_UPD_BULK="0", MF_UPD_LOWK="0"), dict(MF_UPD_BULK="1"), dict(MF_UPD_BULK="1"),
-            dict(MF_UPD_BULK="0", MF_UPD_LOWK="1"), {}]
+            dict(MF_UPD_BULK="0", MF_UPD_LOWK="1"), {}, dict(MF_U_REUSE="0")]   # + U slots not recycled
     for e in envs:
         r = subprocess.run([sys.executable, "-c", _BULK_CHILD, kind, ",".join(map(str, dims)), str(sm)], cwd=root,
                            env=dict(os.environ, **e), capture_output=True, text=True, timeout=600)
