@@ -10,11 +10,14 @@
 //
 // sm_100a has no f64 kind of tcgen05.mma (probe 1), so the FP64
 // tensor path is warp-level mma.sync.m8n8k4.f64 (SASS DMMA.8x8x4).  Operands are
-// staged by 16-byte cp.async (LDGSTS, zero-fill at the edges) into a
-// STAGES-deep shared-memory ring; each warp owns a TM x TN sub-tile whose
-// accumulators start from C (loaded while the first stages are in flight) and
-// accumulate C - A B^T directly (A fragments negated), so the epilogue is a
-// masked store.  Columns are 16-byte aligned (lda even) and every problem's
+// staged into a STAGES-deep shared-memory ring either by every thread's 16-byte
+// cp.async (LDGSTS, zero-fill at the edges; CTA barrier per k-tile) or -- the
+// BULK variant, for launches of many long-K waves -- by warp 0's cp.async.bulk
+// per operand column with full / empty mbarriers (no CTA barrier in the loop).
+// Each warp owns a TM x TN sub-tile whose accumulators start from C (loaded while
+// the first stages are in flight; for the syrk on U^s with the fused extend-add,
+// gathered from the children's U^c instead) and accumulate C - A B^T directly
+// (A fragments negated), so the epilogue is a masked store.  Columns are 16-byte aligned (lda even) and every problem's
 // first row is even: the planner shifts a problem whose first row is odd (the
 // syrk on U^n of a supernode with odd k) one row up, computes the extra leading
 // row / column of the shifted space and masks it out here (flag bit 1).
