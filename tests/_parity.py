@@ -1,0 +1,70 @@
+"""The parity metric of reading C11, shared by the GPU tests.
+
+rel_ij = |L_gpu,ij - L_ref,ij| / max(|L_ref,ij|, TAU * max_i |L_ref(:, j)|), max
+over the stored structure, must be <= TOL_L (north star: "max relative entry
+error of L versus the oracle <= 1e-10").
+
+TAU, the floor, is ONE constant for every config, derived from the long-double
+referee (tests/test_referee.py, oracle.dense_cholesky_longdouble): on Q1
+elasticity fronts (6^3..12^3) the fp64 oracle is within 5.2-7.4 u of the
+column max of the exact factor on every entry, the GPU factor likewise
+(u = 2^-53), so two correct fp64 factors may differ by up to 2 * 8 u * colmax =
+1.8e-15 * colmax on the ~3% of elasticity entries that are cancellation noise
+(down to 0 * colmax).  The smallest floor that keeps that rounding envelope
+inside 1e-10 is 1.8e-5 -> TAU = 2e-5.  The M-matrix stencils have no
+cancellation (all L off-diagonals share a sign), so for them the UNFLOORED
+relative error must ALSO be <= TOL_L (strictly tighter than any floor).
+Reported with every check: the floored max, the unfloored max over entries
+with L_ref != 0, and how many entries lie below the floor."""
+from __future__ import annotations
+
+import numpy as np
+
+TAU = 2e-5
+TOL_L = 1e-10
+U64 = 2.0 ** -53
+
+
+class ParityStats:
+    def __init__(self, tau: float = TAU):
+        self.tau = tau
+        self.floored = 0.0
+        self.unfloored = 0.0
+        self.below_floor = 0
+        self.entries = 0
+        self.ref_zero_gpu_nonzero = 0
+        self.pad_violations = 0
+        self.panels = 0
+        self.worst_panel = -1
+
+    def add(self, s: int, Pg: np.ndarray, Po: np.ndarray, m_matrix: bool = False) -> None:
+        """Compare one panel (f x k) of the GPU factor with the oracle's.  With
+        ``m_matrix`` (stencils: structural entries of L never cancel to 0) an
+        exact 0 in the oracle panel is amalgamation padding, which must be an
+        exact 0 on the GPU too (reading C10)."""
+        k = Po.shape[1]
+        if k == 0:
+            return
+        d = np.abs(Pg - Po)
+        a = np.abs(Po)
+        colmax = a.max(axis=0)
+        floor = self.tau * colmax[None, :]
+        den = np.maximum(a, floor)
+        den[den == 0] = 1.0
+        fl = float((d / den).max())
+        if fl > self.floored:
+            self.floored, self.worst_panel = fl, int(s)
+        nz = a > 0
+        if nz.any():
+            self.unfloored = max(self.unfloored, float((d[nz] / a[nz]).max()))
+        self.ref_zero_gpu_nonzero += int(np.count_nonzero(~nz & (Pg != 0)))
+        self.below_floor += int(np.count_nonzero(nz & (a < floor)))
+        self.entries += Po.size
+        self.panels += 1
+        if m_matrix:
+            self.pad_violations += int(np.count_nonzero(~nz & (Pg != 0)))
+
+    def report(self) -> dict:
+        return dict(panels=self.panels, entries=self.entries, tau=self.tau, floored_max=self.floored,
+                    unfloored_max=self.unfloored, below_floor=self.below_floor,
+                    ref_zero_gpu_nonzero=self.ref_zero_gpu_nonzero, worst_panel=self.worst_panel)

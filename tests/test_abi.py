@@ -114,3 +114,21 @@ def test_plan_memory_is_planned():
     inf = _check_symbolic(A, p)
     assert inf["panel_words"] >= inf["nnzL_stored"]
     assert inf["nlevels"] >= 1 and inf["max_front"] > 128
+
+
+def test_symbolic_postorder_hand_worked():
+    """The hand-worked non-postordered etree (tests/golden/postorder_example.json):
+    the product's symbolic layer relabels by the same DFS postorder."""
+    import json
+    from tests.test_oracle_symbolic import _postorder_case
+    e = json.load(open(os.path.join(ROOT, "tests", "golden", "postorder_example.json")))
+    S = mf.Solver(host_only=True)
+    A = _postorder_case(e)
+    S.analyze(A.n, A.colptr, A.rowind, np.arange(e["n"], dtype=np.int32))
+    np.testing.assert_array_equal(S.perm(), e["final_perm"])
+    np.testing.assert_array_equal(S.etree()[0], e["parent_final"])
+    q = np.array(e["relabel_q"], dtype=np.int32)
+    Aq = _postorder_case(e, q)
+    S.analyze(Aq.n, Aq.colptr, Aq.rowind, q)
+    np.testing.assert_array_equal(S.perm(), e["final_perm_with_q"])
+    _check_symbolic(Aq, q)

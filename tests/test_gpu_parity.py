@@ -2,7 +2,7 @@
 element by element, on seeded synthetic inputs.
 
 Tolerances (north star, BASELINE.json): max relative entry error of L vs the
-oracle <= 1e-10 under reading C11 (floor tau = 1e-6 of the column max);
+oracle <= 1e-10 under reading C11 (one floor, tests/_parity.py TAU);
 amalgamation padding exactly 0.0 (reading C10); backward error
 ||Ax - b||_inf / (||A||_inf ||x||_inf + ||b||_inf) <= 1e-12 (reading C12);
 manufactured integer factors bit-exact.
@@ -13,6 +13,7 @@ import pytest
 import oracle
 from workloads import grids as G
 from tests._grids import dense_from_rows, grid
+from tests._parity import TAU
 
 pytestmark = pytest.mark.gpu
 
@@ -28,7 +29,7 @@ def mf():
     return m
 
 
-def c11(Pg, Po, tau=1e-6):
+def c11(Pg, Po, tau=TAU):
     """Reading C11 floored relative error of one panel (columns = columns of L)."""
     colmax = np.abs(Po).max(axis=0)
     den = np.maximum(np.abs(Po), tau * colmax[None, :])
@@ -45,7 +46,7 @@ def factor_both(mf, A, perm, supernodes=None, **opts):
     return S, sym, panels
 
 
-def check_panels(S, sym, panels, exact=False, tau=1e-6):
+def check_panels(S, sym, panels, exact=False, tau=TAU):
     worst = 0.0
     for s, Po in panels.items():
         f, k = Po.shape
@@ -333,45 +334,3 @@ def test_degenerate_inputs(mf):
     assert S.solve(np.zeros(0)).size == 0
 
 
-@pytest.mark.parametrize("name", ["c5", "c4", "c3", "c2"])
-def test_full_size_sampled(mf, name):
-    """BASELINE config at full size, in bench.py's launch configuration: sampled
-    whole subtrees vs the oracle (subset factorization), closed-form log det and
-    the backward error of a solve."""
-    c = G.CONFIGS[name]
-    A, p = G.make_config(c["kind"], c["N"])
-    S = mf.Solver()
-    S.analyze(A.n, A.colptr, A.rowind, p)
-    S.factor(A.values)
-    sym = oracle.symbolic(A, p)
-    # sample: three subtrees of different heights (leaf region, mid-level, a depth-4 subtree)
-    ch = sym.children()
-    sizes = np.zeros(sym.nsuper, dtype=np.int64)
-    for s in range(sym.nsuper):
-        sizes[s] = 1 + sum(sizes[q] for q in ch[s])
-    picks = [int(np.argmax(np.where(sizes < lim, sizes, 0))) for lim in (40, 400, 3000)]
-    subset = set()
-    for r in picks:
-        stack = [r]
-        while stack:
-            v = stack.pop(); subset.add(v); stack.extend(ch[v])
-    panels = oracle.factor(A, sym, subset=subset)
-    # Reading C11: elasticity is not an M-matrix; its cancellation-noise entries
-    # (down to ~1e-18 of the column max) agree only to fp64 roundoff of the
-    # column max (observed 4.7e-16 * colmax in c4's 7728 x 1875 fronts), so the
-    # relative floor is 1e-4 of the column max there (1e-6 for the stencils).
-    check_panels(S, sym, panels, tau=1e-4 if c["kind"] == "elast" else 1e-6)
-    # closed-form log det of the Laplacian stencils (Kronecker-sum eigenvalues)
-    N = c["N"]
-    th = np.arange(1, N + 1) * np.pi / (N + 1)
-    t1 = 1 + 2 * np.cos(th)
-    k1 = 4 * np.sin(th / 2) ** 2
-    lam = {"27pt": lambda: 27 - t1[:, None, None] * t1[None, :, None] * t1[None, None, :],
-           "9pt": lambda: 9 - t1[:, None] * t1[None, :],
-           "7pt": lambda: k1[:, None, None] + k1[None, :, None] + k1[None, None, :]}.get(c["kind"])
-    if lam is not None:
-        ld = float(np.sum(np.log(lam())))
-        assert 2 * np.sum(np.log(S.diag())) == pytest.approx(ld, rel=1e-12)
-    b = spmv(A, G.rhs(A.n, 0))
-    x = S.solve(b)
-    assert backward_error(A, x, b) <= TOL_BE

@@ -111,7 +111,59 @@ def check_against_brute(A, perm):
     # the postorder: every node's parent comes later, and subtrees are contiguous
     p = sym.parent
     assert all(p[j] == -1 or p[j] > j for j in range(A.n))
+    assert_subtrees_contiguous(p)
     return sym
+
+
+def assert_subtrees_contiguous(parent):
+    """A postorder numbers every subtree as a contiguous range ending at its
+    root: the descendants of j are exactly j - size(j) + 1 .. j."""
+    n = len(parent)
+    size = np.ones(n, dtype=np.int64)
+    lo = np.arange(n, dtype=np.int64)          # smallest label in the subtree of j
+    for j in range(n):                         # children before parents (p[j] > j)
+        q = int(parent[j])
+        if q >= 0:
+            size[q] += size[j]
+            lo[q] = min(lo[q], lo[j])
+    assert (lo == np.arange(n) - size + 1).all()
+
+
+def _postorder_case(e, q=None):
+    n = e["n"]
+    M = np.eye(n) * e["diag"]
+    for i, j in e["offdiag_lower"]:
+        M[i, j] = M[j, i] = e["offdiag_value"]
+    if q is not None:                           # relabel: A'(q[i], q[j]) = A(i, j)
+        Mq = np.zeros_like(M)
+        Mq[np.ix_(q, q)] = M
+        M = Mq
+    return dense_from_rows(M.tolist())
+
+
+def test_postorder_hand_worked():
+    """A natural order whose etree is NOT a postorder (tests/golden/postorder_example.json,
+    hand-worked from PAPER.md L27 and reading C5): the oracle must relabel by the
+    DFS postorder (children ascending) and compose it with the input perm."""
+    e = json.load(open(os.path.join(GOLD, "postorder_example.json")))
+    A = _postorder_case(e)
+    sym = oracle.symbolic(A, None)
+    assert not sym.postorder_was_identity
+    np.testing.assert_array_equal(sym.perm, e["final_perm"])
+    np.testing.assert_array_equal(sym.parent, e["parent_final"])
+    np.testing.assert_array_equal(sym.cc, e["cc_final"])
+    assert_subtrees_contiguous(sym.parent)
+    # natural-order etree by brute force is the hand-derived one (not a postorder)
+    st = brute_structure(A, np.arange(e["n"]))
+    assert [int(s[1]) if s.size > 1 else -1 for s in st] == e["etree_natural"]
+    with pytest.raises(AssertionError):
+        assert_subtrees_contiguous(e["etree_natural"])
+    # the same matrix relabeled by q, with perm = q: final perm = q composed with the postorder
+    q = np.array(e["relabel_q"], dtype=np.int32)
+    Aq = _postorder_case(e, q)
+    symq = oracle.symbolic(Aq, q)
+    np.testing.assert_array_equal(symq.perm, e["final_perm_with_q"])
+    np.testing.assert_array_equal(symq.parent, e["parent_final"])
 
 
 def test_appendix_c_examples():
@@ -204,3 +256,33 @@ def test_invalid_inputs_rejected():
     bad.rowind[3] = A.n + 5
     with pytest.raises(ValueError):
         oracle.symbolic(bad, None)
+
+
+def _front_ops_by_loops(k, m):
+    """Count the flops of the unblocked F-U loops on a k-pivot, m-row front one
+    operation at a time (one FMA = 2, each sqrt / division = 1):
+    potrf column algorithm, trsm by substitution, syrk on the lower triangle."""
+    fl = 0
+    for j in range(k):                       # potrf
+        fl += 1 + (k - 1 - j)                # sqrt, divisions below the pivot
+        fl += 2 * sum(k - b for b in range(j + 1, k))   # rank-1 update of the lower trailing block
+    for _ in range(m):                       # trsm: each row x_j = (x_j - sum x_p L_jp) / L_jj
+        fl += sum(1 + 2 * j for j in range(k))
+    fl += 2 * k * (m * (m + 1) // 2)         # syrk: lower triangle incl. diagonal, k FMAs each
+    return fl
+
+
+@pytest.mark.parametrize("k,m", [(1, 0), (1, 5), (3, 0), (4, 7), (9, 2), (16, 33)])
+def test_front_flops_counts_the_loops(k, m):
+    assert oracle.front_flops(k, m) == _front_ops_by_loops(k, m)
+
+
+@pytest.mark.parametrize("kind,dims", [("5pt", (32, 32, 1)), ("27pt", (6, 5, 4)), ("7pt", (12, 12, 12))])
+def test_front_flops_fundamental_equals_true_count(kind, dims):
+    """On FUNDAMENTAL supernodes there is no padding, so the F-U flops summed over
+    the fronts equal the true count sum_j cc_j^2 -- two different formulas."""
+    A, p = grid(kind, dims)
+    sym = oracle.symbolic(A, p, amalgamate=False)
+    tot = sum(oracle.front_flops(sym.k(s), sym.rows(s).size - sym.k(s)) for s in range(sym.nsuper))
+    assert tot == sym.flops == int((sym.cc.astype(np.int64) ** 2).sum())
+    assert sym.exec_flops == tot
