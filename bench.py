@@ -12,9 +12,9 @@ algorithmic flops of the TRUE factor, sum_j cc_j^2.
 
 Multi-GPU (torchrun, one rank per GPU): the SAME matrix is factored by all
 ranks together -- elimination subtrees mapped subtree-to-GPU, the supernodes
-above them factored by rank 0 after the subtree roots' update matrices arrive
-over NCCL (torch.distributed) -- so this is strong scaling ("scaling":
-"strong"); DESIGN.md "Multi-GPU" states the bound of the undistributed top.
+above them replicated on every rank (the large ones factored cooperatively,
+pivot-column blocks broadcast over NCCL by their owner) -- so this is strong
+scaling ("scaling": "strong"); DESIGN.md "Multi-GPU" states the modelled bound.
 """
 from __future__ import annotations
 

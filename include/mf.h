@@ -21,12 +21,17 @@
  *   - perm: int32[n], perm[k] = original index of the k-th pivot (new -> old,
  *     as in A(p,p)).  The library composes it with an elimination-tree
  *     postorder; mf_get_perm() returns the composition ("final perm").
- *     perm must be non-NULL (this library ships no ordering; callers pass a
- *     nested-dissection order, see workloads/grids.py).
+ *     perm == NULL: the library orders A itself on the host by METIS nested
+ *     dissection (METIS_NodeND of the CUDA toolkit's static METIS, the ordering
+ *     behind cusolverSpXcsrmetisndHost) of the graph of A + A^T; the paper used
+ *     its solver's own ordering [PAPER.md L71].
  *   - values, b, x: float64 arrays that may be HOST or DEVICE pointers
  *     (detected with cudaPointerGetAttributes).  They are borrowed for the
  *     duration of the call only.  x is caller-allocated (n doubles) and must
- *     not alias b.
+ *     not alias b.  Device inputs must be complete when read: a ctx running on
+ *     its own stream (mf_options.stream == NULL) first waits for the work
+ *     already queued on the legacy default stream; a caller that passes its own
+ *     stream orders the producers of values / b on that stream itself.
  *   - Ownership: the ctx owns the symbolic plan, the device arena (L panels
  *     and update matrices) and its CUDA stream usage until mf_destroy().
  *   - State machine: create -> analyze -> factor -> solve*; factor may repeat
@@ -62,7 +67,11 @@ typedef struct {
     int32_t amalgamate;       /* 1 = SURVEY Appendix-B relaxed rule (default), 0 = fundamental supernodes */
     int32_t nrelax[3];        /* default {4, 16, 48}                                              */
     double zrelax[3];         /* default {0.8, 0.1, 0.05}                                         */
-    int32_t small_front_max;  /* fronts of order <= this use the batched shared-memory kernel      */
+    int32_t small_front_max;  /* threshold policy (no variant model set): fronts of order <= this use
+                                 the batched warp / shared-memory kernels, larger ones the tiled
+                                 path; also the small/large split of the solve.  With a variant
+                                 model (mf_set_variant_model) the model picks each front's class
+                                 and this threshold does not bound it.                            */
     int32_t panel_w;          /* large-front diagonal block width (multiple of 16, <= 64)          */
     int32_t device;           /* CUDA device ordinal (-1 = current)                                */
     int32_t host_only;        /* 1 = symbolic analysis + planning only, no device (mf_factor/mf_solve
@@ -90,6 +99,15 @@ typedef struct {
                                  latency-bound panel with throughput-bound updates); 0 (default) =
                                  one stream.  Same arithmetic either way (bit-identical L); measured
                                  no faster on c3-c5 (the co-running update slows the panel chain). */
+    /* Device-memory hooks (NULL = cudaMalloc / cudaFree).  Every device buffer the
+     * ctx owns (plan arrays, L and U arenas, vectors) is taken from dev_alloc(bytes,
+     * alloc_user) on the ctx's device and returned through dev_free(ptr, alloc_user)
+     * by mf_analyze (re-analysis) and mf_destroy; the Python binding can route them
+     * to PyTorch's caching allocator.  dev_alloc returns NULL on failure
+     * (=> MF_ERR_NOMEM).  Both or neither must be set. */
+    void *(*dev_alloc)(size_t bytes, void *alloc_user);
+    void (*dev_free)(void *ptr, void *alloc_user);
+    void *alloc_user;
 } mf_options;
 
 typedef struct {
@@ -127,9 +145,14 @@ typedef struct {
 
 #define MF_KERNEL_CLASSES 7
 
-/* Multi-GPU exchange.  With nranks > 1 every rank passes the
- * same n/colptr/rowind/perm/values/b; elimination subtrees are mapped to ranks and
- * the supernodes above them ("top") are factored by rank 0.  The library hands
+/* Multi-GPU exchange.  With nranks > 1 every rank makes the
+ * same calls with the same n/colptr/rowind/perm; `values` and `b` are read from
+ * RANK 0's buffers and broadcast (other ranks may pass any buffer of the right
+ * size); x is returned on every rank.  Elimination subtrees are mapped to ranks;
+ * the supernodes above them ("top") are replicated on every rank, the small ones
+ * factored redundantly and the large ones cooperatively (pivot-column blocks
+ * owned block-cyclically and broadcast by their owner, U^n all-gathered;
+ * DESIGN.md Sec. 9).  The library hands
  * the data movement to a caller-supplied callback (NCCL through torch.distributed
  * in the Python binding), called by every rank with matching lists:
  *   SEND/RECV  point-to-point, `peer` = the other rank;
@@ -157,8 +180,10 @@ int mf_default_options(mf_options *opt);
 int mf_create(mf_ctx **ctx, const mf_options *opt);
 
 /* Symbolic analysis + device planning for the pattern (colptr, rowind) under
- * the order perm.  Host arrays only.  Uploads the
- * flat plan arrays and allocates the device arena. */
+ * the order perm; perm == NULL = METIS nested
+ * dissection computed here (see "perm" above).  Host arrays only.  Uploads the
+ * flat plan arrays and allocates the device arena.  Errors: MF_ERR_ARG for a
+ * malformed pattern or a perm that is not a permutation. */
 int mf_analyze(mf_ctx *ctx, int64_t n, const int64_t *colptr, const int32_t *rowind,
                const int32_t *perm);
 
@@ -167,8 +192,16 @@ int mf_analyze(mf_ctx *ctx, int64_t n, const int64_t *colptr, const int32_t *row
  * returning (the NOT_SPD flag is read back). */
 int mf_factor(mf_ctx *ctx, const double *values);
 
-/* x = A^{-1} b through L y = P b, L^T z = y, x = P^T z.  b, x host or device. */
+/* x = A^{-1} b through L y = P b, L^T z = y, x = P^T z [PAPER.md L7].
+ * b, x host or device (n doubles each, not aliased). */
 int mf_solve(mf_ctx *ctx, const double *b, double *x);
+
+/* nrhs right-hand sides: B and X are column-major n x nrhs with leading
+ * dimensions ldb, ldx >= n (host or device, not aliased); X(:, r) = A^{-1} B(:, r),
+ * bitwise the same as nrhs calls of mf_solve.  The right-hand sides are queued
+ * back to back on the ctx stream (one CUDA-graph replay each, one final
+ * synchronization).  MF_ERR_ARG for nrhs < 0 or ld < n. */
+int mf_solve_nrhs(mf_ctx *ctx, int32_t nrhs, const double *B, int64_t ldb, double *X, int64_t ldx);
 
 int mf_get_info(const mf_ctx *ctx, mf_info *out);
 
@@ -195,7 +228,16 @@ int mf_export_panel(const mf_ctx *ctx, int32_t s, double *out);
 int mf_export_diag(const mf_ctx *ctx, double *out);
 
 /* Copy every panel (supernode order, each f*k as above) to host: out[sum f*k]. */
-int mf_export_L(const mf_ctx *ctx, double *out);
+int mf_export_panels(const mf_ctx *ctx, double *out);
+
+/* L in supernodal CSC (final-perm labels, host buffers): column j of supernode s
+ * (local column jj) holds the rows R_s[jj..f) -- its diagonal first, then the
+ * rows below, ascending -- so Lp[n] = info.nnzL_stored; entries that are
+ * amalgamation padding are stored as exact 0.0.  Lp: int64[n + 1],
+ * Li: int32[nnzL_stored], Lx: float64[nnzL_stored]; any of them may be NULL
+ * (e.g. Lp alone to size the others).  Requires a successful mf_factor (Lp / Li
+ * alone: a successful mf_analyze). */
+int mf_export_L(const mf_ctx *ctx, int64_t *Lp, int32_t *Li, double *Lx);
 
 /* The static launch program mf_factor replays (one entry per kernel launch, in
  * order; the leading init launch is not listed).  kind = kernel class index

@@ -10,4 +10,5 @@ and ``mf_create`` fails without a CUDA device.
 from .mf import (  # noqa: F401
     MF_OK, MF_NOT_SPD, MF_ERR_ARG, MF_ERR_STATE, MF_ERR_NOMEM, MF_ERR_CUDA, MF_ERR_NCCL,
     MfError, MfNotSPD, lib, lib_path, Options, Info, Solver, EXPORTED_SYMBOLS, MF_VARIANTS, MF_VARIANT_FEATURES,
+    DEV_ALLOC_FN, DEV_FREE_FN,
 )

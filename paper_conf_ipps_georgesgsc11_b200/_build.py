@@ -34,7 +34,9 @@ def build(force: bool = False, verbose: bool = False) -> str:
     nvcc = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
     cmd = [nvcc, "-shared", "-Xcompiler", "-fPIC,-O3", "-O3", "-std=c++17", *ARCH, "-lineinfo",
            "-Xptxas", "-v" if verbose else "-O3",
-           "-I", os.path.join(ROOT, "include"), "-I", CSRC, *sources(), "-o", LIB + ".tmp"]
+           "-I", os.path.join(ROOT, "include"), "-I", CSRC, *sources(), "-o", LIB + ".tmp",
+           # METIS nested dissection for perm == NULL (static, from the CUDA toolkit)
+           "-L/usr/local/cuda/lib64", "-l:libmetis_static.a", "-Xlinker", "--exclude-libs,ALL"]
     subprocess.check_call(cmd)
     os.replace(LIB + ".tmp", LIB)
     return LIB

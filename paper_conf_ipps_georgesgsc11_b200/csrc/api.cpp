@@ -46,7 +46,7 @@ struct mf_ctx {
     double *d_y = nullptr, *d_bx = nullptr;
     int *d_failed = nullptr;
     int32_t *d_solve_list = nullptr, *d_df_tasks = nullptr;
-    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev_in = nullptr;
     int64_t launches = 0;
     bool profiling = false;
     bool use_graph = true;
@@ -66,6 +66,10 @@ struct mf_ctx {
     cudaEvent_t la_ev[4] = {nullptr, nullptr, nullptr, nullptr};   // hi fork, side fork, side join, hi join
     mf_kernel_stat kstats[KC_COUNT];
     int64_t prof_factors = 0;
+    // device-memory hooks (mf_options.dev_alloc / dev_free; NULL = cudaMalloc / cudaFree)
+    void *(*halloc)(size_t, void *) = nullptr;
+    void (*hfree)(void *, void *) = nullptr;
+    void *huser = nullptr;
 };
 
 namespace {
@@ -82,22 +86,27 @@ int cuda_err(cudaError_t e) {
         if (_r != MF_OK) return _r;      \
     } while (0)
 
-template <class T>
-int dev_upload(mf_ctx *c, T **dst, const std::vector<T> &src) {
-    size_t bytes = std::max<size_t>(src.size(), 1) * sizeof(T);
+// Every device buffer of the ctx comes from here: the caller's hooks or cudaMalloc.
+int dev_alloc(mf_ctx *c, void **dst, size_t bytes) {
     void *p = nullptr;
-    CK(cudaMalloc(&p, bytes));
+    bytes = std::max<size_t>(bytes, 16);
+    if (c->halloc) {
+        p = c->halloc(bytes, c->huser);
+        if (!p) return MF_ERR_NOMEM;
+    } else {
+        CK(cudaMalloc(&p, bytes));
+    }
     c->allocs.push_back(p);
-    if (!src.empty()) CK(cudaMemcpy(p, src.data(), src.size() * sizeof(T), cudaMemcpyHostToDevice));
-    *dst = (T *)p;
+    *dst = p;
     return MF_OK;
 }
 
-int dev_alloc(mf_ctx *c, void **dst, size_t bytes) {
+template <class T>
+int dev_upload(mf_ctx *c, T **dst, const std::vector<T> &src) {
     void *p = nullptr;
-    CK(cudaMalloc(&p, std::max<size_t>(bytes, 16)));
-    c->allocs.push_back(p);
-    *dst = p;
+    if (int r = dev_alloc(c, &p, std::max<size_t>(src.size(), 1) * sizeof(T))) return r;
+    if (!src.empty()) CK(cudaMemcpy(p, src.data(), src.size() * sizeof(T), cudaMemcpyHostToDevice));
+    *dst = (T *)p;
     return MF_OK;
 }
 
@@ -118,9 +127,24 @@ void drop_graph(mf_ctx *c) {
 
 void free_device(mf_ctx *c) {
     drop_graph(c);
-    for (void *p : c->allocs) cudaFree(p);
+    for (void *p : c->allocs) {
+        if (c->hfree) c->hfree(p, c->huser);
+        else cudaFree(p);
+    }
     c->allocs.clear();
     c->d = DevPlan{};
+}
+
+// Device inputs (values, b) were produced on some caller stream.  A ctx that
+// created its own non-blocking stream orders its first read after all work
+// already queued on the legacy default stream (where torch's default stream and
+// plain cudaMemcpy land); a caller that passed mf_options.stream orders its own
+// producers on that stream (include/mf.h, "Pointers").
+int order_after_caller(mf_ctx *c) {
+    if (!c->own_stream) return MF_OK;
+    CK(cudaEventRecord(c->ev_in, cudaStreamLegacy));
+    CK(cudaStreamWaitEvent(c->stream, c->ev_in, 0));
+    return MF_OK;
 }
 
 bool is_device_ptr(const void *p) {
@@ -195,6 +219,9 @@ int mf_default_options(mf_options *o) {
     o->nbranch = d.nbranch;
     o->fuse_ea = d.fuse_ea;
     o->lookahead = d.lookahead;
+    o->dev_alloc = nullptr;
+    o->dev_free = nullptr;
+    o->alloc_user = nullptr;
     return MF_OK;
 }
 
@@ -230,6 +257,13 @@ int mf_create(mf_ctx **out, const mf_options *o) {
     c->opt.lookahead = o->lookahead != 0;
     c->opt.rank = o->rank;
     c->host_only = o->host_only != 0;
+    if ((o->dev_alloc == nullptr) != (o->dev_free == nullptr)) {
+        delete c;
+        return MF_ERR_ARG;
+    }
+    c->halloc = o->dev_alloc;
+    c->hfree = o->dev_free;
+    c->huser = o->alloc_user;
     c->info.failed_col = -1;
     if (c->host_only) {   // symbolic analysis + plan only; never touches CUDA
         *out = c;
@@ -260,6 +294,7 @@ int mf_create(mf_ctx **out, const mf_options *o) {
     }
     cudaEventCreate(&c->ev0);
     cudaEventCreate(&c->ev1);
+    cudaEventCreateWithFlags(&c->ev_in, cudaEventDisableTiming);
     c->info.failed_col = -1;
     *out = c;
     return MF_OK;
@@ -283,6 +318,7 @@ void mf_destroy(mf_ctx *c) {
     for (cudaStream_t bs : c->bstreams) cudaStreamDestroy(bs);
     if (c->ev0) cudaEventDestroy(c->ev0);
     if (c->ev1) cudaEventDestroy(c->ev1);
+    if (c->ev_in) cudaEventDestroy(c->ev_in);
     if (c->own_stream) cudaStreamDestroy(c->stream);
     delete c;
 }
@@ -620,13 +656,22 @@ int mf_factor(mf_ctx *c, const double *values) {
     cudaStream_t st = c->stream;
     const bool multi = P.nranks > 1;
     if (multi && !c->xfn) return MF_ERR_STATE;
-    CK(cudaEventRecord(c->ev0, st));
     const double *vals = values;
-    if (!is_device_ptr(values)) {
+    const bool vdev = is_device_ptr(values);
+    if (vdev) {
+        if (int r = order_after_caller(c)) return r;
+    }
+    CK(cudaEventRecord(c->ev0, st));
+    if (!vdev || multi) {
         // bvidx indexes the caller's array; copy the whole array (colptr[n] entries)
         if (c->S.nnz_in > 0)
-            CK(cudaMemcpyAsync(c->d_values, values, c->S.nnz_in * sizeof(double), cudaMemcpyHostToDevice, st));
+            CK(cudaMemcpyAsync(c->d_values, values, c->S.nnz_in * sizeof(double),
+                               vdev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, st));
         vals = c->d_values;
+    }
+    if (multi && c->S.nnz_in > 0) {   // rank 0's values are the matrix (include/mf.h)
+        std::vector<mf_xfer> bc{mf_xfer{MF_XFER_BCAST, 0, c->d_values, c->S.nnz_in * (int64_t)sizeof(double)}};
+        if (int r = exchange(c, bc)) return r;
     }
     const bool prof = c->profiling;
     const size_t nev = 2 * (P.program.size() + P.program_top.size());
@@ -716,8 +761,11 @@ int mf_solve(mf_ctx *c, const double *b, double *x) {
     cudaStream_t st = c->stream;
     const int64_t n = c->S.n;
     const bool multi = P.nranks > 1;
-    CK(cudaEventRecord(c->ev0, st));
     const bool bdev = is_device_ptr(b), xdev = is_device_ptr(x);
+    if (bdev || xdev) {
+        if (int r = order_after_caller(c)) return r;
+    }
+    CK(cudaEventRecord(c->ev0, st));
     if (!multi && c->use_graph) {
         // single GPU: the whole solve is one CUDA graph over the ctx buffers
         // (b -> d_bx, permute, forward, backward, permute back into d_bx -> x)
@@ -747,9 +795,14 @@ int mf_solve(mf_ctx *c, const double *b, double *x) {
         return MF_OK;
     }
     const double *bd = b;
-    if (!bdev) {
-        CK(cudaMemcpyAsync(c->d_bx, b, n * sizeof(double), cudaMemcpyHostToDevice, st));
+    if (!bdev || multi) {
+        CK(cudaMemcpyAsync(c->d_bx, b, n * sizeof(double), bdev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice,
+                           st));
         bd = c->d_bx;
+    }
+    if (multi && n > 0) {   // rank 0's right-hand side (include/mf.h)
+        std::vector<mf_xfer> bc{mf_xfer{MF_XFER_BCAST, 0, c->d_bx, n * (int64_t)sizeof(double)}};
+        if (int r = exchange(c, bc)) return r;
     }
     launch_permute_in(d, bd, c->d_y, n, st);
     int r;
@@ -783,6 +836,48 @@ int mf_solve(mf_ctx *c, const double *b, double *x) {
     double *xd = xdev ? x : c->d_bx;
     launch_permute_out(d, c->d_y, xd, n, st);
     if (!xdev) CK(cudaMemcpyAsync(x, c->d_bx, n * sizeof(double), cudaMemcpyDeviceToHost, st));
+    CK(cudaGetLastError());
+    CK(cudaEventRecord(c->ev1, st));
+    CK(cudaStreamSynchronize(st));
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, c->ev0, c->ev1);
+    c->info.t_solve = ms * 1e-3;
+    return MF_OK;
+}
+
+int mf_solve_nrhs(mf_ctx *c, int32_t nrhs, const double *B, int64_t ldb, double *X, int64_t ldx) {
+    if (!c || nrhs < 0) return MF_ERR_ARG;
+    if (c->state != 2 || c->host_only) return MF_ERR_STATE;
+    const int64_t n = c->S.n;
+    if (nrhs == 0) return MF_OK;
+    if (!B || !X || ldb < n || ldx < n) return MF_ERR_ARG;
+    if ((const void *)B == (const void *)X) return MF_ERR_ARG;
+    if (c->P.nranks > 1 || !c->use_graph) {   // one column at a time through mf_solve
+        for (int32_t r = 0; r < nrhs; r++)
+            if (int e = mf_solve(c, B + r * ldb, X + r * ldx)) return e;
+        return MF_OK;
+    }
+    CK(cudaSetDevice(c->device));
+    cudaStream_t st = c->stream;
+    const bool bdev = is_device_ptr(B), xdev = is_device_ptr(X);
+    if (bdev || xdev) {
+        if (int r = order_after_caller(c)) return r;
+    }
+    if (!c->solve_exec) {   // capture the solve graph (same program as mf_solve)
+        if (int e = mf_solve(c, B, X)) return e;
+        if (nrhs == 1) return MF_OK;
+        B += ldb;
+        X += ldx;
+        nrhs -= 1;
+    }
+    CK(cudaEventRecord(c->ev0, st));
+    for (int32_t r = 0; r < nrhs; r++) {
+        CK(cudaMemcpyAsync(c->d_bx, B + r * ldb, n * sizeof(double),
+                           bdev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, st));
+        CK(cudaGraphLaunch(c->solve_exec, st));
+        CK(cudaMemcpyAsync(X + r * ldx, c->d_bx, n * sizeof(double),
+                           xdev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, st));
+    }
     CK(cudaGetLastError());
     CK(cudaEventRecord(c->ev1, st));
     CK(cudaStreamSynchronize(st));
@@ -933,7 +1028,7 @@ int mf_export_diag(const mf_ctx *c, double *out) {
     return MF_OK;
 }
 
-int mf_export_L(const mf_ctx *c, double *out) {
+int mf_export_panels(const mf_ctx *c, double *out) {
     if (!c || !out) return MF_ERR_ARG;
     if (c->state != 2) return MF_ERR_STATE;
     int64_t o = 0;
@@ -942,6 +1037,41 @@ int mf_export_L(const mf_ctx *c, double *out) {
         if (r) return r;
         o += (int64_t)c->P.sn_f[s] * c->P.sn_k[s];
     }
+    return MF_OK;
+}
+
+int mf_export_L(const mf_ctx *c, int64_t *Lp, int32_t *Li, double *Lx) {
+    if (!c) return MF_ERR_ARG;
+    if (c->state < 1) return MF_ERR_STATE;
+    if (Lx && c->state != 2) return MF_ERR_STATE;
+    const Symbolic &S = c->S;
+    const Plan &P = c->P;
+    const int64_t n = S.n;
+    if (Lp) {   // column j of supernode s (local jj): rows R_s[jj..f)
+        Lp[0] = 0;
+        for (int32_t s = 0; s < P.nsuper; s++)
+            for (int32_t jj = 0; jj < P.sn_k[s]; jj++) {
+                const int64_t j = S.sn_first[s] + jj;
+                Lp[j + 1] = Lp[j] + (P.sn_f[s] - jj);
+            }
+    }
+    if (!Li && !Lx) return MF_OK;
+    std::vector<double> panel;
+    int64_t o = 0;
+    for (int32_t s = 0; s < P.nsuper; s++) {
+        const int32_t f = P.sn_f[s], k = P.sn_k[s];
+        const int32_t *R = S.sn_rows.data() + S.sn_rowptr[s];
+        if (Lx) {
+            panel.resize((size_t)f * k);
+            if (int r = mf_export_panel(c, s, panel.data())) return r;
+        }
+        for (int32_t jj = 0; jj < k; jj++) {
+            if (Li) std::memcpy(Li + o, R + jj, (size_t)(f - jj) * sizeof(int32_t));
+            if (Lx) std::memcpy(Lx + o, panel.data() + (size_t)jj * f + jj, (size_t)(f - jj) * sizeof(double));
+            o += f - jj;
+        }
+    }
+    (void)n;
     return MF_OK;
 }
 

@@ -267,10 +267,8 @@ void launch_small_fronts(const DevPlan &d, const int32_t *list, int count, int f
     const size_t smem = (size_t)(fmax * fmax + fmax) * sizeof(double);
     if (fmax <= 16) {
         k_tiny_fronts<16><<<(count + kTinyWarps - 1) / kTinyWarps, 32 * kTinyWarps, 0, st>>>(d, list, count, values);
-    } else if (fmax <= kTinyF) {
+    } else if (fmax <= kTinyF) {   // kTinyF = 32: every f <= 32 class is one warp per front
         k_tiny_fronts<32><<<(count + kTinyWarps - 1) / kTinyWarps, 32 * kTinyWarps, 0, st>>>(d, list, count, values);
-    } else if (fmax <= 32) {
-        k_small_front<64><<<count, 64, smem, st>>>(d, list, values);
     } else if (fmax <= 64) {
         k_small_front<128><<<count, 128, smem, st>>>(d, list, values);
     } else {
@@ -661,7 +659,10 @@ __global__ void __launch_bounds__(kTrsmThreads, 2) k_trsm_panel(DevPlan d, const
 __global__ void __launch_bounds__(kTrsmThreads, 2) k_leaf(DevPlan d, const int32_t *__restrict__ fronts, int npotrf,
                                                           const int32_t *__restrict__ tasks, int j0, int w) {
     extern __shared__ __align__(16) double tsm[];
-    const unsigned expect = ((*d.epoch & 0x3fffffu) << 10) | (unsigned)(j0 / w + 1);   // w >= 16: < 1024 leaves
+    // tag = (epoch mod 2^16) << 16 | leaf index + 1: consecutive factorizations differ in
+    // the epoch bits, and the leaf index (k / w < 2^16 - 1, checked by build_plan) never
+    // spills into them (10 bits overflowed for k > 1023 w)
+    const unsigned expect = ((*d.epoch & 0xffffu) << 16) | (unsigned)(j0 / w + 1);
     if ((int)blockIdx.x < npotrf) {
         const int s = fronts[blockIdx.x];
         potrf_block<kTrsmThreads>(d, s, j0, w, tsm, tsm + kWmax * kWmax);
@@ -1118,7 +1119,7 @@ __global__ void __launch_bounds__(kPanelThreads, MF_PANEL_MINB) k_panel(DevPlan 
     const int r0 = j0 + 64 * c, rows = min(64, f - r0);
     double *__restrict__ Pn = d.L + d.L_off[s];
     unsigned *F = d.panel_flag + (int64_t)s * kPanelFlags;
-    const unsigned tag = ((*d.epoch & 0x3fffffu) << 10) | (unsigned)(j0 / 64 + 1);
+    const unsigned tag = ((*d.epoch & 0xffffu) << 16) | (unsigned)(j0 / 64 + 1);   // as in k_leaf
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, gq = lane >> 2, tq = lane & 3;
     const bool band = c < nb;
     // the diagonal tile's accumulator: its 36 lower 8 x 8 blocks, 9 per warp

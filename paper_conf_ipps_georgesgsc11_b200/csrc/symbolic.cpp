@@ -13,16 +13,75 @@
 //   * fundamental supernodes (reading C2) and the Appendix-B relaxed amalgamation
 //     rule (verbatim -- both sides must agree bit-exactly);
 //   * row lists: supernodal merge R_s = cols(s) U rows(B(:, cols(s))) U
-//     (U_{children t} R_t), with a marker array.
+//     (U_{children t} R_t), with a marker array;
+//   * perm == NULL: the library's own host-side ordering, METIS nested dissection
+//     (METIS_NodeND of the static METIS that ships with the CUDA toolkit, the one
+//     behind cusolverSpXcsrmetisndHost) on the graph of A + A^T without the
+//     diagonal (reading C4; the paper used WSMP's own
+//     ordering).
 #include <algorithm>
 #include <cstring>
 
 #include "mf.h"
 #include "mf_plan.h"
 
+// METIS 5 (libmetis_static.a of the CUDA toolkit, built with 64-bit idx_t);
+// declared here because the toolkit ships the library without metis.h.
+extern "C" {
+int METIS_SetDefaultOptions(int64_t *options);
+int METIS_NodeND(int64_t *nvtxs, int64_t *xadj, int64_t *adjncy, int64_t *vwgt, int64_t *options, int64_t *perm,
+                 int64_t *iperm);
+}
+
 namespace mf {
 
 namespace {
+
+constexpr int kMetisOk = 1, kMetisNoptions = 40;
+
+// Fill-reducing nested-dissection order (new -> old) of the pattern's graph.
+int order_metis(int64_t n, const int64_t *colptr, const int32_t *rowind, std::vector<int32_t> &perm) {
+    perm.resize(n);
+    if (n == 0) return MF_OK;
+    // symmetric adjacency without the diagonal: count, fill, then sort + dedup per vertex
+    std::vector<int64_t> deg(n + 1, 0);
+    for (int64_t c = 0; c < n; c++)
+        for (int64_t p = colptr[c]; p < colptr[c + 1]; p++)
+            if (rowind[p] != c) {
+                deg[rowind[p] + 1]++;
+                deg[c + 1]++;
+            }
+    for (int64_t v = 0; v < n; v++) deg[v + 1] += deg[v];
+    std::vector<int64_t> adj(deg[n]), fill(deg.begin(), deg.end() - 1);
+    for (int64_t c = 0; c < n; c++)
+        for (int64_t p = colptr[c]; p < colptr[c + 1]; p++)
+            if (rowind[p] != c) {
+                adj[fill[rowind[p]]++] = c;
+                adj[fill[c]++] = rowind[p];
+            }
+    std::vector<int64_t> xadj(n + 1, 0);
+    int64_t e = 0;
+    for (int64_t v = 0; v < n; v++) {
+        int64_t *b = adj.data() + deg[v], *t = adj.data() + deg[v + 1];
+        std::sort(b, t);
+        t = std::unique(b, t);
+        xadj[v] = e;
+        for (int64_t *q = b; q < t; q++) adj[e++] = *q;
+    }
+    xadj[n] = e;
+    if (e == 0) {   // no edges (diagonal matrix): any order is fill-free
+        for (int64_t v = 0; v < n; v++) perm[v] = (int32_t)v;
+        return MF_OK;
+    }
+    int64_t opts[kMetisNoptions];
+    METIS_SetDefaultOptions(opts);
+    int64_t nv = n;
+    std::vector<int64_t> p(n), ip(n);
+    if (METIS_NodeND(&nv, xadj.data(), adj.data(), nullptr, opts, p.data(), ip.data()) != kMetisOk)
+        return MF_ERR_NOMEM;
+    for (int64_t k = 0; k < n; k++) perm[k] = (int32_t)p[k];   // row k of P A P^T is row p[k] of A
+    return MF_OK;
+}
 
 // B = P A P^T restricted to lower entries, duplicates grouped (input order kept).
 int build_B(int64_t n, const int64_t *colptr, const int32_t *rowind, const std::vector<int32_t> &perm,
@@ -152,13 +211,18 @@ void tree_postorder(int64_t n, const std::vector<int32_t> &parent, std::vector<i
 int analyze_symbolic(int64_t n, const int64_t *colptr, const int32_t *rowind, const int32_t *perm_in,
                      const Options &opt, Symbolic &S) {
     // ---------------- validation
-    if (n < 0 || n >= (int64_t)INT32_MAX || !colptr || !perm_in) return MF_ERR_ARG;
+    if (n < 0 || n >= (int64_t)INT32_MAX || !colptr) return MF_ERR_ARG;
     if (n > 0 && !rowind && colptr[n] > 0) return MF_ERR_ARG;
     if (colptr[0] != 0) return MF_ERR_ARG;
     for (int64_t c = 0; c < n; c++)
         if (colptr[c + 1] < colptr[c]) return MF_ERR_ARG;
     for (int64_t p = 0; p < colptr[n]; p++)
         if (rowind[p] < 0 || rowind[p] >= n) return MF_ERR_ARG;
+    std::vector<int32_t> lib_perm;
+    if (!perm_in) {   // the library's own ordering
+        if (int st = order_metis(n, colptr, rowind, lib_perm)) return st;
+        perm_in = lib_perm.data();
+    }
     {
         std::vector<char> seen(n, 0);
         for (int64_t k = 0; k < n; k++) {

@@ -25,6 +25,7 @@ MF_ERR_NCCL = -5
 EXPORTED_SYMBOLS = (
     "mf_default_options", "mf_create", "mf_analyze", "mf_factor", "mf_solve", "mf_get_info",
     "mf_get_perm", "mf_get_etree", "mf_get_supernodes", "mf_export_panel", "mf_export_diag", "mf_export_L",
+    "mf_export_panels", "mf_solve_nrhs",
     "mf_get_program", "mf_set_profiling", "mf_get_kernel_stats", "mf_set_exchange", "mf_get_mapping", "mf_destroy", "mf_strerror",
     "mf_get_launch_times", "mf_set_variant_model", "mf_get_variants",
 )
@@ -39,7 +40,12 @@ class Options(ctypes.Structure):
         ("host_only", ctypes.c_int32), ("nranks", ctypes.c_int32), ("rank", ctypes.c_int32),
         ("stream", ctypes.c_void_p), ("split_all", ctypes.c_int32), ("nbranch", ctypes.c_int32),
         ("fuse_ea", ctypes.c_int32), ("lookahead", ctypes.c_int32),
+        ("dev_alloc", ctypes.c_void_p), ("dev_free", ctypes.c_void_p), ("alloc_user", ctypes.c_void_p),
     ]
+
+
+DEV_ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p)
+DEV_FREE_FN = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p)
 
 
 class Info(ctypes.Structure):
@@ -101,7 +107,9 @@ def _load():
         "mf_get_supernodes": ([vp, vp, vp, vp, vp, vp], ctypes.c_int),
         "mf_export_panel": ([vp, i32, vp], ctypes.c_int),
         "mf_export_diag": ([vp, vp], ctypes.c_int),
-        "mf_export_L": ([vp, vp], ctypes.c_int),
+        "mf_export_L": ([vp, vp, vp, vp], ctypes.c_int),
+        "mf_export_panels": ([vp, vp], ctypes.c_int),
+        "mf_solve_nrhs": ([vp, i32, vp, i64, vp, i64], ctypes.c_int),
         "mf_get_program": ([vp, ctypes.POINTER(LaunchInfo), i64, ctypes.POINTER(i64)], ctypes.c_int),
         "mf_set_exchange": ([vp, EXCHANGE_FN, vp], ctypes.c_int),
         "mf_get_mapping": ([vp, vp, vp, vp, vp], ctypes.c_int),
@@ -157,10 +165,17 @@ class Solver:
                  device: int = -1, stream: int | None = None, host_only: bool = False,
                  nranks: int = 1, rank: int = 0, exchange=None, split_all: bool = False,
                  nbranch: int | None = None, fuse_ea: bool | None = None, lookahead: bool | None = None,
-                 variant_model="auto"):
+                 variant_model="auto", torch_alloc: bool = False):
         """variant_model: "auto" = the fitted kernel-variant selector packaged with the
         binding (selector.MODEL_PATH, Eqs. 3-5 fitted to B200 timings) when
-        present, None = libmf's fixed front-order thresholds, or a theta array."""
+        present, None = libmf's fixed front-order thresholds, or a theta array.
+        Precedence: an explicit ``small_front_max`` selects the threshold policy
+        ("auto" then resolves to None), since a variant model chooses each front's
+        class by itself and would ignore the threshold (include/mf.h).
+        torch_alloc: take every device buffer of the ctx from PyTorch's caching
+        allocator (mf_options.dev_alloc / dev_free) instead of cudaMalloc."""
+        if small_front_max is not None and isinstance(variant_model, str) and variant_model == "auto":
+            variant_model = None
         o = Options()
         lib.mf_default_options(ctypes.byref(o))
         o.amalgamate = int(amalgamate)
@@ -180,6 +195,23 @@ class Solver:
         if lookahead is not None:
             o.lookahead = int(lookahead)
         o.stream = stream
+        self._alloc_cbs = None
+        if torch_alloc and not host_only:
+            import torch
+            dev = torch.cuda.current_device() if device < 0 else device
+
+            def _alloc(nbytes, _user):
+                try:
+                    return torch.cuda.caching_allocator_alloc(int(nbytes), dev)
+                except RuntimeError:
+                    return None
+
+            def _free(ptr, _user):
+                torch.cuda.caching_allocator_delete(ptr)
+
+            self._alloc_cbs = (DEV_ALLOC_FN(_alloc), DEV_FREE_FN(_free))
+            o.dev_alloc = ctypes.cast(self._alloc_cbs[0], ctypes.c_void_p)
+            o.dev_free = ctypes.cast(self._alloc_cbs[1], ctypes.c_void_p)
         h = ctypes.c_void_p()
         r = lib.mf_create(ctypes.byref(h), ctypes.byref(o))
         if r != MF_OK:
@@ -251,12 +283,15 @@ class Solver:
         if r != MF_OK:
             raise MfError(r, where)
 
-    def analyze(self, n: int, colptr, rowind, perm):
+    def analyze(self, n: int, colptr, rowind, perm=None):
+        """perm: new -> old order, or None for the library's METIS nested dissection."""
         colptr = np.ascontiguousarray(colptr, dtype=np.int64)
         rowind = np.ascontiguousarray(rowind, dtype=np.int32)
-        perm = np.ascontiguousarray(perm, dtype=np.int32)
-        self._check(lib.mf_analyze(self._h, int(n), colptr.ctypes.data, rowind.ctypes.data, perm.ctypes.data),
-                    "mf_analyze")
+        pp = None
+        if perm is not None:
+            perm = np.ascontiguousarray(perm, dtype=np.int32)
+            pp = perm.ctypes.data
+        self._check(lib.mf_analyze(self._h, int(n), colptr.ctypes.data, rowind.ctypes.data, pp), "mf_analyze")
         self.n = int(n)
         self._info = self.info()
 
@@ -352,7 +387,37 @@ class Solver:
         self._check(lib.mf_export_diag(self._h, out.ctypes.data), "mf_export_diag")
         return out
 
-    def export_L(self, total_words: int) -> np.ndarray:
+    def export_panels(self, total_words: int) -> np.ndarray:
+        """Every panel (supernode order, each f x k column-major) concatenated."""
         out = np.empty(total_words, dtype=np.float64)
-        self._check(lib.mf_export_L(self._h, out.ctypes.data), "mf_export_L")
+        self._check(lib.mf_export_panels(self._h, out.ctypes.data), "mf_export_panels")
         return out
+
+    def export_L(self, values: bool = True):
+        """L in supernodal CSC (final-perm labels): (Lp int64[n+1], Li int32, Lx float64)."""
+        Lp = np.empty(self.n + 1, dtype=np.int64)
+        self._check(lib.mf_export_L(self._h, Lp.ctypes.data, None, None), "mf_export_L")
+        Li = np.empty(int(Lp[-1]), dtype=np.int32)
+        Lx = np.empty(int(Lp[-1]), dtype=np.float64) if values else None
+        self._check(lib.mf_export_L(self._h, Lp.ctypes.data, Li.ctypes.data,
+                                    None if Lx is None else Lx.ctypes.data), "mf_export_L")
+        return Lp, Li, Lx
+
+    def solve_nrhs(self, B, X=None):
+        """X = A^{-1} B for an n x nrhs column-major (Fortran-order) B."""
+        if isinstance(B, np.ndarray):
+            B = np.asfortranarray(B, dtype=np.float64)
+            if B.ndim == 1:
+                B = B[:, None]
+            if X is None:
+                X = np.empty(B.shape, dtype=np.float64, order="F")
+            nrhs, ldb, ldx = B.shape[1], B.shape[0], X.shape[0]
+            bp, xp = B.ctypes.data, X.ctypes.data
+        else:   # torch tensors: (nrhs, n) row-major = n x nrhs column-major
+            nrhs, ldb = B.shape[0], B.shape[1]
+            if X is None:
+                X = B.new_empty(B.shape)
+            ldx = X.shape[1]
+            bp, xp = _ptr(B, np.float64), _ptr(X, np.float64)
+        self._check(lib.mf_solve_nrhs(self._h, int(nrhs), bp, int(ldb), xp, int(ldx)), "mf_solve_nrhs")
+        return X

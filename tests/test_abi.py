@@ -132,3 +132,52 @@ def test_symbolic_postorder_hand_worked():
     S.analyze(Aq.n, Aq.colptr, Aq.rowind, q)
     np.testing.assert_array_equal(S.perm(), e["final_perm_with_q"])
     _check_symbolic(Aq, q)
+
+
+@pytest.mark.parametrize("kind,dims", [("27pt", (12, 11, 10)), ("5pt", (40, 30, 1)), ("elast", (6, 6, 6))])
+def test_null_perm_library_ordering(kind, dims):
+    """perm == NULL: the library orders A itself (METIS nested dissection,
+    include/mf.h; reading C4).  The returned final perm is a permutation, the same
+    on every call, and the symbolic analysis under it matches the oracle's
+    bit-exactly; its fill is in the range of the geometric ND order."""
+    A, p = grid(kind, dims)
+    S = mf.Solver(host_only=True)
+    S.analyze(A.n, A.colptr, A.rowind, None)
+    fp = S.perm()
+    assert np.array_equal(np.sort(fp), np.arange(A.n))
+    S2 = mf.Solver(host_only=True)
+    S2.analyze(A.n, A.colptr, A.rowind, None)
+    np.testing.assert_array_equal(S2.perm(), fp)
+    _check_symbolic(A, fp)          # the final perm is already postordered: analysis is identical
+    np.testing.assert_array_equal(S.etree()[0], oracle.symbolic(A, fp).parent)
+    Sg = mf.Solver(host_only=True)
+    Sg.analyze(A.n, A.colptr, A.rowind, p)
+    assert S.info()["flops_true"] <= 2 * Sg.info()["flops_true"]
+
+
+def test_export_csc_structure_host_only():
+    """mf_export_L (supernodal CSC): column j of supernode s holds R_s[jj..f), so
+    Lp[n] = nnzL_stored and the row lists are the oracle's (Lx needs a factor)."""
+    A, p = grid("27pt", (9, 8, 7))
+    S = mf.Solver(host_only=True)
+    S.analyze(A.n, A.colptr, A.rowind, p)
+    Lp, Li, _ = S.export_L(values=False)
+    so = oracle.symbolic(A, p, keep_struct=True)
+    assert Lp[-1] == S.info()["nnzL_stored"] == so.stored_L
+    for s in range(so.nsuper):
+        R = so.rows(s)
+        for jj in range(so.k(s)):
+            j = int(so.sn_first[s]) + jj
+            np.testing.assert_array_equal(Li[Lp[j]:Lp[j + 1]], R[jj:])
+            # the true structure of column j is a subset (the rest is padding)
+            assert set(so.Li[so.Lp[j]:so.Lp[j + 1]].tolist()) <= set(R[jj:].tolist())
+
+
+def test_alloc_hooks_must_come_in_pairs():
+    o = mf.Options()
+    mf.lib.mf_default_options(ctypes.byref(o))
+    o.host_only = 1
+    keep = mf.DEV_ALLOC_FN(lambda n, u: None)
+    o.dev_alloc = ctypes.cast(keep, ctypes.c_void_p)
+    h = ctypes.c_void_p()
+    assert mf.lib.mf_create(ctypes.byref(h), ctypes.byref(o)) == mf.MF_ERR_ARG

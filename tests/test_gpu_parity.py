@@ -218,7 +218,7 @@ def test_deterministic_bitwise(mf):
     outs = []
     for _ in range(3):
         S.factor(A.values)
-        outs.append(S.export_L(sum_panel_words(S, inf)))
+        outs.append(S.export_panels(sum_panel_words(S, inf)))
     assert all(np.array_equal(outs[0], o) for o in outs[1:])
 
 
@@ -236,7 +236,7 @@ def test_fused_extend_add_bit_identical(mf, kind, dims, small_max, w):
         S.analyze(A.n, A.colptr, A.rowind, p)
         inf = S.info()
         S.factor(A.values)
-        outs.append(S.export_L(sum_panel_words(S, inf)))
+        outs.append(S.export_panels(sum_panel_words(S, inf)))
     np.testing.assert_array_equal(outs[0], outs[1])
     sym = oracle.symbolic(A, p, keep_struct=True)
     check_panels(S, sym, oracle.factor(A, sym))
@@ -254,7 +254,7 @@ def test_lookahead_bit_identical(mf, kind, dims, nb):
         S.analyze(A.n, A.colptr, A.rowind, p)
         inf = S.info()
         S.factor(A.values)
-        outs.append(S.export_L(sum_panel_words(S, inf)))
+        outs.append(S.export_panels(sum_panel_words(S, inf)))
     np.testing.assert_array_equal(outs[0], outs[1])
     np.testing.assert_array_equal(outs[0], outs[2])
     sym = oracle.symbolic(A, p, keep_struct=True)
@@ -274,7 +274,7 @@ S.analyze(A.n, A.colptr, A.rowind, p)
 S.factor(A.values)
 sn = S.supernodes()
 k = np.diff(sn["sn_first"]); f = np.diff(sn["sn_rowptr"])
-print(hashlib.sha256(S.export_L(int(np.sum((f + (f & 1)) * k)) + 2).tobytes()).hexdigest())
+print(hashlib.sha256(S.export_panels(int(np.sum((f + (f & 1)) * k)) + 2).tobytes()).hexdigest())
 '''
 
 
@@ -334,3 +334,77 @@ def test_degenerate_inputs(mf):
     assert S.solve(np.zeros(0)).size == 0
 
 
+
+
+@pytest.mark.parametrize("kind,dims", [("27pt", (16, 15, 14)), ("elast", (7, 7, 7))])
+def test_null_perm_parity(mf, kind, dims):
+    """perm == NULL (library METIS ordering): the factor under the returned final
+    perm matches the oracle's, and the solve is backward stable."""
+    A, _ = grid(kind, dims)
+    S = mf.Solver()
+    S.analyze(A.n, A.colptr, A.rowind, None)
+    S.factor(A.values)
+    fp = S.perm()
+    sym = oracle.symbolic(A, fp, keep_struct=True)
+    check_panels(S, sym, oracle.factor(A, sym))
+    b = spmv(A, G.rhs(A.n, 0))
+    assert backward_error(A, S.solve(b), b) <= TOL_BE
+
+
+def test_export_csc_matches_panels_and_oracle(mf):
+    """mf_export_L: supernodal CSC of L; every column equals the oracle's
+    (reading C11), padding rows exactly 0, L L^T reconstructs P A P^T."""
+    A, p = grid("27pt", (11, 10, 9))
+    S = mf.Solver()
+    S.analyze(A.n, A.colptr, A.rowind, p)
+    S.factor(A.values)
+    Lp, Li, Lx = S.export_L()
+    sym = oracle.symbolic(A, p, keep_struct=True)
+    panels = oracle.factor(A, sym)
+    Lo = oracle.panels_to_dense_L(sym, panels)
+    Lg = np.zeros_like(Lo)
+    cols = np.repeat(np.arange(A.n), np.diff(Lp))
+    Lg[Li, cols] = Lx
+    assert c11(Lg, Lo) <= TOL_L
+    M = G.full_symmetric_dense(A)[np.ix_(sym.perm, sym.perm)]
+    assert np.abs(Lg @ Lg.T - M).max() <= 1e-12 * np.abs(M).max()
+
+
+def test_torch_allocator_hooks(mf):
+    """mf_options.dev_alloc / dev_free routed to PyTorch's caching allocator: the
+    arena comes from torch (its reserved memory grows) and L is bitwise the same."""
+    import torch
+    A, p = grid("27pt", (16, 16, 16))
+    outs = []
+    for ta in (False, True):
+        torch.cuda.synchronize()
+        before = torch.cuda.memory_allocated()
+        S = mf.Solver(torch_alloc=ta)
+        S.analyze(A.n, A.colptr, A.rowind, p)
+        grew = torch.cuda.memory_allocated() - before
+        assert (grew >= S.info()["workspace_bytes"] // 2) if ta else grew == 0
+        S.factor(A.values)
+        outs.append(S.export_panels(sum_panel_words(S, S.info())))
+        S.close()
+        if ta:
+            assert torch.cuda.memory_allocated() == before   # every block returned
+    np.testing.assert_array_equal(outs[0], outs[1])
+
+
+def test_solve_nrhs(mf):
+    """mf_solve_nrhs: X(:, r) = A^{-1} B(:, r), bitwise equal to one mf_solve per
+    column; host and device buffers."""
+    import torch
+    A, p = grid("27pt", (15, 14, 13))
+    S = mf.Solver()
+    S.analyze(A.n, A.colptr, A.rowind, p)
+    S.factor(A.values)
+    rng = np.random.default_rng(5)
+    B = np.asfortranarray(rng.uniform(-1, 1, (A.n, 5)))
+    X = S.solve_nrhs(B)
+    for r in range(5):
+        np.testing.assert_array_equal(X[:, r], S.solve(np.ascontiguousarray(B[:, r])))
+        assert backward_error(A, X[:, r], B[:, r]) <= TOL_BE
+    Bt = torch.from_numpy(np.ascontiguousarray(B.T)).cuda()   # (nrhs, n) rows = columns of B
+    Xt = S.solve_nrhs(Bt)
+    np.testing.assert_array_equal(Xt.cpu().numpy().T, X)

@@ -117,7 +117,7 @@ def test_gloo_world2_mapping_and_exchange():
 
 
 # ---------------------------------------------------------------- GPU (loopback ranks)
-def run_loopback(A, perm, R, values=None, b=None, split_all=True, **opts):
+def run_loopback(A, perm, R, values=None, b=None, split_all=True, junk_others=True, **opts):
     from paper_conf_ipps_georgesgsc11_b200.exchange import LoopbackHub
     hub = LoopbackHub(R)
     solvers = [mf.Solver(nranks=R, rank=r, exchange=hub.for_rank(r), split_all=split_all, **opts) for r in range(R)]
@@ -129,9 +129,10 @@ def run_loopback(A, perm, R, values=None, b=None, split_all=True, **opts):
 
     def work(r):
         try:
-            solvers[r].factor(vals)
+            # only rank 0's values / b are read (include/mf.h): the others pass junk
+            solvers[r].factor(vals if r == 0 or not junk_others else np.full_like(vals, np.nan))
             if b is not None:
-                xs[r] = solvers[r].solve(b)
+                xs[r] = solvers[r].solve(b if r == 0 or not junk_others else np.zeros_like(b))
         except Exception as e:  # noqa: BLE001
             errs[r] = e
     th = [threading.Thread(target=work, args=(r,)) for r in range(R)]

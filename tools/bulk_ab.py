@@ -21,7 +21,7 @@ if len(sys.argv) > 2 and sys.argv[2] == "child":
     inf = S.info()
     ld = f + (f & 1)
     tot = int(np.sum(ld * k)) + 2
-    Lx = S.export_L(tot)
+    Lx = S.export_panels(tot)
     off = np.concatenate([[0], np.cumsum(ld * k)])
     sums = np.array([np.abs(Lx[off[s]:off[s + 1]]).sum() for s in range(len(k))])
     import hashlib

@@ -18,7 +18,7 @@ if len(sys.argv) > 3 and sys.argv[3] == "child":
     sn = S.supernodes()
     k = np.diff(sn["sn_first"]); f = np.diff(sn["sn_rowptr"])
     ld = f + (f & 1)
-    Lx = S.export_L(int(np.sum(ld * k)) + 2)
+    Lx = S.export_panels(int(np.sum(ld * k)) + 2)
     np.save(sys.argv[4], Lx)
     np.savez(sys.argv[4] + ".meta.npz", k=k, f=f, par=sn["sn_parent"])
     sys.exit(0)
