@@ -44,6 +44,7 @@ def parse():
     ap.add_argument("--config", default="c5", choices=sorted(G.CONFIGS))
     ap.add_argument("--impl", default="mf", choices=["mf", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-modes", action="store_true", help="skip the Ozaki int8 Schur-update mode lines")
     ap.add_argument("--cpu-sample-gflop", type=float, default=170.0,
                     help="true GFLOP of the oracle sample (one whole subtree)")
     ap.add_argument("--small-front-max", type=int, default=None)
@@ -207,6 +208,65 @@ def run_reference(args):
     return 0
 
 
+# ------------------------------------------------------------------ Schur-update modes (NEXT-3)
+def int8_peak_tops() -> tuple[float, str]:
+    """Dense int8 tensor peak: MEASURED_PEAKS.json bf16 burst x 2 (the guide's
+    nominal int8 : bf16 ratio, 4.5 : 2.25 POPS), else the nominal 4.5 POPS."""
+    try:
+        bf16 = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["bf16_tflops"]
+        return 2.0 * bf16, "MEASURED_PEAKS.json bf16_tflops (burst) x 2 (nominal int8/bf16 ratio)"
+    except (OSError, ValueError, KeyError):
+        return 4500.0, "nominal 4.5 POPS dense int8 (no MEASURED_PEAKS.json)"
+
+
+def bench_mode(torch, mf, A, perm, vals_d, stream, slices: int, steps: int, warmup: int, b=None):
+    """One Schur-update mode (mf_options.ozaki_slices) on the same workload: device
+    time per factorization, the int8 tensor-core launches' roofline, and -- when
+    b is given -- the mixed-precision solve with fp64 refinement."""
+    S = mf.Solver(stream=stream.cuda_stream, ozaki_slices=slices)
+    S.analyze(A.n, A.colptr, A.rowind, perm)
+    for _ in range(max(warmup, 3)):
+        S.factor(vals_d)
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(steps):
+        S.factor(vals_d)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / steps
+    info = S.info()
+    S.set_profiling(True)
+    S.factor(vals_d)
+    prog, times = S.program(), S.launch_times()
+    S.set_profiling(False)
+    oz = [i for i, L in enumerate(prog) if L["int8_ops"] > 0]
+    t_oz = float(sum(times[i] for i in oz))
+    ops = float(sum(prog[i]["int8_ops"] for i in oz))
+    peak, src = int8_peak_tops()
+    out = {"ozaki_slices": slices, "ms_per_step": ms, "value": info["flops_true"] / (ms * 1e-3) / 1e9,
+           "unit": "GFLOP/s (fp64-equivalent, true-L flops)", "int8_launches": len(oz),
+           "int8_launch_ms": t_oz, "int8_share_of_step": t_oz / (S.info()["t_factor"] * 1e3),
+           "roofline_int8": {"bound": "tensor", "achieved": ops / (t_oz * 1e-3) / 1e12 if t_oz else None,
+                             "peak": peak, "unit": "TOPS (int8 MMA ops executed)",
+                             "frac": (ops / (t_oz * 1e-3) / 1e12) / peak if t_oz else None, "peak_source": src,
+                             "fp64_equiv_TFLOPs": float(sum(prog[i]["flops"] for i in oz)) / (t_oz * 1e-3) / 1e12
+                             if t_oz else None}}
+    if b is not None:
+        x = S.solve(b)
+        inf = S.info()
+        out["solve"] = {"refine_steps": inf["refine_steps"], "backward_error": inf["solve_berr"],
+                        "solve_ms": inf["t_solve"] * 1e3,
+                        "e2e_ms": ms + inf["t_solve"] * 1e3,
+                        "what": "factor (reduced-precision Schur updates) + solve with fp64 iterative refinement; "
+                                "backward error ||b-Ax||/(||A|| ||x|| + ||b||) (inf norms) computed on the GPU"}
+        del x
+    S.close()
+    torch.cuda.empty_cache()
+    return out
+
+
 # ------------------------------------------------------------------ product arm
 def main():
     args = parse()
@@ -360,6 +420,15 @@ def main():
         "kernels": [{k: (round(v, 4) if isinstance(v, float) else v) for k, v in s.items()} for s in stats],
         "profiled_ms_per_step": prof_ms,
     }
+    if world == 1 and not args.no_modes:
+        # NEXT-3 modes on the same workload (the fp64 DMMA line above is the headline)
+        S.close()
+        torch.cuda.empty_cache()
+        line["schur_modes"] = {
+            "ozaki8_fp64_emulated": bench_mode(torch, mf, A, perm, vals_d, stream, 8, args.steps, args.warmup),
+            "ozaki4_mixed_refined": bench_mode(torch, mf, A, perm, vals_d, stream, 4, args.steps, args.warmup,
+                                               b=G.rhs(A.n, 0)),
+        }
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         sym, subset, gflop, root = oracle_sample(A, perm, args.cpu_sample_gflop)
         times = run_oracle_steps(A, sym, subset, 1)

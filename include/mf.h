@@ -108,6 +108,23 @@ typedef struct {
     void *(*dev_alloc)(size_t bytes, void *alloc_user);
     void (*dev_free)(void *ptr, void *alloc_user);
     void *alloc_user;
+    /* Schur updates (the SYRK/GEMM of every large front) on the int8 tensor cores
+     * (tcgen05.mma .kind::i8, TMEM accumulators) by the Ozaki scheme: each row of
+     * the panel is scaled by a power of two and cut into ozaki_slices signed 7-bit
+     * digits; digit products are exact in int32 and recombined in fp64 (SURVEY.md
+     * NEXT-3; Sec. III-B: the paper's GPU part ran in single
+     * precision with double-precision refinement).
+     *   0 (default) = FP64 DMMA (mma.sync.m8n8k4.f64);
+     *   8 = FP64-class emulation (digit truncation 2^-56 of the row scales);
+     *   3..7 = reduced precision; mf_solve then refines in fp64 (refine_iters).
+     * Update launches with a short average inner dimension (< 2048, where DMMA
+     * measured faster) stay on DMMA.  Forces lookahead = 0. */
+    int32_t ozaki_slices;
+    /* mf_solve: maximum fp64 iterative-refinement steps x += A^{-1}(b - A x) with
+     * the residual in fp64 from the original values; stops when the backward error
+     * ||b - A x||_inf / (||A||_inf ||x||_inf + ||b||_inf) <= 2^-52 or stops
+     * decreasing.  -1 (default) = auto: 0 for ozaki_slices 0 or 8, else 10. */
+    int32_t refine_iters;
 } mf_options;
 
 typedef struct {
@@ -130,6 +147,10 @@ typedef struct {
     double t_factor;          /* seconds (device events) of the last mf_factor */
     double t_solve;           /* seconds (device events) of the last mf_solve */
     int32_t nbranch;          /* concurrent subtree branches the factorization uses (single GPU)   */
+    int32_t ozaki_slices;     /* Schur-update mode in use (mf_options.ozaki_slices)                 */
+    int32_t refine_steps;     /* refinement steps taken by the last mf_solve                        */
+    double solve_berr;        /* backward error of the last mf_solve's x when refinement ran, else -1 */
+    int64_t launches_ozaki;   /* Schur-update launches of mf_factor on the int8 tensor cores       */
 } mf_info;
 
 /* Per-kernel-class statistics of profiled factorizations (mf_set_profiling):
@@ -248,6 +269,8 @@ typedef struct {
     int64_t count;
     double flops;
     double bytes;
+    double int8_ops;   /* Schur update on the int8 tensor cores (ozaki_slices): int8 MMA
+                          operations executed (2 x MACs, padding included), else 0 */
 } mf_launch_info;
 
 /* out may be NULL to query *count only. */

@@ -67,6 +67,16 @@ struct mf_ctx {
     mf_kernel_stat kstats[KC_COUNT];
     int64_t prof_factors = 0;
     // device-memory hooks (mf_options.dev_alloc / dev_free; NULL = cudaMalloc / cudaFree)
+    // Ozaki-scheme Schur updates (ozaki_slices > 0): problem / tile / split lists, scratch
+    OzProb *d_oz_probs = nullptr;
+    OzTile *d_oz_tiles = nullptr;
+    int32_t *d_oz_split = nullptr;
+    int8_t *d_oz_scratch = nullptr;
+    int32_t *d_oz_expo = nullptr;
+    // fp64 iterative refinement (refine_iters > 0): symmetric CSR of B, B values, vectors
+    int64_t *d_rs_ptr = nullptr;
+    int32_t *d_rs_col = nullptr, *d_rs_ent = nullptr;
+    double *d_bval = nullptr, *d_rb = nullptr, *d_rx = nullptr, *d_norms = nullptr;
     void *(*halloc)(size_t, void *) = nullptr;
     void (*hfree)(void *, void *) = nullptr;
     void *huser = nullptr;
@@ -176,10 +186,17 @@ void fill_info(mf_ctx *c, int64_t n, int with_device) {
     I.nbranch = P.nbranch;
     I.rows_total = P.rows_total;
     I.failed_col = -1;
+    I.ozaki_slices = P.oz_slices;
+    I.refine_steps = 0;
+    I.solve_berr = -1.0;
+    I.launches_ozaki = 0;
+    for (const Launch &L : P.program) I.launches_ozaki += L.oz;
+    for (const Launch &L : P.program_top) I.launches_ozaki += L.oz;
     int64_t ws = 0;
     ws += (P.L_words + P.U_words + P.fv_words + 2 * std::max<int64_t>(n, 1) + S.nnz_in) * 8;
     ws += (int64_t)P.tiles.size() * sizeof(TileTask) + (int64_t)P.probs.size() * sizeof(GemmProb);
     ws += (int64_t)(S.bvidx.size() * 16 + S.brow.size() * 16 + P.relmap.size() * 4);
+    ws += P.oz_scratch_bytes + P.oz_expo_words * 4 + (int64_t)P.oz_tiles.size() * sizeof(OzTile);
     I.workspace_bytes = with_device ? ws : 0;
 }
 
@@ -222,6 +239,8 @@ int mf_default_options(mf_options *o) {
     o->dev_alloc = nullptr;
     o->dev_free = nullptr;
     o->alloc_user = nullptr;
+    o->ozaki_slices = 0;
+    o->refine_iters = -1;
     return MF_OK;
 }
 
@@ -255,6 +274,14 @@ int mf_create(mf_ctx **out, const mf_options *o) {
     c->opt.nbranch = o->nbranch;
     c->opt.fuse_ea = o->fuse_ea != 0;
     c->opt.lookahead = o->lookahead != 0;
+    if (o->ozaki_slices != 0 && (o->ozaki_slices < 3 || o->ozaki_slices > 8)) {
+        delete c;
+        return MF_ERR_ARG;
+    }
+    c->opt.ozaki_slices = o->ozaki_slices;
+    c->opt.refine_iters = o->refine_iters < 0 ? ((o->ozaki_slices == 0 || o->ozaki_slices == 8) ? 0 : 10)
+                                              : o->refine_iters;
+    if (c->opt.ozaki_slices) c->opt.lookahead = 0;   // the Ozaki scratch is per stream: no side stream
     c->opt.rank = o->rank;
     c->host_only = o->host_only != 0;
     if ((o->dev_alloc == nullptr) != (o->dev_free == nullptr)) {
@@ -347,6 +374,7 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     const Plan &P = c->P;
     DevPlan &d = c->d;
     int r;
+    void *p0 = nullptr;
 #define UP(dst, vec)                                   \
     if ((r = dev_upload(c, dst, vec)) != MF_OK) return r;
     int32_t *sn_first, *sn_k, *sn_f, *sn_ld, *child_ptr, *child_list, *relmap, *blrow, *perm_d;
@@ -386,6 +414,51 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     UP(&ea_qs, P.ea_qs);
     UP(&c->d_top_list, P.top_list);
     UP(&c->d_own_list, P.own_list);
+    UP(&c->d_oz_probs, P.oz_probs);
+    UP(&c->d_oz_tiles, P.oz_tiles);
+    UP(&c->d_oz_split, P.oz_split);
+    if (c->opt.refine_iters > 0) {
+        // row k of B = P A P^T (final labels): (column, entry) of every stored entry of
+        // row k and of column k -- the residual of the refinement walks whole rows
+        const int64_t nb = (int64_t)S.brow.size();
+        std::vector<int64_t> rp(n + 1, 0);
+        for (int64_t j = 0; j < n; j++)
+            for (int64_t e = S.bcolptr[j]; e < S.bcolptr[j + 1]; e++) {
+                rp[S.brow[e] + 1]++;
+                if (S.brow[e] != j) rp[j + 1]++;
+            }
+        for (int64_t k = 0; k < n; k++) rp[k + 1] += rp[k];
+        std::vector<int32_t> rc(rp[n]), re(rp[n]);
+        std::vector<int64_t> fill(rp.begin(), rp.end() - 1);
+        for (int64_t j = 0; j < n; j++)
+            for (int64_t e = S.bcolptr[j]; e < S.bcolptr[j + 1]; e++) {
+                const int32_t i = S.brow[e];
+                rc[fill[i]] = (int32_t)j;
+                re[fill[i]++] = (int32_t)e;
+                if (i != j) {
+                    rc[fill[j]] = i;
+                    re[fill[j]++] = (int32_t)e;
+                }
+            }
+        if (nb >= INT32_MAX) return MF_ERR_ARG;
+        UP(&c->d_rs_ptr, rp);
+        UP(&c->d_rs_col, rc);
+        UP(&c->d_rs_ent, re);
+        if ((r = dev_alloc(c, &p0, (size_t)std::max<int64_t>(nb, 1) * sizeof(double)))) return r;
+        c->d_bval = (double *)p0;
+        if ((r = dev_alloc(c, &p0, (size_t)std::max<int64_t>(n, 1) * sizeof(double)))) return r;
+        c->d_rb = (double *)p0;
+        if ((r = dev_alloc(c, &p0, (size_t)std::max<int64_t>(n, 1) * sizeof(double)))) return r;
+        c->d_rx = (double *)p0;
+        if ((r = dev_alloc(c, &p0, 4 * sizeof(double)))) return r;
+        c->d_norms = (double *)p0;
+    }
+    if (P.oz_slices > 0) {
+        if ((r = dev_alloc(c, &p0, (size_t)std::max<int64_t>(P.oz_scratch_bytes, 16)))) return r;
+        c->d_oz_scratch = (int8_t *)p0;
+        if ((r = dev_alloc(c, &p0, (size_t)std::max<int64_t>(P.oz_expo_words, 4) * sizeof(int32_t)))) return r;
+        c->d_oz_expo = (int32_t *)p0;
+    }
 #undef UP
     d.sn_first = sn_first;
     d.sn_k = sn_k;
@@ -537,8 +610,13 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
                 case KC_POTRF: launch_potrf_diag(d, c->d_large + L.off, (int)L.count, L.param, P.w, st); break;
                 case KC_TRSM: launch_trsm_panel(d, c->d_trsm + 2 * L.off, L.count, L.param, P.w, st); break;
                 case KC_UPDATE:   // long-K launches of many waves take the bulk-copy pipeline
-                    launch_update(d, c->d_probs, c->d_tiles + L.off, L.count,
-                                  L.count > 0 ? L.flops / (2.0 * kTileM * kTileN * L.count) : 0.0, st);
+                    if (L.oz)   // int8 tensor cores, Ozaki scheme
+                        launch_update_oz(d, c->d_probs, c->d_oz_probs, c->d_oz_split + 3 * L.oz_s, L.oz_ns,
+                                         c->d_oz_tiles + L.oz_t, L.oz_nt, c->d_oz_scratch, c->d_oz_expo + L.oz_e,
+                                         L.oz_ne, P.oz_slices, st);
+                    else
+                        launch_update(d, c->d_probs, c->d_tiles + L.off, L.count,
+                                      L.count > 0 ? L.flops / (2.0 * kTileM * kTileN * L.count) : 0.0, st);
                     break;
                 case KC_PANEL: launch_panel(d, c->d_panel + 2 * L.off, L.count, L.param, (int)L.count2, st); break;
                 case KC_LEAF:
@@ -706,6 +784,7 @@ int mf_factor(mf_ctx *c, const double *values) {
         std::vector<mf_xfer> red{mf_xfer{MF_XFER_ALLREDUCE_MIN_I32, 0, c->d_failed, (int64_t)sizeof(int)}};
         if ((r = exchange(c, red))) return r;
     }
+    if (c->d_bval) launch_refine_bval(c->d, vals, c->d_bval, (int64_t)c->S.brow.size(), st);   // for mf_solve's residuals
     CK(cudaGetLastError());
     int failed = INT_MAX;
     CK(cudaMemcpyAsync(&failed, c->d_failed, sizeof(int), cudaMemcpyDeviceToHost, st));
@@ -784,7 +863,34 @@ int mf_solve(mf_ctx *c, const double *b, double *x) {
             CK(cudaGraphInstantiate(&c->solve_exec, g, 0));
         }
         CK(cudaGraphLaunch(c->solve_exec, st));
-        CK(cudaMemcpyAsync(x, c->d_bx, n * sizeof(double), xdev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
+        const double *xsrc = c->d_bx;
+        if (c->opt.refine_iters > 0 && c->d_rx) {
+            // fp64 iterative refinement on the (reduced-precision) factor: r = b - A x
+            // with the caller's values, dx = A^{-1} r through the same solve graph
+            CK(cudaMemcpyAsync(c->d_rb, b, n * sizeof(double), bdev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice,
+                               st));
+            CK(cudaMemcpyAsync(c->d_rx, c->d_bx, n * sizeof(double), cudaMemcpyDeviceToDevice, st));
+            double prev = 1e300, berr = 0.0;
+            int steps = 0;
+            for (;;) {
+                launch_refine_resid(d, c->d_rs_ptr, c->d_rs_col, c->d_rs_ent, c->d_bval, c->d_rb, c->d_rx, c->d_bx,
+                                    c->d_norms, n, st);
+                double nrm[4];
+                CK(cudaMemcpyAsync(nrm, c->d_norms, sizeof nrm, cudaMemcpyDeviceToHost, st));
+                CK(cudaStreamSynchronize(st));
+                const double den = nrm[3] * nrm[1] + nrm[2];
+                berr = den > 0 ? nrm[0] / den : 0.0;
+                if (berr <= 0x1p-52 || steps >= c->opt.refine_iters || berr > 0.5 * prev) break;
+                prev = berr;
+                CK(cudaGraphLaunch(c->solve_exec, st));   // d_bx: r -> dx
+                launch_refine_axpy(c->d_rx, c->d_bx, n, st);
+                steps++;
+            }
+            c->info.refine_steps = steps;
+            c->info.solve_berr = berr;
+            xsrc = c->d_rx;
+        }
+        CK(cudaMemcpyAsync(x, xsrc, n * sizeof(double), xdev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
                            st));
         CK(cudaGetLastError());
         CK(cudaEventRecord(c->ev1, st));
@@ -852,7 +958,7 @@ int mf_solve_nrhs(mf_ctx *c, int32_t nrhs, const double *B, int64_t ldb, double 
     if (nrhs == 0) return MF_OK;
     if (!B || !X || ldb < n || ldx < n) return MF_ERR_ARG;
     if ((const void *)B == (const void *)X) return MF_ERR_ARG;
-    if (c->P.nranks > 1 || !c->use_graph) {   // one column at a time through mf_solve
+    if (c->P.nranks > 1 || !c->use_graph || c->opt.refine_iters > 0) {   // one column at a time through mf_solve
         for (int32_t r = 0; r < nrhs; r++)
             if (int e = mf_solve(c, B + r * ldb, X + r * ldx)) return e;
         return MF_OK;
@@ -974,7 +1080,8 @@ int mf_get_program(const mf_ctx *c, mf_launch_info *out, int64_t max, int64_t *c
     *count = (int64_t)prog.size();
     if (out)
         for (int64_t i = 0; i < std::min<int64_t>(max, (int64_t)prog.size()); i++)
-            out[i] = mf_launch_info{prog[i].kind, prog[i].level, prog[i].count, prog[i].flops, prog[i].bytes};
+            out[i] = mf_launch_info{prog[i].kind, prog[i].level, prog[i].count, prog[i].flops, prog[i].bytes,
+                                    prog[i].int8_ops};
     return MF_OK;
 }
 

@@ -12,12 +12,14 @@
 // Determinism: extend-add has no atomics; every destination entry receives
 // 0, then its A value, then the children's contributions in ascending child
 // order (reading C6) -- the same summation order as the oracle.
+#include <algorithm>
 #include <cstdlib>
 #include <climits>
 #include <cstdio>
 
 #include "dmma_update.cuh"
 #include "kernels.cuh"
+#include "ozaki_update.cuh"
 
 namespace mf {
 
@@ -1312,7 +1314,28 @@ int kernels_init() {
     if (e == cudaSuccess)
         e = cudaFuncSetAttribute(k_update_t<UpdLowK, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  (int)UpdLowK::SMEM);
+    if (e == cudaSuccess) e = oz_set_attr<3>();
+    if (e == cudaSuccess) e = oz_set_attr<4>();
+    if (e == cudaSuccess) e = oz_set_attr<5>();
+    if (e == cudaSuccess) e = oz_set_attr<6>();
+    if (e == cudaSuccess) e = oz_set_attr<7>();
+    if (e == cudaSuccess) e = oz_set_attr<8>();
     return e == cudaSuccess ? 0 : -1;
+}
+
+// Ozaki-scheme Schur update of one KC_UPDATE launch (S = slices, 3..8)
+void launch_update_oz(const DevPlan &d, const GemmProb *probs, const OzProb *oprobs, const int32_t *split,
+                      int64_t nsplit, const OzTile *tiles, int64_t ntiles, int8_t *scratch, int32_t *expo,
+                      int64_t expo_words, int S, cudaStream_t st) {
+    const UpdGather gv{d.child_ptr, d.child_list, d.sn_k, d.sn_f, d.U_off, d.relmap_ptr, d.relmap, d.ea_qs};
+    switch (S) {
+        case 3: launch_oz<3>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv); break;
+        case 4: launch_oz<4>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv); break;
+        case 5: launch_oz<5>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv); break;
+        case 6: launch_oz<6>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv); break;
+        case 7: launch_oz<7>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv); break;
+        default: launch_oz<8>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv); break;
+    }
 }
 
 // diag(L) in final labels (one warp per supernode)
@@ -1707,4 +1730,79 @@ void launch_bwd_solve(const DevPlan &d, const int32_t *list, int count, double *
     if (count > 0) k_bwd_solve<<<count, kSolveThreads, 0, st>>>(d, list, y, sn_rows, sn_rowptr);
 }
 
+}  // namespace mf
+
+// ============================================================ fp64 iterative refinement
+// (mixed-precision mode; "single precision on the
+// GPU ... iterative refinement in double precision")  r = b - A x in fp64 from the
+// caller's values, in ORIGINAL labels (rows / columns reached through the final
+// perm), over the symmetric CSR of B = P A P^T built at analyze time: row k lists
+// (column k', B entry e) for every stored entry of row k and of column k.
+namespace mf {
+// bval[e] = sum of the caller's values of B entry e, in input order (reading C6)
+__global__ void k_refine_bval(const int64_t *__restrict__ bvptr, const int64_t *__restrict__ bvidx,
+                              const double *__restrict__ values, double *__restrict__ bval, int64_t nb) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < nb; e += (int64_t)gridDim.x * blockDim.x) {
+        double v = 0.0;
+        for (int64_t q = bvptr[e]; q < bvptr[e + 1]; q++) v += values[bvidx[q]];
+        bval[e] = v;
+    }
+}
+__device__ __forceinline__ void atomic_max_nonneg(double *addr, double v) {
+    // non-negative doubles order like their bit patterns
+    atomicMax(reinterpret_cast<unsigned long long *>(addr), (unsigned long long)__double_as_longlong(v));
+}
+// r = b - A x (original labels); norms[0] = ||r||, [1] = ||x||, [2] = ||b||, [3] = ||A|| (inf norms)
+__global__ void k_refine_resid(const int64_t *__restrict__ rs_ptr, const int32_t *__restrict__ rs_col,
+                               const int32_t *__restrict__ rs_ent, const double *__restrict__ bval,
+                               const int32_t *__restrict__ perm, const double *__restrict__ b,
+                               const double *__restrict__ x, double *__restrict__ r, double *__restrict__ norms,
+                               int64_t n) {
+    double mr = 0.0, mx = 0.0, mb = 0.0, ma = 0.0;
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t i = perm[k];
+        double ax = 0.0, aa = 0.0;
+        for (int64_t q = rs_ptr[k]; q < rs_ptr[k + 1]; q++) {
+            const double v = bval[rs_ent[q]];
+            ax = fma(v, x[perm[rs_col[q]]], ax);
+            aa += fabs(v);
+        }
+        const double ri = b[i] - ax;
+        r[i] = ri;
+        mr = fmax(mr, fabs(ri));
+        mx = fmax(mx, fabs(x[i]));
+        mb = fmax(mb, fabs(b[i]));
+        ma = fmax(ma, aa);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        mr = fmax(mr, __shfl_xor_sync(0xffffffffu, mr, o));
+        mx = fmax(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        mb = fmax(mb, __shfl_xor_sync(0xffffffffu, mb, o));
+        ma = fmax(ma, __shfl_xor_sync(0xffffffffu, ma, o));
+    }
+    if ((threadIdx.x & 31) == 0) {
+        atomic_max_nonneg(norms + 0, mr);
+        atomic_max_nonneg(norms + 1, mx);
+        atomic_max_nonneg(norms + 2, mb);
+        atomic_max_nonneg(norms + 3, ma);
+    }
+}
+__global__ void k_refine_axpy(double *__restrict__ x, const double *__restrict__ dx, int64_t n) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        x[i] += dx[i];
+}
+static unsigned grid_for(int64_t n) { return (unsigned)std::max<int64_t>(1, std::min<int64_t>((n + 255) / 256, 148 * 8)); }
+void launch_refine_bval(const DevPlan &d, const double *values, double *bval, int64_t nb, cudaStream_t st) {
+    if (nb > 0) k_refine_bval<<<grid_for(nb), 256, 0, st>>>(d.bvptr, d.bvidx, values, bval, nb);
+}
+void launch_refine_resid(const DevPlan &d, const int64_t *rs_ptr, const int32_t *rs_col, const int32_t *rs_ent,
+                         const double *bval, const double *b, const double *x, double *r, double *norms, int64_t n,
+                         cudaStream_t st) {
+    cudaMemsetAsync(norms, 0, 4 * sizeof(double), st);
+    if (n > 0) k_refine_resid<<<grid_for(n), 256, 0, st>>>(rs_ptr, rs_col, rs_ent, bval, d.perm, b, x, r, norms, n);
+}
+void launch_refine_axpy(double *x, const double *dx, int64_t n, cudaStream_t st) {
+    if (n > 0) k_refine_axpy<<<grid_for(n), 256, 0, st>>>(x, dx, n);
+}
 }  // namespace mf

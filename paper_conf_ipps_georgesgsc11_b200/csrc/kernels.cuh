@@ -54,6 +54,16 @@ constexpr double kBulkMinK = 512;
 constexpr double kLowKMax = 256;
 void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tiles, int64_t ntiles, double kavg,
                    cudaStream_t st);
+// Schur update of one launch on the int8 tensor cores (Ozaki scheme, S slices)
+void launch_update_oz(const DevPlan &d, const GemmProb *probs, const OzProb *oprobs, const int32_t *split,
+                      int64_t nsplit, const OzTile *tiles, int64_t ntiles, int8_t *scratch, int32_t *expo,
+                      int64_t expo_words, int S, cudaStream_t st);
+// fp64 iterative refinement (mixed-precision mode): B entry values, residual + norms, x += dx
+void launch_refine_bval(const DevPlan &d, const double *values, double *bval, int64_t nb, cudaStream_t st);
+void launch_refine_resid(const DevPlan &d, const int64_t *rs_ptr, const int32_t *rs_col, const int32_t *rs_ent,
+                         const double *bval, const double *b, const double *x, double *r, double *norms, int64_t n,
+                         cudaStream_t st);
+void launch_refine_axpy(double *x, const double *dx, int64_t n, cudaStream_t st);
 void launch_permute_in(const DevPlan &d, const double *b, double *y, int64_t n, cudaStream_t st);
 void launch_permute_out(const DevPlan &d, const double *xf, double *x, int64_t n, cudaStream_t st);
 void launch_fwd_solve(const DevPlan &d, const int32_t *list, int count, double *y, cudaStream_t st);

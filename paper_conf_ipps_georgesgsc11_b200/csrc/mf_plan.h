@@ -30,6 +30,11 @@ struct Options {
     // front-order thresholds.  force_variant >= 0 forces that class wherever feasible.
     std::vector<double> variant_theta;
     int force_variant = -1;
+    // Schur updates on the int8 tensor cores (Ozaki scheme):
+    // 0 = FP64 DMMA; 8 = FP64-class emulation; 3..7 = reduced precision (mf_solve
+    // then refines in fp64).  refine_iters: max refinement steps (-1 = auto).
+    int ozaki_slices = 0;
+    int refine_iters = -1;
 };
 
 // Kernel variants a front can be factored with (the GPU-only policy classes that
@@ -112,6 +117,25 @@ struct TileTask {       // one kTileM x kTileN output tile of a GemmProb
     int32_t tij;        // (ti << 16) | tj
 };
 
+constexpr int kOzBM = 128, kOzBN = 64, kOzBK = 64;   // Ozaki tile rows, tile columns, int8 k per stage
+constexpr int kOzMaxK = 16000;                       // int32-exact inner dimension (S <= 8)
+constexpr int kOzSeg = 256;                          // k values per split task
+// Ozaki-scheme form of a GemmProb (csrc/ozaki_update.cuh): its A rows are cut into
+// int8 digit slices in a per-stream scratch before the int8 tensor-core update.
+struct OzProb {
+    int32_t prob;       // GemmProb index
+    int32_t Mpad;       // rows padded to kOzBM (128)
+    int32_t Kpad;       // inner dimension padded to kOzBK (64)
+    int32_t pad_;
+    int64_t sl_off;     // byte offset of its slices in the scratch: [S][Kpad/16][Mpad][16 bytes]
+    int64_t ex_off;     // int32 offset of its row exponents E_i
+};
+static_assert(sizeof(OzProb) == 32, "OzProb layout");
+struct OzTile {         // one 128 x 64 output tile
+    int32_t oprob;
+    int32_t tij;        // (ti << 16) | tj
+};
+
 // The factorization is a static launch program built once per pattern
 // (mf_analyze) and replayed by every mf_factor.
 enum KernelClass : int32_t {
@@ -153,6 +177,12 @@ struct Launch {
     // side stream, forked from the main stream at this point; join = 1 makes the
     // main stream wait for the side stream before this launch
     int32_t side = 0, join = 0;
+    // KC_UPDATE on the int8 tensor cores (Ozaki): oprobs [oz_p, oz_p + oz_np), split
+    // tasks (triples) [oz_s, oz_s + oz_ns), tiles [oz_t, oz_t + oz_nt); exponent
+    // words [oz_e, oz_e + oz_ne) of the scratch
+    int32_t oz = 0;
+    double int8_ops = 0;   // int8 MMA operations of an Ozaki launch
+    int64_t oz_p = 0, oz_np = 0, oz_s = 0, oz_ns = 0, oz_t = 0, oz_nt = 0, oz_e = 0, oz_ne = 0;
 };
 
 // Triangular-solve program (forward sweep bottom-up, backward sweep top-down).
@@ -217,6 +247,12 @@ struct Plan {
     std::vector<Launch> program_top;                 // every rank: top supernodes, with exchange points
     std::vector<std::vector<XferSpec>> xfers;        // transfer groups of the KC_EXCHANGE entries
     std::vector<SolveLaunch> fsolve_top, bsolve_top; // rank 0: top supernodes
+    // ---- Ozaki-scheme Schur updates (ozaki_slices > 0)
+    int32_t oz_slices = 0;
+    std::vector<OzProb> oz_probs;
+    std::vector<OzTile> oz_tiles;
+    std::vector<int32_t> oz_split;                   // (oprob, 128-row block, k segment) triples
+    int64_t oz_scratch_bytes = 0, oz_expo_words = 0; // per-stream regions, summed
     std::vector<int32_t> top_list, own_list;         // supernode lists (copy / mask kernels)
 };
 

@@ -17,6 +17,7 @@
 #include <algorithm>
 #include <cstdlib>
 #include <map>
+#include <set>
 #include <cmath>
 #include <functional>
 #include <numeric>
@@ -409,6 +410,93 @@ static void plan_u_reuse(Plan &P) {
     run_group(-1);
     for (int32_t s = 0; s < ns; s++) P.U_off[s] = off[s] >= 0 ? off[s] : 0;
     P.U_words = hw + 2;
+}
+
+// Ozaki-scheme Schur updates (csrc/ozaki_update.cuh): every
+// KC_UPDATE launch whose average inner dimension is long enough for the int8
+// tensor cores to beat FP64 DMMA (the split pass and the TMEM epilogue are paid
+// per launch and per tile) is given an Ozaki form: its problems (rows padded to
+// 128, K to 64), the (problem, 128-row block, k segment) split tasks and its
+// 128 x 64 tiles -- the union of its 64 x 64 DMMA tiles, so partial tile sets
+// (multi-GPU column ownership) carry over.  Slices live in a scratch region per
+// stream (branches run concurrently), sized for the largest launch of the stream.
+constexpr double kOzMinK = 2048;   // measured per launch on c5 (tools/oz_launches.py): DMMA wins below
+static int plan_ozaki(Plan &P, int S) {
+    P.oz_slices = S;
+    if (S <= 0) return MF_OK;
+    auto up = [](int64_t x, int64_t a) { return (x + a - 1) / a * a; };
+    std::map<int32_t, std::pair<int64_t, int64_t>> region;   // stream -> (slice bytes, exponent words)
+    std::vector<std::pair<std::vector<Launch> *, size_t>> conv;
+    double min_k = kOzMinK;   // MF_OZ_MIN_K: tests drive small problems through the int8 path
+    if (const char *e = getenv("MF_OZ_MIN_K")) min_k = atof(e);
+    for (std::vector<Launch> *prog : {&P.program, &P.program_top}) {
+        for (size_t li = 0; li < prog->size(); li++) {
+            Launch &L = (*prog)[li];
+            if (L.kind != KC_UPDATE || L.count == 0) continue;
+            if (L.flops / (2.0 * kTileM * kTileN * L.count) < min_k) continue;
+            std::vector<int32_t> probs;
+            std::map<int32_t, int32_t> local;
+            bool ok = true;
+            for (int64_t t = L.off; t < L.off + L.count; t++) {
+                const int32_t p = P.tiles[t].prob;
+                if (local.emplace(p, (int32_t)probs.size()).second) probs.push_back(p);
+            }
+            for (int32_t p : probs)
+                if (P.probs[p].K > kOzMaxK) ok = false;
+            if (!ok) continue;
+            L.oz = 1;
+            L.oz_p = (int64_t)P.oz_probs.size();
+            L.oz_np = (int64_t)probs.size();
+            int64_t bytes = 0, words = 0;
+            for (int32_t p : probs) {
+                const GemmProb &g = P.probs[p];
+                OzProb o{p, (int32_t)up(g.M, kOzBM), (int32_t)up(g.K, kOzBK), 0, bytes, words};
+                bytes += (int64_t)S * o.Mpad * o.Kpad;
+                words += o.Mpad;
+                P.oz_probs.push_back(o);
+            }
+            L.oz_s = (int64_t)P.oz_split.size() / 3;
+            for (int64_t q = 0; q < L.oz_np; q++) {
+                const OzProb &o = P.oz_probs[L.oz_p + q];
+                for (int32_t rb = 0; rb < o.Mpad / kOzBM; rb++)
+                    for (int32_t sg = 0; sg < (o.Kpad + kOzSeg - 1) / kOzSeg; sg++)
+                        P.oz_split.insert(P.oz_split.end(), {(int32_t)(L.oz_p + q), rb, sg});
+            }
+            L.oz_ns = (int64_t)P.oz_split.size() / 3 - L.oz_s;
+            L.oz_t = (int64_t)P.oz_tiles.size();
+            std::set<std::pair<int32_t, int32_t>> seen;
+            for (int64_t t = L.off; t < L.off + L.count; t++) {
+                const TileTask &tt = P.tiles[t];
+                const int32_t q = local[tt.prob], tij = (((tt.tij >> 16) * kTileM / kOzBM) << 16) | (tt.tij & 0xffff);
+                static_assert(kTileN == kOzBN, "Ozaki tiles keep the DMMA tile columns");
+                if (seen.emplace(q, tij).second) P.oz_tiles.push_back(OzTile{(int32_t)(L.oz_p + q), tij});
+            }
+            L.oz_nt = (int64_t)P.oz_tiles.size() - L.oz_t;
+            for (int64_t t = L.oz_t; t < L.oz_t + L.oz_nt; t++)
+                L.int8_ops += 2.0 * kOzBM * kOzBN * (double)P.oz_probs[P.oz_tiles[t].oprob].Kpad * (S * (S + 1) / 2);
+            L.oz_ne = words;
+            auto &rg = region[L.stream];
+            rg.first = std::max(rg.first, bytes);
+            rg.second = std::max(rg.second, words);
+            conv.emplace_back(prog, li);
+        }
+    }
+    std::map<int32_t, std::pair<int64_t, int64_t>> base;
+    int64_t tb = 0, tw = 0;
+    for (auto &kv : region) {
+        base[kv.first] = {tb, tw};
+        tb += up(kv.second.first, 1024);
+        tw += up(kv.second.second, 32);
+    }
+    for (auto &c : conv) {
+        Launch &L = (*c.first)[c.second];
+        const auto b = base[L.stream];
+        for (int64_t q = L.oz_p; q < L.oz_p + L.oz_np; q++) P.oz_probs[q].sl_off += b.first;
+        L.oz_e = b.second;   // ex_off stays relative to the launch's exponent region
+    }
+    P.oz_scratch_bytes = tb;
+    P.oz_expo_words = tw;
+    return MF_OK;
 }
 
 int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
@@ -822,7 +910,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     for (const Pass &pass : passes) {
     const std::vector<char> &inc = pass.inc;
     cur = pass.prog;
-    lookahead_pass = opt.lookahead && R == 1 && pass.stream < 0;
+    lookahead_pass = opt.lookahead && opt.ozaki_slices == 0 && R == 1 && pass.stream < 0;
     const size_t pass_begin = cur->size();
     for (int32_t l = 0; l < nlev; l++) {
         std::vector<int32_t> fronts;
@@ -999,7 +1087,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     P.df_part_off.assign(ns, -1);
     build_solve_plan(S, P, inc_local, P.fsolve, P.bsolve);
     build_solve_plan(S, P, inc_top_solve, P.fsolve_top, P.bsolve_top);
-    return MF_OK;
+    return plan_ozaki(P, opt.ozaki_slices);
 }
 
 }  // namespace mf

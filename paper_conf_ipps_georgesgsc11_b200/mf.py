@@ -41,6 +41,7 @@ class Options(ctypes.Structure):
         ("stream", ctypes.c_void_p), ("split_all", ctypes.c_int32), ("nbranch", ctypes.c_int32),
         ("fuse_ea", ctypes.c_int32), ("lookahead", ctypes.c_int32),
         ("dev_alloc", ctypes.c_void_p), ("dev_free", ctypes.c_void_p), ("alloc_user", ctypes.c_void_p),
+        ("ozaki_slices", ctypes.c_int32), ("refine_iters", ctypes.c_int32),
     ]
 
 
@@ -56,7 +57,8 @@ class Info(ctypes.Structure):
         ("nlevels", ctypes.c_int32), ("max_front", ctypes.c_int32), ("rows_total", ctypes.c_int64),
         ("failed_col", ctypes.c_int64), ("workspace_bytes", ctypes.c_int64), ("launches_factor", ctypes.c_int64),
         ("t_analyze", ctypes.c_double), ("t_factor", ctypes.c_double), ("t_solve", ctypes.c_double),
-        ("nbranch", ctypes.c_int32),
+        ("nbranch", ctypes.c_int32), ("ozaki_slices", ctypes.c_int32), ("refine_steps", ctypes.c_int32),
+        ("solve_berr", ctypes.c_double), ("launches_ozaki", ctypes.c_int64),
     ]
 
     def as_dict(self) -> dict:
@@ -82,7 +84,7 @@ EXCHANGE_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.POINTER(Xfe
 
 class LaunchInfo(ctypes.Structure):
     _fields_ = [("kind", ctypes.c_int32), ("level", ctypes.c_int32), ("count", ctypes.c_int64),
-                ("flops", ctypes.c_double), ("bytes", ctypes.c_double)]
+                ("flops", ctypes.c_double), ("bytes", ctypes.c_double), ("int8_ops", ctypes.c_double)]
 
 
 def lib_path() -> str:
@@ -165,7 +167,8 @@ class Solver:
                  device: int = -1, stream: int | None = None, host_only: bool = False,
                  nranks: int = 1, rank: int = 0, exchange=None, split_all: bool = False,
                  nbranch: int | None = None, fuse_ea: bool | None = None, lookahead: bool | None = None,
-                 variant_model="auto", torch_alloc: bool = False):
+                 variant_model="auto", torch_alloc: bool = False, ozaki_slices: int = 0,
+                 refine_iters: int | None = None):
         """variant_model: "auto" = the fitted kernel-variant selector packaged with the
         binding (selector.MODEL_PATH, Eqs. 3-5 fitted to B200 timings) when
         present, None = libmf's fixed front-order thresholds, or a theta array.
@@ -173,7 +176,10 @@ class Solver:
         ("auto" then resolves to None), since a variant model chooses each front's
         class by itself and would ignore the threshold (include/mf.h).
         torch_alloc: take every device buffer of the ctx from PyTorch's caching
-        allocator (mf_options.dev_alloc / dev_free) instead of cudaMalloc."""
+        allocator (mf_options.dev_alloc / dev_free) instead of cudaMalloc.
+        ozaki_slices: Schur updates on the int8 tensor cores (0 = FP64 DMMA, 8 =
+        FP64-class Ozaki emulation, 3..7 = reduced precision + fp64 refinement in
+        solve); refine_iters: max refinement steps (None = auto)."""
         if small_front_max is not None and isinstance(variant_model, str) and variant_model == "auto":
             variant_model = None
         o = Options()
@@ -195,6 +201,8 @@ class Solver:
         if lookahead is not None:
             o.lookahead = int(lookahead)
         o.stream = stream
+        o.ozaki_slices = int(ozaki_slices)
+        o.refine_iters = -1 if refine_iters is None else int(refine_iters)
         self._alloc_cbs = None
         if torch_alloc and not host_only:
             import torch
@@ -344,7 +352,8 @@ class Solver:
         self._check(lib.mf_get_program(self._h, None, 0, ctypes.byref(cnt)), "mf_get_program")
         arr = (LaunchInfo * max(cnt.value, 1))()
         self._check(lib.mf_get_program(self._h, arr, cnt.value, ctypes.byref(cnt)), "mf_get_program")
-        return [dict(kind=a.kind, level=a.level, count=a.count, flops=a.flops, bytes=a.bytes) for a in arr[:cnt.value]]
+        return [dict(kind=a.kind, level=a.level, count=a.count, flops=a.flops, bytes=a.bytes, int8_ops=a.int8_ops)
+                for a in arr[:cnt.value]]
 
     def launch_times(self) -> np.ndarray:
         """CUDA-event ms of every launch of the last profiled factorization (program order)."""
