@@ -46,7 +46,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-modes", action="store_true", help="skip the Ozaki int8 Schur-update mode lines")
     ap.add_argument("--cpu-sample-gflop", type=float, default=170.0,
-                    help="true GFLOP of the oracle sample (one whole subtree)")
+                    help="--impl reference: true GFLOP of the oracle sample per step (one whole subtree)")
+    ap.add_argument("--cpu-baseline-gflop", type=float, default=1500.0,
+                    help="cpu_baseline of the product arm: true GFLOP of its one-off oracle sample (~10-30 s)")
     ap.add_argument("--small-front-max", type=int, default=None)
     ap.add_argument("--panel-w", type=int, default=None)
     ap.add_argument("--nbranch", type=int, default=None, help="concurrent subtree branches (single GPU)")
@@ -171,14 +173,48 @@ def run_oracle_steps(A, sym, subset, steps: int):
 
 
 def cpu_cores() -> int:
+    """Threads the oracle's OpenMP loops use (oracle/numeric.c: the default team,
+    OMP_NUM_THREADS or every host core)."""
+    env = os.environ.get("OMP_NUM_THREADS")
+    return int(env) if env and env.isdigit() else (len(os.sched_getaffinity(0)) or 1)
+
+
+def cpu_model() -> str:
     try:
-        from threadpoolctl import threadpool_info
-        th = [i.get("num_threads", 0) for i in threadpool_info() if i.get("user_api") == "blas"]
-        if th:
-            return int(max(th))
-    except Exception:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except OSError:
         pass
-    return os.cpu_count() or 1
+    return "unknown"
+
+
+def single_thread_reference() -> dict | None:
+    """Single-thread oracle seconds for c1-c3 (tools/oracle_single_thread.py on
+    the GPU box's host, committed under profiles/): a fixed measurement, not
+    re-run by every bench."""
+    try:
+        return json.load(open(os.path.join(ROOT, "profiles", "oracle_single_thread.json")))
+    except (OSError, ValueError):
+        return None
+
+
+def traffic_for(cfg: str, kernel: str, launches_per_step: int):
+    """ncu DRAM bytes per launch of `kernel` for THIS program (profiles/ncu_traffic_<cfg>.json,
+    tools/gpu/profile.sh) -- refused when the capture's launch count differs from
+    the benched program's."""
+    path = os.path.join(ROOT, "profiles", f"ncu_traffic_{cfg}.json")
+    try:
+        prof = json.load(open(path))
+    except (OSError, ValueError):
+        return None, f"no {os.path.basename(path)}"
+    k = prof.get("kernels", {}).get(kernel)
+    if not k:
+        return None, f"{kernel} not in {os.path.basename(path)}"
+    if k.get("launches") != launches_per_step:
+        return None, (f"{os.path.basename(path)} has {k.get('launches')} {kernel} launches, "
+                      f"the benched program {launches_per_step}: stale capture refused")
+    return k["dram_bytes_per_launch"], os.path.basename(path)
 
 
 # ------------------------------------------------------------------ reference arm
@@ -200,7 +236,8 @@ def run_reference(args):
         "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": c["desc"] + f" [{args.config}], CPU oracle sample", "n": A.n},
-        "cpu_baseline": {"value": value, "unit": "GFLOP/s", "cores": cpu_cores(), "kind": "oracle", "sample": sample},
+        "cpu_baseline": {"value": value, "unit": "GFLOP/s", "cores": cpu_cores(), "kind": "oracle", "sample": sample,
+                         "cpu_model": cpu_model()},
         "e2e": {"value": value, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
         "gpu_launches": 0,
     }
@@ -371,16 +408,12 @@ def main():
     # ---- roofline of the dominant kernel (by event time inside the timed region)
     dom = max(stats, key=lambda s: s["ms"])
     peak_meas = measured_dgemm_peak(torch)
-    traffic = None
-    try:
-        prof = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
-        traffic = prof.get(dom["name"])
-    except (OSError, ValueError):
-        pass
+    traffic, traffic_src = traffic_for(args.config, dom["name"], dom["launches"] // max(args.steps, 1))
     if dom["name"] == "dmma_schur_update":
         achieved = dom["flops"] / (dom["ms"] * 1e-3) / 1e12
         roof = {"kernel": dom["name"], "bound": "tensor", "achieved": achieved, "peak": peak_meas / 1e12,
                 "unit": "TFLOP/s", "frac": achieved / (peak_meas / 1e12), "traffic": traffic,
+                "traffic_source": traffic_src,
                 "peak_source": "cuBLAS DGEMM 8192^3 burst measured in this run (fp64 DMMA path)",
                 "frac_of_nominal_37.2": achieved / (PEAK_NOMINAL_FP64 / 1e12),
                 "launches": dom["launches"] // max(args.steps, 1), "share_of_step": dom["ms"] / (prof_ms * args.steps),
@@ -390,7 +423,7 @@ def main():
             if os.path.exists(os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6650.0
         achieved = dom["bytes"] / (dom["ms"] * 1e-3) / 1e9
         roof = {"kernel": dom["name"], "bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
-                "frac": achieved / hbm, "traffic": traffic,
+                "frac": achieved / hbm, "traffic": traffic, "traffic_source": traffic_src,
                 "launches": dom["launches"] // max(args.steps, 1), "share_of_step": dom["ms"] / (prof_ms * args.steps)}
 
     line = {
@@ -420,6 +453,30 @@ def main():
         "kernels": [{k: (round(v, 4) if isinstance(v, float) else v) for k, v in s.items()} for s in stats],
         "profiled_ms_per_step": prof_ms,
     }
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import oracle
+        sym, subset, gflop, root = oracle_sample(A, perm, args.cpu_baseline_gflop)
+        t0 = time.perf_counter()
+        panels = oracle.factor(A, sym, subset=subset)
+        t_or = time.perf_counter() - t0
+        line["cpu_baseline"] = {
+            "value": gflop / t_or / 1e9, "unit": "GFLOP/s", "cores": cpu_cores(), "kind": "oracle",
+            "cpu_model": cpu_model(),
+            "sample": (f"oracle.factor (plain C + OpenMP, no BLAS) of the whole elimination subtree rooted at "
+                       f"supernode {root} ({len(subset)} fronts, {gflop:.3e} true flops) of {args.config}, "
+                       "incl. B assembly"),
+            "seconds": t_or, "single_thread_c1_c3": single_thread_reference()}
+        # parity of the benched factor on that sample: every panel of the subtree
+        sys.path.insert(0, os.path.join(ROOT, "tests"))
+        from tests._parity import ParityStats
+        st = ParityStats()
+        for sn, Po in panels.items():
+            st.add(sn, S.panel(sn, *Po.shape), Po, m_matrix=c["kind"] != "elast")
+        rep = st.report()
+        line["parity"] = dict(rep, what=("GPU panels of the benched factorization vs the oracle's on the "
+                                          "cpu_baseline sample subtree; reading C11 (tests/_parity.py)"),
+                              ok=rep["floored_max"] <= 1e-10)
+        del panels
     if world == 1 and not args.no_modes:
         # NEXT-3 modes on the same workload (the fp64 DMMA line above is the headline)
         S.close()
@@ -429,14 +486,6 @@ def main():
             "ozaki4_mixed_refined": bench_mode(torch, mf, A, perm, vals_d, stream, 4, args.steps, args.warmup,
                                                b=G.rhs(A.n, 0)),
         }
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        sym, subset, gflop, root = oracle_sample(A, perm, args.cpu_sample_gflop)
-        times = run_oracle_steps(A, sym, subset, 1)
-        line["cpu_baseline"] = {
-            "value": gflop / times[0] / 1e9, "unit": "GFLOP/s", "cores": cpu_cores(), "kind": "oracle",
-            "sample": (f"oracle.factor of the whole elimination subtree rooted at supernode {root} "
-                       f"({len(subset)} fronts, {gflop:.3e} true flops) of {args.config}, incl. B assembly"),
-            "seconds": times[0]}
     if rank == 0:
         print(json.dumps(line), flush=True)
     if world > 1:

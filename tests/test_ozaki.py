@@ -103,3 +103,30 @@ def test_ozaki8_full_tree_parity(name):
     rep = st.report()
     print(name, "ozaki8", rep, "t_factor", S.info()["t_factor"])
     assert rep["floored_max"] <= TOL_L, rep
+
+
+@gpu
+@pytest.mark.parametrize("slices,kind,dims", [(4, "27pt", (24, 24, 24)), (3, "elast", (10, 10, 10)),
+                                              (5, "7pt", (36, 36, 36))])
+def test_mixed_precision_refined_solve(slices, kind, dims, all_int8):
+    """Reduced-precision Schur updates (3..5 slices) + fp64 iterative refinement in
+    mf_solve: the refined x meets reading C12 (backward error <= 1e-12, checked
+    here on the host); the unrefined factor alone does not need to."""
+    from tests.test_gpu_parity import backward_error, spmv
+    A, p = grid(kind, dims)
+    S = mf.Solver(ozaki_slices=slices)
+    S.analyze(A.n, A.colptr, A.rowind, p)
+    assert S.info()["launches_ozaki"] > 0
+    S.factor(A.values)
+    b = spmv(A, G.rhs(A.n, 0))
+    x = S.solve(b)
+    inf = S.info()
+    be = backward_error(A, x, b)
+    print(kind, dims, "slices", slices, "refine steps", inf["refine_steps"], "device berr", inf["solve_berr"],
+          "host berr", be)
+    assert be <= 1e-12
+    assert inf["refine_steps"] >= 1 and 0 <= inf["solve_berr"] <= 1e-12
+    S0 = mf.Solver(ozaki_slices=slices, refine_iters=0)   # the same factor without refinement
+    S0.analyze(A.n, A.colptr, A.rowind, p)
+    S0.factor(A.values)
+    assert backward_error(A, S0.solve(b), b) > be
