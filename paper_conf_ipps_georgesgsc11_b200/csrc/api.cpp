@@ -46,6 +46,7 @@ struct mf_ctx {
     double *d_y = nullptr, *d_bx = nullptr;
     int *d_failed = nullptr;
     int32_t *d_solve_list = nullptr, *d_df_tasks = nullptr;
+    unsigned *d_tickets = nullptr;   // ticket-counter pair per dataflow launch slot (kernels.cu take_ticket)
     cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev_in = nullptr;
     int64_t launches = 0;
     bool profiling = false;
@@ -491,6 +492,13 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     d.fv = (double *)p;
     if ((r = dev_alloc(c, &p, sizeof(int) * 4)) != MF_OK) return r;
     c->d_failed = (int *)p;
+    {   // one counter pair per launch slot of every program (factor local / top, solves)
+        const size_t slots = P.program.size() + P.program_top.size() + P.fsolve.size() + P.bsolve.size() +
+                             P.fsolve_top.size() + P.bsolve_top.size() + 1;
+        if ((r = dev_alloc(c, &p, 2 * slots * sizeof(unsigned))) != MF_OK) return r;
+        c->d_tickets = (unsigned *)p;
+        CK(cudaMemsetAsync(p, 0, 2 * slots * sizeof(unsigned), c->stream));
+    }
     if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.df_nparts, 1) * sizeof(double))) != MF_OK) return r;
     d.df_parts = (double *)p;
     if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.df_nflags, 1) * sizeof(unsigned))) != MF_OK) return r;
@@ -556,6 +564,7 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
     const Plan &P = c->P;
     const DevPlan &d = c->d;
     cudaStream_t st = c->stream;
+    unsigned *tk0 = c->d_tickets + 2 * (&prog == &P.program ? 0 : P.program.size());   // this program's slots
     auto issue = [&](const double *v, bool with_events) -> int {
         if (with_init) launch_init_failed(c->d_failed, st);
         // subtree branches run on their own streams (forked after the init launch,
@@ -618,9 +627,12 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
                         launch_update(d, c->d_probs, c->d_tiles + L.off, L.count,
                                       L.count > 0 ? L.flops / (2.0 * kTileM * kTileN * L.count) : 0.0, st);
                     break;
-                case KC_PANEL: launch_panel(d, c->d_panel + 2 * L.off, L.count, L.param, (int)L.count2, st); break;
+                case KC_PANEL:
+                    launch_panel(d, c->d_panel + 2 * L.off, L.count, L.param, (int)L.count2, tk0 + 2 * li, st);
+                    break;
                 case KC_LEAF:
-                    launch_leaf(d, c->d_large + L.off, (int)L.count, c->d_trsm + 2 * L.off2, L.count2, L.param, P.w, st);
+                    launch_leaf(d, c->d_large + L.off, (int)L.count, c->d_trsm + 2 * L.off2, L.count2, L.param, P.w,
+                                tk0 + 2 * li, st);
                     break;
                 default: return MF_ERR_STATE;   // exchange points are handled by run_with_exchanges
             }
@@ -814,18 +826,25 @@ void run_solve_program(mf_ctx *c, const std::vector<SolveLaunch> &prog) {
     const Plan &P = c->P;
     const DevPlan &d = c->d;
     cudaStream_t st = c->stream;
-    for (const SolveLaunch &L : prog) {
+    size_t base = P.program.size() + P.program_top.size();   // ticket slots of this solve program
+    for (const std::vector<SolveLaunch> *q : {&P.fsolve, &P.bsolve, &P.fsolve_top, &P.bsolve_top}) {
+        if (q == &prog) break;
+        base += q->size();
+    }
+    unsigned *tk0 = c->d_tickets + 2 * base;
+    for (size_t li = 0; li < prog.size(); li++) {
+        const SolveLaunch &L = prog[li];
         switch (L.kind) {
             case SK_SMALL_F: launch_fwd_solve(d, c->d_solve_list + L.off, (int)L.count, c->d_y, st); break;
             case SK_INIT_F: launch_fsolve_init(d, c->d_solve_list + L.off, (int)L.count, c->d_y, st); break;
-            case SK_DF_F: launch_fsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, c->d_y, st); break;
+            case SK_DF_F: launch_fsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, c->d_y, tk0 + 2 * li, st); break;
             case SK_SMALL_B:
                 launch_bwd_solve(d, c->d_solve_list + L.off, (int)L.count, c->d_y, c->d_sn_rows, c->d_sn_rowptr, st);
                 break;
             case SK_INIT_B:
                 launch_bsolve_init(d, c->d_solve_list + L.off, (int)L.count, c->d_y, c->d_sn_rows, c->d_sn_rowptr, st);
                 break;
-            case SK_DF_B: launch_bsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, c->d_y, st); break;
+            case SK_DF_B: launch_bsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, c->d_y, tk0 + 2 * li, st); break;
         }
     }
 }

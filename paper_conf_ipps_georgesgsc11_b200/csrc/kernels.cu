@@ -652,21 +652,43 @@ __global__ void __launch_bounds__(kTrsmThreads, 2) k_trsm_panel(DevPlan d, const
     trsm_block(d, tasks[2 * blockIdx.x], tasks[2 * blockIdx.x + 1], j0, w, tsm, nullptr, 0);
 }
 
+// Ticket-ordered task ids.  The dataflow kernels below spin-
+// wait on tasks with smaller ids; a CTA takes the next ticket as its task id when it
+// starts, so every smaller ticket belongs to a CTA that is already resident and
+// forward progress never depends on the hardware dispatching CTAs in blockIdx
+// order (nor on how concurrent graph branches share the SMs).  Each launch slot
+// owns a pair of counters; the last CTA to finish resets it for the next launch of
+// the slot (stream-ordered, so no other launch of the slot is in flight).
+__device__ __forceinline__ int take_ticket(unsigned *tk) {
+    __shared__ int tkt;
+    if (threadIdx.x == 0) tkt = (int)atomicAdd(tk, 1u);
+    __syncthreads();
+    return tkt;
+}
+__device__ __forceinline__ void drop_ticket(unsigned *tk) {
+    __syncthreads();
+    if (threadIdx.x == 0 && atomicAdd(tk + 1, 1u) == gridDim.x - 1) {
+        tk[0] = 0u;
+        tk[1] = 0u;
+        __threadfence();
+    }
+}
+
 // Fused leaf: blocks [0, npotrf) factor the diagonal blocks of the active fronts
 // (then publish a per-front flag), blocks [npotrf, ...) solve the row blocks below;
 // each TRSM block stages its rows, waits for its front's flag, then loads L11.
 // The diagonal-block CTAs have the lowest block indices, so they are dispatched
 // first and never wait: no deadlock.  Saves one launch (and the row-block load
 // latency) per leaf on the sequential chain of the top fronts.
-__global__ void __launch_bounds__(kTrsmThreads, 2) k_leaf(DevPlan d, const int32_t *__restrict__ fronts, int npotrf,
-                                                          const int32_t *__restrict__ tasks, int j0, int w) {
+__device__ __forceinline__ void leaf_task(const DevPlan &d, const int32_t *__restrict__ fronts, int npotrf,
+                                          const int32_t *__restrict__ tasks, int j0, int w, const int task) {
     extern __shared__ __align__(16) double tsm[];
     // tag = (epoch mod 2^16) << 16 | leaf index + 1: consecutive factorizations differ in
     // the epoch bits, and the leaf index (k / w < 2^16 - 1, checked by build_plan) never
     // spills into them (10 bits overflowed for k > 1023 w)
     const unsigned expect = ((*d.epoch & 0xffffu) << 16) | (unsigned)(j0 / w + 1);
-    if ((int)blockIdx.x < npotrf) {
-        const int s = fronts[blockIdx.x];
+    if (task < npotrf) {
+        const int s = fronts[task];
         potrf_block<kTrsmThreads>(d, s, j0, w, tsm, tsm + kWmax * kWmax);
         __threadfence();
         __syncthreads();
@@ -674,15 +696,21 @@ __global__ void __launch_bounds__(kTrsmThreads, 2) k_leaf(DevPlan d, const int32
             asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(d.leaf_flag + s), "r"(expect) : "memory");
         return;
     }
-    const int t = blockIdx.x - npotrf;
+    const int t = task - npotrf;
     const int s = tasks[2 * t];
     trsm_block(d, s, tasks[2 * t + 1], j0, w, tsm, d.leaf_flag + s, expect);
 }
+__global__ void __launch_bounds__(kTrsmThreads, 2) k_leaf(DevPlan d, const int32_t *__restrict__ fronts, int npotrf,
+                                                          const int32_t *__restrict__ tasks, int j0, int w,
+                                                          unsigned *tk) {
+    leaf_task(d, fronts, npotrf, tasks, j0, w, take_ticket(tk));
+    drop_ticket(tk);
+}
 
 void launch_leaf(const DevPlan &d, const int32_t *fronts, int npotrf, const int32_t *tasks, int64_t ntrsm, int j0,
-                 int w, cudaStream_t st) {
+                 int w, unsigned *tk, cudaStream_t st) {
     if (npotrf <= 0) return;
-    k_leaf<<<(unsigned)(npotrf + ntrsm), kTrsmThreads, kTrsmSmem, st>>>(d, fronts, npotrf, tasks, j0, w);
+    k_leaf<<<(unsigned)(npotrf + ntrsm), kTrsmThreads, kTrsmSmem, st>>>(d, fronts, npotrf, tasks, j0, w, tk);
 }
 
 // ============================================================ dataflow panel ("super-leaf")
@@ -721,22 +749,6 @@ constexpr size_t kPanelSmem = (size_t)(kPanelRingWords + 64 * kPLD + 64) * sizeo
 static_assert(64 * kPLD <= kPanelRingWords, "the L_bb tile aliases the staging ring");
 
 __device__ __forceinline__ int panel_tri(int c, int b) { return c * (c + 1) / 2 + b; }
-
-// Optional device-side timeline of the panel tasks (tools/ubench/panel_bench.cu
-// compiles this file with -DMF_PANEL_TRACE); compiled out of libmf.
-#ifdef MF_PANEL_TRACE
-__device__ unsigned long long g_panel_trace[4096][32];
-__device__ __forceinline__ void panel_mark(int ev) {
-    if (threadIdx.x == 0 && blockIdx.x < 4096 && ev < 32) {
-        unsigned long long t;
-        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-        g_panel_trace[blockIdx.x][ev] = t;
-    }
-}
-#define PANEL_MARK(ev) panel_mark(ev)
-#else
-#define PANEL_MARK(ev)
-#endif
 
 // acc(64 x 64 tile; this warp's 32 x 32 fragment) -= A B^T with A = rows [ra0, ra0+64),
 // B = rows [rb0, rb0+64), columns [kc0, kc0 + K) of the panel Pn (column-major, ld);
@@ -819,83 +831,6 @@ __device__ __forceinline__ void panel_frag_to_smem(const double (&acc)[4][4][2],
     }
 }
 
-// Factor the first `we` columns of the R x we panel A (shared memory, column-major,
-// stride kPLD; R <= 64 rows, the top we x we block is the diagonal block): the
-// algorithm of potrf_block, extended to rows below the diagonal block (the last
-// block of a front whose k ends inside a 64-row tile).
-__device__ __forceinline__ void panel_potrf(const DevPlan &d, double *A, double *sinv, int R, int we, int first_col) {
-    constexpr int SB = 8, G = kPanelThreads / 64;
-    const int tid = threadIdx.x;
-#pragma unroll 1
-    for (int s0 = 0; s0 < we; s0 += SB) {
-        const int nb = min(SB, we - s0);
-        if (tid == 0) {
-            double a[SB][SB];
-#pragma unroll
-            for (int c = 0; c < SB; c++)
-#pragma unroll
-                for (int r = c; r < SB; r++) a[r][c] = (r < nb) ? A[(s0 + c) * kPLD + s0 + r] : (r == c ? 1.0 : 0.0);
-#pragma unroll
-            for (int q = 0; q < SB; q++) {
-                if (q < nb) note_pivot(d, a[q][q], first_col + s0 + q);
-                const double inv = rsqrt(a[q][q]);
-                a[q][q] *= inv;
-                sinv[s0 + q] = inv;
-#pragma unroll
-                for (int r = q + 1; r < SB; r++) a[r][q] *= inv;
-#pragma unroll
-                for (int c = q + 1; c < SB; c++)
-#pragma unroll
-                    for (int r = c; r < SB; r++) a[r][c] = fma(-a[r][q], a[c][q], a[r][c]);
-            }
-#pragma unroll
-            for (int c = 0; c < SB; c++)
-#pragma unroll
-                for (int r = c; r < SB; r++)
-                    if (r < nb) A[(s0 + c) * kPLD + s0 + r] = a[r][c];
-        }
-        __syncthreads();
-        const int rb = s0 + nb;
-        if (rb >= R) break;
-        // rows [rb, R) against the sub-block (columns >= nb of a partial sub-block are padding)
-        if (tid < R - rb) {
-            const int r = rb + tid;
-            double x[SB];
-#pragma unroll
-            for (int q = 0; q < SB; q++) x[q] = (q < nb) ? A[(s0 + q) * kPLD + r] : 0.0;
-#pragma unroll
-            for (int q = 0; q < SB; q++) {
-                if (q < nb) {
-                    x[q] *= sinv[s0 + q];
-#pragma unroll
-                    for (int q2 = q + 1; q2 < SB; q2++)
-                        if (q2 < nb) x[q2] -= x[q] * A[(s0 + q) * kPLD + s0 + q2];
-                }
-            }
-#pragma unroll
-            for (int q = 0; q < SB; q++)
-                if (q < nb) A[(s0 + q) * kPLD + r] = x[q];
-        }
-        __syncthreads();
-        // trailing update of columns [rb, we), rows i >= column
-        if (rb < we) {
-            const int i = tid & 63, h = tid >> 6;
-            if (i >= rb && i < R) {
-                double li[SB];
-#pragma unroll
-                for (int q = 0; q < SB; q++) li[q] = A[(s0 + q) * kPLD + i];
-                const int cmax = min(i, we - 1);
-                for (int c = rb + h; c <= cmax; c += G) {
-                    double acc = A[c * kPLD + i];
-#pragma unroll
-                    for (int q = 0; q < SB; q++) acc -= li[q] * A[(s0 + q) * kPLD + c];
-                    A[c * kPLD + i] = acc;
-                }
-            }
-        }
-        __syncthreads();
-    }
-}
 
 // 1/sqrt(x): MUFU.RSQ64H seed + two Newton steps (exact 2^-p for x = 4^p, so the
 // manufactured integer factors stay exact; ~1 ulp otherwise, reading C9).
@@ -974,23 +909,13 @@ __device__ __forceinline__ void panel_potrf_dmma(const DevPlan &d, double *A, do
     constexpr int SB = 8;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int nrb = (R + 7) / 8, ncb = (we + 7) / 8;
-#ifdef MF_PANEL_TRACE
-    long long ta = 0, tb = 0, tc = 0, x1 = 0, x2 = 0;
-    x1 = clock64();
-#endif
     if (tid == 0) factor_diag8(d, A, sinv, 0, min(SB, we), first_col);
     __syncthreads();
-#ifdef MF_PANEL_TRACE
-    ta += clock64() - x1;
-#endif
 #pragma unroll 1
     for (int st = 0; st < ncb; st++) {
         const int s0 = st * SB, nb = min(SB, we - s0);
         const int rb = s0 + nb;
         if (rb >= R) break;
-#ifdef MF_PANEL_TRACE
-        x1 = clock64();
-#endif
         // rows [rb, R) against the factored pivot block st
         if (tid < R - rb) {
             const int r = rb + tid;
@@ -1010,10 +935,6 @@ __device__ __forceinline__ void panel_potrf_dmma(const DevPlan &d, double *A, do
                 if (q < nb) A[(s0 + q) * kPLD + r] = x[q];
         }
         __syncthreads();
-#ifdef MF_PANEL_TRACE
-        x2 = clock64();
-        tb += x2 - x1;
-#endif
         if (st + 1 < ncb) {
             const int J1 = st + 1;
             if (warp == 0) {
@@ -1029,15 +950,7 @@ __device__ __forceinline__ void panel_potrf_dmma(const DevPlan &d, double *A, do
             }
         }
         __syncthreads();
-#ifdef MF_PANEL_TRACE
-        tc += clock64() - x2;
-#endif
     }
-#ifdef MF_PANEL_TRACE
-    if (threadIdx.x == 0 && blockIdx.x < 4096) {
-        g_panel_trace[blockIdx.x][25] = ta; g_panel_trace[blockIdx.x][26] = tb; g_panel_trace[blockIdx.x][27] = tc;
-    }
-#endif
 }
 
 // X <- X L^-T for the 64 rows of Xs over wb columns; Ls = the wb x wb lower factor
@@ -1109,13 +1022,13 @@ __device__ __forceinline__ void panel_publish(unsigned *flag, unsigned tag) {
     if (threadIdx.x == 0) asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(flag), "r"(tag) : "memory");
 }
 
-__global__ void __launch_bounds__(kPanelThreads, MF_PANEL_MINB) k_panel(DevPlan d, const int32_t *__restrict__ tasks, int j0,
-                                                             int nbk) {
+__device__ __forceinline__ void panel_task(const DevPlan &d, const int32_t *__restrict__ tasks, int j0, int nbk,
+                                           const int task) {
     extern __shared__ __align__(16) double psm[];
     double *ring = psm;                         // accumulate staging; the L_bb tile afterwards
     double *Xs = psm + kPanelRingWords;         // the tile being finished
     double *inv = Xs + 64 * kPLD;
-    const int s = tasks[2 * blockIdx.x], c = tasks[2 * blockIdx.x + 1];
+    const int s = tasks[2 * task], c = tasks[2 * task + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s];
     const int nb = min(nbk, (k - j0 + 63) / 64);
     const int r0 = j0 + 64 * c, rows = min(64, f - r0);
@@ -1127,7 +1040,6 @@ __global__ void __launch_bounds__(kPanelThreads, MF_PANEL_MINB) k_panel(DevPlan 
     // the diagonal tile's accumulator: its 36 lower 8 x 8 blocks, 9 per warp
     // (block rows `warp` and 7 - warp), so the row's own products cost 144 DMMA per warp
     double dacc[9][2];
-    PANEL_MARK(0);
     if (band) {
         const int cols = min(64, k - r0);
 #pragma unroll
@@ -1149,13 +1061,10 @@ __global__ void __launch_bounds__(kPanelThreads, MF_PANEL_MINB) k_panel(DevPlan 
         panel_frag_load(acc, Pn, ld, r0, rows, cb0, wb);
         if (b > 0) {
             wait_flag(F + panel_tri(b, b - 1), tag);   // band tiles (b, 0..b-1) are final
-            PANEL_MARK(1 + 6 * b);
             panel_tile_mma(acc, ring, Pn, ld, r0, rows, cb0, min(64, f - cb0), j0, 64 * b);
         }
         panel_frag_to_smem(acc, Xs);
-        PANEL_MARK(2 + 6 * b);
         wait_flag(F + panel_tri(b, b), tag);           // L_bb is final
-        PANEL_MARK(3 + 6 * b);
         {
             const double *__restrict__ D = Pn + (int64_t)cb0 * ld + cb0;
             for (int q = tid; q < 32 * 64; q += kPanelThreads) {
@@ -1177,9 +1086,7 @@ __global__ void __launch_bounds__(kPanelThreads, MF_PANEL_MINB) k_panel(DevPlan 
             if (tid < 64) inv[tid] = __drcp_rn(ring[tid + tid * kPLD]);
             __syncthreads();
         }
-        PANEL_MARK(4 + 6 * b);
         panel_trsm(Xs, ring, inv, wb);
-        PANEL_MARK(5 + 6 * b);
         for (int q = tid; q < 64 * 64; q += kPanelThreads) {
             const int i = q & 63, j = q >> 6;
             if (i < rows && j < wb) Pn[(r0 + i) + (int64_t)(cb0 + j) * ld] = Xs[i + j * kPLD];
@@ -1199,10 +1106,8 @@ __global__ void __launch_bounds__(kPanelThreads, MF_PANEL_MINB) k_panel(DevPlan 
 #pragma unroll
                 for (int t = 0; t < 9; t++) dmma(dacc[t][0], dacc[t][1], t <= warp ? a0 : a1, bj[t]);
             }
-            PANEL_MARK(31);
             panel_publish(F + panel_tri(c, b), tag);   // X(c,b) is stored: band tile final (+ CTA barrier:
                                                        // Xs / ring are rewritten by the next step)
-            PANEL_MARK(6 + 6 * b);
         } else {
             __syncthreads();   // Xs / ring are rewritten by the next step
         }
@@ -1217,25 +1122,25 @@ __global__ void __launch_bounds__(kPanelThreads, MF_PANEL_MINB) k_panel(DevPlan 
             for (int e = 0; e < 2; e++) Xs[I * 8 + gq + (J * 8 + 2 * tq + e) * kPLD] = dacc[t][e];
         }
         __syncthreads();
-        PANEL_MARK(28);
-#ifdef MF_PANEL_OLD_POTRF
-        panel_potrf(d, Xs, inv, rows, we, d.sn_first[s] + r0);
-#else
         panel_potrf_dmma(d, Xs, inv, rows, we, d.sn_first[s] + r0);
-#endif
-        PANEL_MARK(29);
         for (int q = tid; q < 64 * 64; q += kPanelThreads) {
             const int i = q & 63, j = q >> 6;
             if (i < rows && j < we && i >= j) Pn[(r0 + i) + (int64_t)(r0 + j) * ld] = Xs[i + j * kPLD];
         }
         panel_publish(F + panel_tri(c, c), tag);
-        PANEL_MARK(30);
     }
 }
 
-void launch_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int nbk, cudaStream_t st) {
+__global__ void __launch_bounds__(kPanelThreads, MF_PANEL_MINB) k_panel(DevPlan d, const int32_t *__restrict__ tasks,
+                                                                         int j0, int nbk, unsigned *tk) {
+    panel_task(d, tasks, j0, nbk, take_ticket(tk));
+    drop_ticket(tk);
+}
+
+void launch_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int nbk, unsigned *tk,
+                  cudaStream_t st) {
     if (count <= 0) return;
-    k_panel<<<(unsigned)count, kPanelThreads, kPanelSmem, st>>>(d, tasks, j0, nbk);
+    k_panel<<<(unsigned)count, kPanelThreads, kPanelSmem, st>>>(d, tasks, j0, nbk, tk);
 }
 
 void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, cudaStream_t st) {
@@ -1540,11 +1445,11 @@ __device__ __forceinline__ void warp_trsv_bwd(const double *__restrict__ Lb, con
     }
 }
 
-__global__ void __launch_bounds__(kSolveThreads) k_fsolve_df(DevPlan d, const int32_t *__restrict__ tasks, int w,
-                                                             double *__restrict__ y) {
+__device__ __forceinline__ void fsolve_df_task(const DevPlan &d, const int32_t *__restrict__ tasks, int w,
+                                               double *__restrict__ y, const int task) {
     __shared__ double Lb[kSW * kSLD];
     __shared__ double xs[kSW], dinv[kSW];
-    const int s = tasks[2 * blockIdx.x], c = tasks[2 * blockIdx.x + 1];
+    const int s = tasks[2 * task], c = tasks[2 * task + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
     const double *__restrict__ P = d.L + d.L_off[s];
     double *__restrict__ v = d.fv + d.fv_off[s];
@@ -1598,6 +1503,11 @@ __global__ void __launch_bounds__(kSolveThreads) k_fsolve_df(DevPlan d, const in
     }
     if (rok && r >= k) v[r] = vr;   // the update vector the parent gathers
 }
+__global__ void __launch_bounds__(kSolveThreads) k_fsolve_df(DevPlan d, const int32_t *__restrict__ tasks, int w,
+                                                             double *__restrict__ y, unsigned *tk) {
+    fsolve_df_task(d, tasks, w, y, take_ticket(tk));
+    drop_ticket(tk);
+}
 
 // Butterfly reduce-scatter over the warp: 64 values per lane in, lane l ends with
 // the warp sums of q = 2 l + {0, 1} in p[0], p[1] (62 shuffles).
@@ -1616,12 +1526,12 @@ __device__ __forceinline__ void warp_reduce_scatter64(double (&p)[kSW]) {
     }
 }
 
-__global__ void __launch_bounds__(kSolveThreads) k_bsolve_df(DevPlan d, const int32_t *__restrict__ tasks, int w,
-                                                             double *__restrict__ y) {
+__device__ __forceinline__ void bsolve_df_task(const DevPlan &d, const int32_t *__restrict__ tasks, int w,
+                                               double *__restrict__ y, const int task) {
     __shared__ double red[kSolveThreads / 32][kSW];
     __shared__ double Lb[kSW * kSLD];
     __shared__ double tv[kSW], dinv[kSW];
-    const int s = tasks[2 * blockIdx.x], c = tasks[2 * blockIdx.x + 1];
+    const int s = tasks[2 * task], c = tasks[2 * task + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
     const double *__restrict__ P = d.L + d.L_off[s];
     double *__restrict__ v = d.fv + d.fv_off[s];
@@ -1695,19 +1605,26 @@ __global__ void __launch_bounds__(kSolveThreads) k_bsolve_df(DevPlan d, const in
         __syncthreads();
     }
 }
+__global__ void __launch_bounds__(kSolveThreads) k_bsolve_df(DevPlan d, const int32_t *__restrict__ tasks, int w,
+                                                             double *__restrict__ y, unsigned *tk) {
+    bsolve_df_task(d, tasks, w, y, take_ticket(tk));
+    drop_ticket(tk);
+}
 
 void launch_fsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, cudaStream_t st) {
     if (count > 0) k_fsolve_init<<<count, kSolveThreads, 0, st>>>(d, list, y);
 }
-void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, cudaStream_t st) {
-    if (count > 0) k_fsolve_df<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, w, y);
+void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, unsigned *tk,
+                      cudaStream_t st) {
+    if (count > 0) k_fsolve_df<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, w, y, tk);
 }
 void launch_bsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, const int32_t *sn_rows,
                         const int64_t *sn_rowptr, cudaStream_t st) {
     if (count > 0) k_bsolve_init<<<count, kSolveThreads, 0, st>>>(d, list, y, sn_rows, sn_rowptr);
 }
-void launch_bsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, cudaStream_t st) {
-    if (count > 0) k_bsolve_df<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, w, y);
+void launch_bsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, unsigned *tk,
+                      cudaStream_t st) {
+    if (count > 0) k_bsolve_df<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, w, y, tk);
 }
 
 // dst[first_s + j] = src[first_s + j] for the columns of the listed supernodes

@@ -39,9 +39,11 @@ void launch_init_failed(int *failed, cudaStream_t st);
 void launch_small_fronts(const DevPlan &d, const int32_t *list, int count, int fmax, const double *values,
                          cudaStream_t st);
 void launch_assemble(const DevPlan &d, const int32_t *tasks, int64_t count, const double *values, cudaStream_t st);
+// tk: the launch slot's ticket-counter pair (zeroed at analyze; see take_ticket in kernels.cu)
 void launch_leaf(const DevPlan &d, const int32_t *fronts, int npotrf, const int32_t *tasks, int64_t ntrsm, int j0,
-                 int w, cudaStream_t st);
-void launch_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int nbk, cudaStream_t st);
+                 int w, unsigned *tk, cudaStream_t st);
+void launch_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int nbk, unsigned *tk,
+                  cudaStream_t st);
 void launch_potrf_diag(const DevPlan &d, const int32_t *fronts, int count, int j0, int w, cudaStream_t st);
 void launch_trsm_panel(const DevPlan &d, const int32_t *tasks, int64_t count, int j0, int w, cudaStream_t st);
 // kavg = the launch's average inner dimension.  Variant per launch (measured per
@@ -70,8 +72,10 @@ void launch_fwd_solve(const DevPlan &d, const int32_t *list, int count, double *
 void launch_bwd_solve(const DevPlan &d, const int32_t *list, int count, double *y, const int32_t *sn_rows,
                       const int64_t *sn_rowptr, cudaStream_t st);
 void launch_fsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, cudaStream_t st);
-void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, cudaStream_t st);
-void launch_bsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, cudaStream_t st);
+void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, unsigned *tk,
+                      cudaStream_t st);
+void launch_bsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, unsigned *tk,
+                      cudaStream_t st);
 void launch_bsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, const int32_t *sn_rows,
                         const int64_t *sn_rowptr, cudaStream_t st);
 

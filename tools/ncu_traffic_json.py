@@ -20,7 +20,8 @@ CLASS = {"k_update_t": "dmma_schur_update", "k_oz_gemm": "dmma_schur_update", "k
          "k_potrf_diag": "potrf_diag", "k_trsm_panel": "trsm_panel"}
 KIND = {"small_front_fused": 0, "assemble_extend_add": 1, "potrf_diag": 2, "trsm_panel": 3, "dmma_schur_update": 4,
         "leaf_potrf_trsm": 5, "dataflow_panel": 6}
-SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "KB": 1e3, "MB": 1e6, "GB": 1e9,
+SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "KB": 1e3, "MB": 1e6, "GB": 1e9, "ns": 1e-9, "us": 1e-6,
+         "ms": 1e-3,
          "nsecond": 1e-9, "usecond": 1e-6, "msecond": 1e-3, "second": 1.0}
 
 csv_path, cfg = sys.argv[1], (sys.argv[2] if len(sys.argv) > 2 else "c5")

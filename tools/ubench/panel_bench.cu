@@ -1,7 +1,7 @@
-// Latency / timeline microbenchmark of the dataflow panel kernel (k_panel) on one
-// dense front: f rows, k pivot columns, panel of nbk blocks at j0 = 0.
-// Builds kernels.cu with -DMF_PANEL_TRACE and prints per-task globaltimer marks.
-//   nvcc -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -DMF_PANEL_TRACE \
+// Latency microbenchmark of the dataflow panel kernel (k_panel) on one dense
+// front: f rows, k pivot columns, panel of nbk blocks at j0 = 0; checks L L^T = A
+// on the panel columns.
+//   nvcc -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a \
 //        -I include -I paper_conf_ipps_georgesgsc11_b200/csrc tools/ubench/panel_bench.cu -o tools/ubench/panel_bench
 #include "../../paper_conf_ipps_georgesgsc11_b200/csrc/kernels.cu"
 
@@ -35,6 +35,7 @@ int main(int argc, char **argv) {
     int hf[4] = {INT_MAX, 1, 0, 0};
     cudaMemcpy(failed, hf, 16, cudaMemcpyHostToDevice);
     unsigned *pflag; cudaMalloc(&pflag, kPanelFlags * 4);
+    unsigned *tk; cudaMalloc(&tk, 8); cudaMemset(tk, 0, 8);
     DevPlan d{};
     d.L = L; d.sn_first = dfirst; d.sn_k = dk; d.sn_f = df; d.sn_ld = dld; d.L_off = doff;
     d.failed = failed; d.epoch = reinterpret_cast<const unsigned *>(failed + 1); d.panel_flag = pflag;
@@ -50,7 +51,7 @@ int main(int argc, char **argv) {
         cudaMemcpy(L, L0, h.size() * 8, cudaMemcpyDeviceToDevice);
         cudaMemset(pflag, 0, kPanelFlags * 4);
         cudaEventRecord(e0);
-        launch_panel(d, dt, nch, 0, nbk, 0);
+        launch_panel(d, dt, nch, 0, nbk, tk, 0);
         cudaEventRecord(e1);
         cudaEventSynchronize(e1);
         float ms; cudaEventElapsedTime(&ms, e0, e1);
@@ -58,20 +59,6 @@ int main(int argc, char **argv) {
     }
     cudaError_t err = cudaGetLastError();
     printf("f=%d k=%d nbk=%d tasks=%d: best %.2f us (%s)\n", f, k, nbk, nch, best * 1e3, cudaGetErrorString(err));
-    static unsigned long long tr[4096][32];
-    cudaMemcpyFromSymbol(tr, g_panel_trace, sizeof(tr));
-    unsigned long long t0 = ~0ull;
-    for (int c = 0; c < nch; c++) if (tr[c][0] && tr[c][0] < t0) t0 = tr[c][0];
-    auto show = [&](int c) {
-        printf("task %4d:", c);
-        printf(" [potrf clk a %llu b %llu c %llu]", tr[c][25], tr[c][26], tr[c][27]);
-        for (int e = 0; e < 32; e++)
-            if (e < 25 || e > 27) if (tr[c][e] >= t0 && tr[c][e] - t0 < 10000000ull) printf(" %d:%.1f", e, (tr[c][e] - t0) / 1e3);
-        printf("\n");
-    };
-    for (int c = 0; c < std::min(nch, nbk + 1); c++) show(c);
-    show(nch / 2);
-    show(nch - 1);
     // check: the leading W x W block of L L^T reproduces A (W = 64 nbk), and the rows
     // below: (L L^T)(i, j) = A(i, j) for j < W
     std::vector<double> Lh(h.size());
