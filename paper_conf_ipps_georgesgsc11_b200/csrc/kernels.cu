@@ -86,6 +86,7 @@ __device__ __forceinline__ void warp_factor16(double *A, int lda, int s0, int nb
             }
         }
     }
+    __syncwarp();   // every lane's reads of the block precede the write-back
     if (lane < nb) {
 #pragma unroll
         for (int q = 0; q < 16; q++)
@@ -927,7 +928,8 @@ __device__ __forceinline__ void panel_potrf_dmma(const DevPlan &d, double *A, do
                 if (q < nb) {
                     x[q] *= sinv[s0 + q];
 #pragma unroll
-                    for (int q2 = q + 1; q2 < SB; q2++) x[q2] = fma(-x[q], A[(s0 + q) * kPLD + s0 + q2], x[q2]);
+                    for (int q2 = q + 1; q2 < SB; q2++)   // (q2 < nb: rows past the pivot block are other threads')
+                        if (q2 < nb) x[q2] = fma(-x[q], A[(s0 + q) * kPLD + s0 + q2], x[q2]);
                 }
             }
 #pragma unroll

@@ -16,7 +16,7 @@ case = sys.argv[1]
 if case == "c1":
     A, p = grid("5pt", (32, 32, 1))
     opts = {}
-elif case == "tiled_bulk":
+elif case in ("tiled", "tiled_bulk"):
     A, p = grid("27pt", (16, 16, 16))
     opts = dict(small_front_max=8, variant_model=None)
 elif case == "ozaki":
