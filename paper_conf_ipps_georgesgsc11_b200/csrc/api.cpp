@@ -47,6 +47,8 @@ struct mf_ctx {
     int *d_failed = nullptr;
     int32_t *d_solve_list = nullptr, *d_df_tasks = nullptr;
     unsigned *d_tickets = nullptr;   // ticket-counter pair per dataflow launch slot (kernels.cu take_ticket)
+    int32_t *d_dinv_tasks = nullptr; // solve setup: (supernode, 64-block) pairs whose inverse the solves use
+    bool dinv_stale = true;          // set by mf_factor; the next solve recomputes the block inverses
     cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev_in = nullptr;
     int64_t launches = 0;
     bool profiling = false;
@@ -408,9 +410,11 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     UP(&c->d_tiles, P.tiles);
     UP(&c->d_solve_list, P.solve_list);
     UP(&c->d_df_tasks, P.df_tasks);
-    int64_t *df_blk_off = nullptr, *df_part_off = nullptr;
+    int64_t *df_blk_off = nullptr, *df_part_off = nullptr, *dinv_off = nullptr;
     UP(&df_blk_off, P.df_blk_off);
     UP(&df_part_off, P.df_part_off);
+    UP(&dinv_off, P.dinv_off);
+    UP(&c->d_dinv_tasks, P.dinv_tasks);
     int32_t *ea_qs = nullptr;
     UP(&ea_qs, P.ea_qs);
     UP(&c->d_top_list, P.top_list);
@@ -479,6 +483,7 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     d.perm = perm_d;
     d.df_blk_off = df_blk_off;
     d.df_part_off = df_part_off;
+    d.dinv_off = dinv_off;
     d.ea_qs = ea_qs;
     d.fuse_ea = P.fuse_ea;
     void *p;
@@ -501,6 +506,9 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     }
     if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.df_nparts, 1) * sizeof(double))) != MF_OK) return r;
     d.df_parts = (double *)p;
+    if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.dinv_words, 1) * sizeof(double))) != MF_OK) return r;
+    d.dinv = (double *)p;
+    c->dinv_stale = true;
     if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.df_nflags, 1) * sizeof(unsigned))) != MF_OK) return r;
     d.df_flags = (unsigned *)p;
     CK(cudaMemsetAsync(d.df_flags, 0, (size_t)std::max<int64_t>(P.df_nflags, 1) * sizeof(unsigned), c->stream));
@@ -797,6 +805,7 @@ int mf_factor(mf_ctx *c, const double *values) {
         if ((r = exchange(c, red))) return r;
     }
     if (c->d_bval) launch_refine_bval(c->d, vals, c->d_bval, (int64_t)c->S.brow.size(), st);   // for mf_solve's residuals
+    c->dinv_stale = true;
     CK(cudaGetLastError());
     int failed = INT_MAX;
     CK(cudaMemcpyAsync(&failed, c->d_failed, sizeof(int), cudaMemcpyDeviceToHost, st));
@@ -864,6 +873,10 @@ int mf_solve(mf_ctx *c, const double *b, double *x) {
         if (int r = order_after_caller(c)) return r;
     }
     CK(cudaEventRecord(c->ev0, st));
+    if (c->dinv_stale) {   // solve setup, once per factorization: inverses of the 64 x 64 diagonal blocks
+        launch_diag_inv(d, c->d_dinv_tasks, (int64_t)P.dinv_tasks.size() / 2, P.w, st);
+        c->dinv_stale = false;
+    }
     if (!multi && c->use_graph) {
         // single GPU: the whole solve is one CUDA graph over the ctx buffers
         // (b -> d_bx, permute, forward, backward, permute back into d_bx -> x)
@@ -988,7 +1001,7 @@ int mf_solve_nrhs(mf_ctx *c, int32_t nrhs, const double *B, int64_t ldb, double 
     if (bdev || xdev) {
         if (int r = order_after_caller(c)) return r;
     }
-    if (!c->solve_exec) {   // capture the solve graph (same program as mf_solve)
+    if (!c->solve_exec || c->dinv_stale) {   // capture the solve graph / solve setup (same program as mf_solve)
         if (int e = mf_solve(c, B, X)) return e;
         if (nrhs == 1) return MF_OK;
         B += ldb;

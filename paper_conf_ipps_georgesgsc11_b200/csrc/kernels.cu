@@ -1400,64 +1400,86 @@ __device__ __forceinline__ void load_row_block(const double *__restrict__ P, int
     for (int q = 0; q < kSW; q++) Lr[q] = (ok && q < we) ? col[(int64_t)q * ld] : 0.0;
 }
 
-// Row i of the diagonal block (held in a row slab, entries q <= i) into shared
-// memory, its pivot's reciprocal into dinv, and xv into xs[i]; the slab row is
-// then zeroed so that the row takes no part in the block's off-diagonal product.
-__device__ __forceinline__ void stash_diag_row(double (&Lr)[kSW], int i, double xv, double *__restrict__ Lb,
-                                               double *__restrict__ dinv, double *__restrict__ xs) {
-    double dd = 1.0;
+// ---- solve setup: inv(L_bb) of every 64 x 64 diagonal block of the dataflow-solved
+// supernodes (once per factorization, by the first solve), so the block chains of the
+// sweeps below apply a 64 x 64 matrix-vector product (x_b = inv(L_bb) t_b, all threads)
+// instead of a 64-step substitution on one warp.  One CTA of 64 threads per block;
+// thread j forms column j of the inverse by forward substitution, L_bb in shared memory.
+// Stored column-major 64 x 64 (zero above the diagonal; a ragged last block is
+// extended by the identity).  Power-of-two pivots give exact inverses (the
+// manufactured factors stay exact through the solve).
+__global__ void __launch_bounds__(64) k_diag_inv(DevPlan d, const int32_t *__restrict__ tasks, int w) {
+    __shared__ double Ls[kSW * kSLD];
+    const int s = tasks[2 * blockIdx.x], b = tasks[2 * blockIdx.x + 1];
+    const int k = d.sn_k[s], ld = d.sn_ld[s];
+    const int j0 = b * w, we = min(w, k - j0);   // block b of width w (<= 64) in a 64 x 64 slot
+    const double *__restrict__ D = d.L + d.L_off[s] + (int64_t)j0 * ld + j0;
+    const int j = threadIdx.x;
+    for (int q = 0; q < kSW; q++)   // row j, column q of the (identity-extended) block
+        Ls[j + q * kSLD] = (j < we && q < we) ? (q <= j ? D[j + (int64_t)q * ld] : 0.0) : (j == q ? 1.0 : 0.0);
+    __syncthreads();
+    // column j of inv(L): x_i = (delta_ij - sum_{q < i} L_iq x_q) / L_ii, x_q = 0 for q < j
+    // (fully unrolled: x stays in registers; the terms with q < j add exact zeros)
+    double x[kSW];
 #pragma unroll
-    for (int q = 0; q < kSW; q++) {
-        if (q <= i) Lb[i + q * kSLD] = Lr[q];
-        if (q == i) dd = Lr[q];
-        Lr[q] = 0.0;
+    for (int i = 0; i < kSW; i++) {
+        double t = (i == j) ? 1.0 : 0.0;
+#pragma unroll
+        for (int q = 0; q < i; q++) t = fma(-Ls[i + q * kSLD], x[q], t);
+        x[i] = (i >= j) ? t / Ls[i + i * kSLD] : 0.0;
     }
-    dinv[i] = 1.0 / dd;
-    xs[i] = xv;
+    __syncthreads();
+#pragma unroll
+    for (int i = 0; i < kSW; i++) Ls[i + j * kSLD] = x[i];   // column j
+    __syncthreads();
+    double *__restrict__ out = d.dinv + d.dinv_off[s] + (int64_t)b * kSW * kSW;
+    for (int q = 0; q < kSW; q++) out[j + q * kSW] = Ls[j + q * kSLD];   // coalesced
+}
+void launch_diag_inv(const DevPlan &d, const int32_t *tasks, int64_t count, int w, cudaStream_t st) {
+    if (count > 0) k_diag_inv<<<(unsigned)count, 64, 0, st>>>(d, tasks, w);
 }
 
-
-// One warp: x = L_bb^{-1} t (forward, right-looking) with t in (a0, a1) = entries
-// lane, lane + 32.
-__device__ __forceinline__ void warp_trsv_fwd(const double *__restrict__ Lb, const double *__restrict__ dinv, int we,
-                                              double &a0, double &a1) {
-    const int lane = threadIdx.x & 31;
-#pragma unroll 8
-    for (int q = 0; q < we; q++) {
-        const double xq = __shfl_sync(0xffffffffu, q < 32 ? a0 : a1, q & 31) * dinv[q];
-        if (lane == (q & 31)) {
-            if (q < 32) a0 = xq; else a1 = xq;
-        }
-        if (lane > q && lane < we) a0 -= Lb[lane + q * kSLD] * xq;
-        if (lane + 32 > q && lane + 32 < we) a1 -= Lb[lane + 32 + q * kSLD] * xq;
+// 256 threads: out[i] = sum_q M[i + q 64] v[q] (trans = 0) or sum_q M[q + i 64] v[q]
+// (trans = 1) for the 64 x 64 column-major M; thread (i, g) sums q in [16 g, 16 g + 16)
+// from registers mr[16] (prefetched with oz_prefetch_inv), then the four quarters are
+// added in a fixed order (deterministic).
+__device__ __forceinline__ void inv_prefetch(const double *__restrict__ M, bool trans, double (&mr)[16]) {
+    const int i = threadIdx.x & 63, g = threadIdx.x >> 6;
+#pragma unroll
+    for (int u = 0; u < 16; u++) {
+        const int q = 16 * g + u;
+        mr[u] = __ldg(trans ? M + q + i * kSW : M + i + q * kSW);
     }
 }
-// One warp: x = L_bb^{-T} t (backward, right-looking on the transpose).
-__device__ __forceinline__ void warp_trsv_bwd(const double *__restrict__ Lb, const double *__restrict__ dinv, int we,
-                                              double &a0, double &a1) {
-    const int lane = threadIdx.x & 31;
-#pragma unroll 8
-    for (int q = we - 1; q >= 0; q--) {
-        const double xq = __shfl_sync(0xffffffffu, q < 32 ? a0 : a1, q & 31) * dinv[q];
-        if (lane == (q & 31)) {
-            if (q < 32) a0 = xq; else a1 = xq;
-        }
-        if (lane < q) a0 -= Lb[q + lane * kSLD] * xq;
-        if (lane + 32 < q) a1 -= Lb[q + (lane + 32) * kSLD] * xq;
-    }
+__device__ __forceinline__ double inv_apply(const double (&mr)[16], const double *__restrict__ v,
+                                            double (*red)[kSW]) {
+    const int i = threadIdx.x & 63, g = threadIdx.x >> 6;
+    double a = 0.0;
+#pragma unroll
+    for (int u = 0; u < 16; u++) a = fma(mr[u], v[16 * g + u], a);
+    red[g][i] = a;
+    __syncthreads();
+    return (red[0][i] + red[1][i]) + (red[2][i] + red[3][i]);   // valid for threads < 64
 }
 
+// Forward: CTA = 256-row chunk c of front s; for each 64-column block b whose rows
+// reach the chunk: every row's slab L(r, b) is loaded before any wait; the chunk that
+// holds block b's rows (the owner) forms x_b = inv(L_bb) t_b with all 256 threads
+// and publishes it (flag = solve epoch); the others wait for it; then every row
+// applies v_r -= L(r, b) x_b.  The owner's own block rows take no part in that
+// product (their slab entries are zeroed): their value becomes x.
 __device__ __forceinline__ void fsolve_df_task(const DevPlan &d, const int32_t *__restrict__ tasks, int w,
                                                double *__restrict__ y, const int task) {
-    __shared__ double Lb[kSW * kSLD];
-    __shared__ double xs[kSW], dinv[kSW];
+    __shared__ double xs[kSW];
+    __shared__ double red[4][kSW];
     const int s = tasks[2 * task], c = tasks[2 * task + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
     const double *__restrict__ P = d.L + d.L_off[s];
+    const double *__restrict__ Dinv = d.dinv + d.dinv_off[s];
     double *__restrict__ v = d.fv + d.fv_off[s];
     unsigned *__restrict__ bflag = d.df_flags + d.df_blk_off[s];
     const unsigned epoch = *d.solve_epoch;
-    const int tid = threadIdx.x, lane = tid & 31;
+    const int tid = threadIdx.x;
     const int c_lo = c * kSolveRows, c_hi = min(c_lo + kSolveRows, f);
     const int r = c_lo + tid;
     const bool rok = r < c_hi;
@@ -1467,26 +1489,28 @@ __device__ __forceinline__ void fsolve_df_task(const DevPlan &d, const int32_t *
     for (int b = 0; b < nb; b++) {
         const int j0 = b * w, we = min(w, k - j0);
         if (j0 >= c_hi) break;   // blocks below this chunk never update it
-        // this row's slab of the block (needs no x): issued before any wait; the
-        // owner's rows of the block carry the diagonal block itself
+        // this row's slab of the block (needs no x): issued before any wait
         load_row_block(P, ld, r, j0, we, rok && r >= j0, Lr);
-        if (j0 >= c_lo) {        // this chunk owns the block: solve its triangle
+        if (j0 >= c_lo) {        // this chunk owns the block: x_b = inv(L_bb) t_b
+            double mr[16];
+            inv_prefetch(Dinv + (int64_t)b * kSW * kSW, false, mr);
             const int i = r - j0;
-            if (rok && i >= 0 && i < we) stash_diag_row(Lr, i, vr, Lb, dinv, xs);
-            if (tid >= we && tid < kSW) xs[tid] = 0.0;
-            __syncthreads();
-            if (tid < 32) {
-                double a0 = xs[lane], a1 = xs[lane + 32];
-                warp_trsv_fwd(Lb, dinv, we, a0, a1);
-                xs[lane] = a0;
-                xs[lane + 32] = a1;
-                if (lane < we) y[first + j0 + lane] = a0;
-                if (lane + 32 < we) y[first + j0 + lane + 32] = a1;
-                __threadfence();
+            const bool own = rok && i >= 0 && i < we;
+            if (own) {
+                xs[i] = vr;
+#pragma unroll
+                for (int q = 0; q < kSW; q++) Lr[q] = 0.0;
             }
+            if (tid < kSW && !(tid < we && j0 + tid < c_hi)) xs[tid] = 0.0;
+            __syncthreads();
+            const double xb = inv_apply(mr, xs, red);
+            if (tid < we) y[first + j0 + tid] = xb;
+            __syncthreads();     // every thread read xs / red
+            if (tid < kSW) xs[tid] = tid < we ? xb : 0.0;
+            __threadfence();
             __syncthreads();
             if (tid == 0) st_release_u32(bflag + b, epoch);
-            if (rok && i >= 0 && i < we) vr = xs[i];
+            if (own) vr = xs[i];
         } else {                 // a block above: wait for its solution
             if (tid == 0)
                 while (ld_acquire_u32(bflag + b) != epoch) __nanosleep(32);
@@ -1531,11 +1555,11 @@ __device__ __forceinline__ void warp_reduce_scatter64(double (&p)[kSW]) {
 __device__ __forceinline__ void bsolve_df_task(const DevPlan &d, const int32_t *__restrict__ tasks, int w,
                                                double *__restrict__ y, const int task) {
     __shared__ double red[kSolveThreads / 32][kSW];
-    __shared__ double Lb[kSW * kSLD];
-    __shared__ double tv[kSW], dinv[kSW];
+    __shared__ double tv[kSW];
     const int s = tasks[2 * task], c = tasks[2 * task + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
     const double *__restrict__ P = d.L + d.L_off[s];
+    const double *__restrict__ Dinv = d.dinv + d.dinv_off[s];
     double *__restrict__ v = d.fv + d.fv_off[s];
     const int nb = (k + w - 1) / w, nc = (f + kSolveRows - 1) / kSolveRows;
     unsigned *__restrict__ cflag = d.df_flags + d.df_blk_off[s] + nb;
@@ -1551,9 +1575,11 @@ __device__ __forceinline__ void bsolve_df_task(const DevPlan &d, const int32_t *
     for (int b = nb - 1; b >= 0; b--) {
         const int j0 = b * w, we = min(w, k - j0);
         if (j0 >= c_hi) continue;                // block below this chunk: it contributes nothing
+        const bool owner = j0 >= c_lo;
+        double mr[16];
+        if (owner) inv_prefetch(Dinv + (int64_t)b * kSW * kSW, true, mr);
         // partial L(rows, b)^T x(rows) over this chunk's rows below the block
-        load_row_block(P, ld, r, j0, we, rok && r >= j0, pr);
-        if (rok && r >= j0 && r < j0 + we) stash_diag_row(pr, r - j0, 0.0, Lb, dinv, tv);   // owner's block rows
+        load_row_block(P, ld, r, j0, we, rok && r >= j0 + (owner ? we : 0), pr);   // the owner's block rows: none
 #pragma unroll
         for (int q = 0; q < kSW; q++) pr[q] *= xr;
         warp_reduce_scatter64(pr);
@@ -1564,44 +1590,36 @@ __device__ __forceinline__ void bsolve_df_task(const DevPlan &d, const int32_t *
         if (tid < we)
 #pragma unroll
             for (int q = 0; q < kSolveThreads / 32; q++) mine += red[q][tid];
-        if (j0 < c_lo) {                          // not the owner: publish the partial
+        // the partial of every chunk below, accumulated down the chunks: chunk cc publishes
+        // S_cc(b) = own_cc(b) + S_{cc+1}(b) (a fixed order: deterministic), so the owner
+        // reads one vector instead of summing all the chunks below on its critical path,
+        // and the chunks pass the sums along like a systolic array
+        double below = 0.0;
+        if (c + 1 < nc) {
+            if (tid == 0)
+                for (;;) {
+                    const unsigned fl = ld_acquire_u32(cflag + c + 1);
+                    if ((fl >> 12) == epoch && (fl & 0xfffu) >= (unsigned)(nb - b)) break;
+                    __nanosleep(32);
+                }
+            __syncthreads();
+            if (tid < we) below = __ldcg(part + ((int64_t)(c + 1) * nb + b) * w + tid);
+        }
+        if (!owner) {                             // publish own + everything below
             if (tid < we) {
-                part[((int64_t)c * nb + b) * w + tid] = mine;
+                part[((int64_t)c * nb + b) * w + tid] = mine + below;
                 __threadfence();
             }
             __syncthreads();
             if (tid == 0) st_release_u32(cflag + c, (epoch << 12) | (unsigned)(nb - b));
             continue;
         }
-        // owner: t = y_b - own partial - partials of every chunk below, in chunk order
-        if (warp == kSolveThreads / 32 - 1)   // poll every chunk below in parallel (its counter only grows)
-            for (int cc = c + 1 + lane; cc < nc; cc += 32)
-                for (;;) {
-                    const unsigned fl = ld_acquire_u32(cflag + cc);
-                    if ((fl >> 12) == epoch && (fl & 0xfffu) >= (unsigned)(nb - b)) break;
-                    __nanosleep(32);
-                }
+        if (tid < kSW) tv[tid] = tid < we ? y[first + j0 + tid] - (mine + below) : 0.0;
         __syncthreads();
-        if (tid < we) {
-            double t = y[first + j0 + tid] - mine;
-            const double *__restrict__ pc = part + (int64_t)b * w + tid;
-#pragma unroll 8
-            for (int cc = c + 1; cc < nc; cc++) t -= __ldcg(pc + (int64_t)cc * nb * w);
-            tv[tid] = t;
-        }
-        __syncthreads();
-        if (tid < 32) {
-            double a0 = lane < we ? tv[lane] : 0.0, a1 = lane + 32 < we ? tv[lane + 32] : 0.0;
-            warp_trsv_bwd(Lb, dinv, we, a0, a1);
-            if (lane < we) {
-                tv[lane] = a0;
-                y[first + j0 + lane] = a0;
-            }
-            if (lane + 32 < we) {
-                tv[lane + 32] = a1;
-                y[first + j0 + lane + 32] = a1;
-            }
-        }
+        const double xb = inv_apply(mr, tv, red);   // x_b = inv(L_bb)^T t
+        if (tid < we) y[first + j0 + tid] = xb;
+        __syncthreads();                            // tv / red read by every thread
+        if (tid < kSW) tv[tid] = tid < we ? xb : 0.0;
         __syncthreads();
         if (rok && r >= j0 && r < j0 + we) xr = tv[r - j0];
         __syncthreads();

@@ -30,6 +30,8 @@ struct DevPlan {
     unsigned *df_flags;      // dataflow solve flags (forward per block, backward per chunk)
     double *df_parts;        // dataflow backward partial sums per (chunk, block)
     const int64_t *df_blk_off, *df_part_off;
+    double *dinv;            // dataflow solve: inverses of the 64 x 64 diagonal blocks (solve setup)
+    const int64_t *dinv_off; // per supernode: word offset of its blocks in dinv (-1: none)
     const int32_t *ea_qs;    // fused extend-add: tile-row start tables of the syrk problems
     int fuse_ea;             // 1: large-front assembly covers the panel columns only
 };
@@ -71,6 +73,8 @@ void launch_permute_out(const DevPlan &d, const double *xf, double *x, int64_t n
 void launch_fwd_solve(const DevPlan &d, const int32_t *list, int count, double *y, cudaStream_t st);
 void launch_bwd_solve(const DevPlan &d, const int32_t *list, int count, double *y, const int32_t *sn_rows,
                       const int64_t *sn_rowptr, cudaStream_t st);
+// solve setup: inverses of the 64 x 64 diagonal blocks of the dataflow-solved supernodes
+void launch_diag_inv(const DevPlan &d, const int32_t *tasks, int64_t count, int w, cudaStream_t st);
 void launch_fsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, cudaStream_t st);
 void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, unsigned *tk,
                       cudaStream_t st);

@@ -229,6 +229,12 @@ struct Plan {
     std::vector<int32_t> df_tasks;                   // dataflow solve: (front, chunk) pairs
     std::vector<int64_t> df_blk_off, df_part_off;    // per supernode: block-flag and partial-sum bases
     int64_t df_nflags = 0, df_nparts = 0;            // u32 flags / fp64 partial words
+    // inverses of the 64 x 64 diagonal blocks of the dataflow-solved supernodes (solve setup,
+    // computed once per factorization by the first solve): per supernode the word offset of
+    // its ceil(k / 64) column-major 64 x 64 blocks; (supernode, block) task pairs
+    std::vector<int64_t> dinv_off;
+    std::vector<int32_t> dinv_tasks;
+    int64_t dinv_words = 0;
     std::vector<SolveLaunch> fsolve, bsolve;
     // ---- multi-GPU: subtree-to-GPU mapping.  Subtrees below a
     // frontier are factored by their owner; the supernodes above the frontier ("top")

@@ -101,6 +101,9 @@ static void build_solve_plan(const Symbolic &S, Plan &P, const std::vector<char>
         const int64_t nb = (P.sn_k[s] + w - 1) / w, nc = (P.sn_f[s] + kSolveRows - 1) / kSolveRows;
         P.df_blk_off[s] = P.df_nflags;
         P.df_nflags += nb + nc;   // nb forward block flags, then nc backward chunk flags
+        P.dinv_off[s] = P.dinv_words;
+        P.dinv_words += nb * 64 * 64;   // one 64 x 64 slot per block (w <= 64; identity-extended)
+        for (int32_t b = 0; b < nb; b++) P.dinv_tasks.insert(P.dinv_tasks.end(), {s, b});
         P.df_part_off[s] = P.df_nparts;
         P.df_nparts += nc * nb * w;
     };
@@ -1085,6 +1088,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         if ((g.a_off & 1) || (g.lda & 1)) return MF_ERR_STATE;
     P.df_blk_off.assign(ns, -1);
     P.df_part_off.assign(ns, -1);
+    P.dinv_off.assign(ns, -1);
     build_solve_plan(S, P, inc_local, P.fsolve, P.bsolve);
     build_solve_plan(S, P, inc_top_solve, P.fsolve_top, P.bsolve_top);
     return plan_ozaki(P, opt.ozaki_slices);
