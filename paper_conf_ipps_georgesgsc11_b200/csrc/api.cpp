@@ -13,6 +13,7 @@
 #include <climits>
 #include <cstdio>
 #include <cstring>
+#include <cstdlib>
 #include <new>
 #include <map>
 #include <vector>
@@ -551,8 +552,17 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
         CK(cudaStreamCreateWithPriority(&c->la_side, cudaStreamNonBlocking, least));
         for (cudaEvent_t &e : c->la_ev) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     }
-    // the L arena starts zeroed once so that never-written padding words are defined
-    CK(cudaMemsetAsync(d.L, 0, (P.L_words + kTileM) * sizeof(double), c->stream));
+    // the L arena starts zeroed once so that never-written padding words are defined.
+    // MF_DEBUG_NANFILL=1 (debug): fill the L / U / front-vector arenas with NaN
+    // instead -- every word a kernel reads into a real output must have been written
+    // by this factorization first (tests/test_gpu_parity.py runs it bitwise vs 0-fill)
+    const char *nanfill = getenv("MF_DEBUG_NANFILL");
+    const int fillb = (nanfill && atoi(nanfill) == 1) ? 0xff : 0;
+    CK(cudaMemsetAsync(d.L, fillb, (P.L_words + kTileM) * sizeof(double), c->stream));
+    if (fillb) {
+        CK(cudaMemsetAsync(d.U, fillb, P.U_words * sizeof(double), c->stream));
+        CK(cudaMemsetAsync(d.fv, fillb, P.fv_words * sizeof(double), c->stream));
+    }
     CK(cudaStreamSynchronize(c->stream));
 
     fill_info(c, n, 1);

@@ -42,12 +42,16 @@ def host_tensor(ptr: int, nbytes: int, int32: bool = False) -> torch.Tensor:
 
 
 class TorchDistExchange:
-    """NCCL collectives/point-to-point through the default torch.distributed group
-    (``host=True``: the pointers are host memory, e.g. gloo tests on CPU)."""
+    """NCCL collectives/point-to-point through the default torch.distributed group.
+    ``host=True``: the pointers are host memory (gloo tests on CPU).
+    ``stage=True``: the pointers are device memory but the group's backend cannot
+    touch it (gloo): every buffer is staged through a host copy -- lets several
+    ranks share ONE GPU in tests (NCCL refuses two ranks on one device)."""
 
-    def __init__(self, host: bool = False):
+    def __init__(self, host: bool = False, stage: bool = False):
         self.view = host_tensor if host else device_tensor
         self.host = host
+        self.stage = stage and not host
         self._first = True
 
     def __call__(self, ops):
@@ -56,6 +60,15 @@ class TorchDistExchange:
             dist.barrier()
             self._first = False
         view = self.view
+        if self.stage:   # device buffers through host copies (gloo), written back after the transfers
+            torch.cuda.synchronize()
+            staged = []
+
+            def view(ptr, nbytes, int32=False, _dev=device_tensor):
+                d = _dev(ptr, nbytes, int32=int32)
+                h = d.cpu()
+                staged.append((d, h))
+                return h
         p2p = []
         for op, peer, ptr, nbytes in ops:
             if op in (MF_XFER_SEND, MF_XFER_RECV):
@@ -71,6 +84,9 @@ class TorchDistExchange:
                 dist.all_reduce(view(ptr, nbytes))
             elif op == MF_XFER_ALLREDUCE_MIN_I32:
                 dist.all_reduce(view(ptr, nbytes, int32=True), op=dist.ReduceOp.MIN)
+        if self.stage:
+            for d, h in staged:
+                d.copy_(h)
         if not self.host:
             torch.cuda.synchronize()
 

@@ -235,3 +235,79 @@ def test_loopback_not_spd_reported_on_every_rank():
     for t in th:
         t.join()
     assert cols == [victim] * R
+
+
+def _staged_worker(rank, world, port, dims, q):
+    """One rank of a real torch.distributed job on ONE GPU: gloo with host staging
+    (TorchDistExchange(stage=True)); returns the hashes of its panels."""
+    import hashlib
+    import oracle
+    from workloads import grids as G
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_ipps_georgesgsc11_b200.exchange import TorchDistExchange
+        A0, p = grid("27pt", dims)
+        s0 = oracle.symbolic(A0, p, keep_struct=True)
+        A, _ = G.manufactured(A0.n, s0.Lp, s0.Li, s0.perm, seed=1234)
+        S = mf.Solver(nranks=world, rank=rank, exchange=TorchDistExchange(stage=True), split_all=True,
+                      panel_w=16)
+        S.analyze(A.n, A.colptr, A.rowind, s0.perm)
+        # only rank 0's values are read: the others pass NaN
+        S.factor(A.values if rank == 0 else np.full_like(A.values, np.nan))
+        owner, top, _, _ = S.mapping()
+        sn = S.supernodes()
+        h = {}
+        for s in range(S.info()["nsuper"]):
+            if top[s] or owner[s] == rank:
+                f = int(sn["sn_rowptr"][s + 1] - sn["sn_rowptr"][s])
+                k = int(sn["sn_first"][s + 1] - sn["sn_first"][s])
+                h[s] = hashlib.sha256(S.panel(s, f, k).tobytes()).hexdigest()
+        b = np.arange(A.n, dtype=np.float64) % 7 - 3.0
+        x = S.solve(b if rank == 0 else np.zeros_like(b))
+        q.put((rank, h, hashlib.sha256(x.tobytes()).hexdigest(), int(S.cooperative().sum())))
+    except Exception as e:  # noqa: BLE001
+        import traceback
+        q.put((rank, None, traceback.format_exc(), 0))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("dims", [(14, 14, 14), (16, 15, 14)])
+def test_torchdist_two_processes_one_gpu_bitwise(dims):
+    """the real TorchDistExchange (torch.distributed, here gloo with host
+    staging: two processes on one GPU) reproduces the single-rank factor BITWISE on
+    manufactured input (SURVEY.md Sec. 8(c) multi-GPU pin), with cooperative top fronts,
+    rank 0's values / b broadcast, and the same solve on every rank."""
+    import hashlib
+    import oracle
+    from workloads import grids as G
+    A0, p = grid("27pt", dims)
+    s0 = oracle.symbolic(A0, p, keep_struct=True)
+    A, _ = G.manufactured(A0.n, s0.Lp, s0.Li, s0.perm, seed=1234)
+    ref = mf.Solver(panel_w=16)
+    ref.analyze(A.n, A.colptr, A.rowind, s0.perm)
+    ref.factor(A.values)
+    b = np.arange(A.n, dtype=np.float64) % 7 - 3.0
+    xref = hashlib.sha256(ref.solve(b).tobytes()).hexdigest()
+    sn = ref.supernodes()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = 29700 + os.getpid() % 1000
+    procs = [ctx.Process(target=_staged_worker, args=(r, 2, port, dims, q)) for r in range(2)]
+    for pr in procs:
+        pr.start()
+    res = dict((r, (h, x, nc)) for r, h, x, nc in (q.get(timeout=900) for _ in procs))
+    for pr in procs:
+        pr.join(timeout=120)
+    for r in range(2):
+        h, x, nc = res[r]
+        assert h is not None, x
+        assert nc > 0   # cooperative top fronts exercised
+        for s, hs in h.items():
+            f = int(sn["sn_rowptr"][s + 1] - sn["sn_rowptr"][s])
+            k = int(sn["sn_first"][s + 1] - sn["sn_first"][s])
+            assert hs == hashlib.sha256(ref.panel(s, f, k).tobytes()).hexdigest(), (r, s)
+        assert x == xref, r
