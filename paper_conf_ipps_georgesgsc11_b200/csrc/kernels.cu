@@ -1400,6 +1400,32 @@ __device__ __forceinline__ void load_row_block(const double *__restrict__ P, int
     for (int q = 0; q < kSW; q++) Lr[q] = (ok && q < we) ? col[(int64_t)q * ld] : 0.0;
 }
 
+// Half a row slab: row r's 32 entries of the columns [j0 + 32 h, j0 + 32 h + 32) of a
+// block (zero past we or when !ok).  The sweeps below keep two halves in registers:
+// while one is used, the next one is in flight (software pipelining across blocks).
+__device__ __forceinline__ void load_half(const double *__restrict__ P, int64_t ld, int r, int j0, int h, int we,
+                                          bool ok, double (&Lh)[32]) {
+    const double *__restrict__ col = P + (int64_t)(j0 + 32 * h) * ld + r;
+#pragma unroll
+    for (int q = 0; q < 32; q++) Lh[q] = (ok && 32 * h + q < we) ? col[(int64_t)q * ld] : 0.0;
+}
+// Butterfly reduce-scatter over the warp: 32 values per lane in, lane l ends with the
+// warp sum of value l in p[0] (31 shuffles).
+__device__ __forceinline__ void warp_reduce_scatter32(double (&p)[32]) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int st = 0; st < 5; st++) {
+        const int half = 16 >> st, off = 16 >> st;
+        const bool up = (lane & off) != 0;
+#pragma unroll
+        for (int i = 0; i < half; i++) {
+            const double send = up ? p[i] : p[i + half];
+            const double keep = up ? p[i + half] : p[i];
+            p[i] = keep + __shfl_xor_sync(0xffffffffu, send, off);
+        }
+    }
+}
+
 // ---- solve setup: inv(L_bb) of every 64 x 64 diagonal block of the dataflow-solved
 // supernodes (once per factorization, by the first solve), so the block chains of the
 // sweeps below apply a 64 x 64 matrix-vector product (x_b = inv(L_bb) t_b, all threads)
@@ -1463,11 +1489,12 @@ __device__ __forceinline__ double inv_apply(const double (&mr)[16], const double
 }
 
 // Forward: CTA = 256-row chunk c of front s; for each 64-column block b whose rows
-// reach the chunk: every row's slab L(r, b) is loaded before any wait; the chunk that
-// holds block b's rows (the owner) forms x_b = inv(L_bb) t_b with all 256 threads
-// and publishes it (flag = solve epoch); the others wait for it; then every row
-// applies v_r -= L(r, b) x_b.  The owner's own block rows take no part in that
-// product (their slab entries are zeroed): their value becomes x.
+// reach the chunk: every row's slab L(r, b) is in registers (two 32-column halves,
+// each loaded one half ahead of its use, so a lagging chunk streams its slabs
+// instead of paying a load latency per block); the chunk that holds block b's rows
+// (the owner) forms x_b = inv(L_bb) t_b with all 256 threads and publishes it (flag
+// = solve epoch); the others wait for it; then every row applies v_r -= L(r, b) x_b.
+// The owner's own block rows take no part in that product: their value becomes x.
 __device__ __forceinline__ void fsolve_df_task(const DevPlan &d, const int32_t *__restrict__ tasks, int w,
                                                double *__restrict__ y, const int task) {
     __shared__ double xs[kSW];
@@ -1484,13 +1511,13 @@ __device__ __forceinline__ void fsolve_df_task(const DevPlan &d, const int32_t *
     const int r = c_lo + tid;
     const bool rok = r < c_hi;
     double vr = rok ? v[r] : 0.0;
-    const int nb = (k + w - 1) / w;
-    double Lr[kSW];
+    const int nb = min((k + w - 1) / w, (c_hi + w - 1) / w);   // blocks reaching this chunk
+    double H0[32], H1[32];
+    if (nb > 0) load_half(P, ld, r, 0, 0, min(w, k), rok, H0);
     for (int b = 0; b < nb; b++) {
         const int j0 = b * w, we = min(w, k - j0);
-        if (j0 >= c_hi) break;   // blocks below this chunk never update it
-        // this row's slab of the block (needs no x): issued before any wait
-        load_row_block(P, ld, r, j0, we, rok && r >= j0, Lr);
+        const bool okr = rok && r >= j0;
+        load_half(P, ld, r, j0, 1, we, okr, H1);   // second half in flight
         if (j0 >= c_lo) {        // this chunk owns the block: x_b = inv(L_bb) t_b
             double mr[16];
             inv_prefetch(Dinv + (int64_t)b * kSW * kSW, false, mr);
@@ -1499,9 +1526,9 @@ __device__ __forceinline__ void fsolve_df_task(const DevPlan &d, const int32_t *
             if (own) {
                 xs[i] = vr;
 #pragma unroll
-                for (int q = 0; q < kSW; q++) Lr[q] = 0.0;
+                for (int q = 0; q < 32; q++) H0[q] = H1[q] = 0.0;
             }
-            if (tid < kSW && !(tid < we && j0 + tid < c_hi)) xs[tid] = 0.0;
+            if (tid < kSW && tid >= we) xs[tid] = 0.0;
             __syncthreads();
             const double xb = inv_apply(mr, xs, red);
             if (tid < we) y[first + j0 + tid] = xb;
@@ -1515,16 +1542,25 @@ __device__ __forceinline__ void fsolve_df_task(const DevPlan &d, const int32_t *
             if (tid == 0)
                 while (ld_acquire_u32(bflag + b) != epoch) __nanosleep(32);
             __syncthreads();
-            if (tid < kSW) xs[tid] = tid < we ? __ldcg(y + first + j0 + tid) : 0.0;   // (Lr = 0 past we; 0 * junk)
+            if (tid < kSW) xs[tid] = tid < we ? __ldcg(y + first + j0 + tid) : 0.0;
             __syncthreads();
         }
         double a0 = 0.0, a1 = 0.0;
 #pragma unroll
-        for (int q = 0; q < kSW; q += 2) {
-            a0 += Lr[q] * xs[q];
-            a1 += Lr[q + 1] * xs[q + 1];
+        for (int q = 0; q < 32; q += 2) {
+            a0 += H0[q] * xs[q];
+            a1 += H0[q + 1] * xs[q + 1];
         }
-        vr -= a0 + a1;           // rows not below the block have Lr = 0 (and xs past we is not read: Lr = 0)
+        if (b + 1 < nb) {        // the next block's first half, while the second half is used
+            const int j1 = j0 + w;
+            load_half(P, ld, r, j1, 0, min(w, k - j1), rok && r >= j1, H0);
+        }
+#pragma unroll
+        for (int q = 0; q < 32; q += 2) {
+            a0 += H1[q] * xs[32 + q];
+            a1 += H1[q + 1] * xs[33 + q];
+        }
+        vr -= a0 + a1;           // rows not below the block have zero slabs
         __syncthreads();
     }
     if (rok && r >= k) v[r] = vr;   // the update vector the parent gathers
@@ -1569,22 +1605,34 @@ __device__ __forceinline__ void bsolve_df_task(const DevPlan &d, const int32_t *
     const int c_lo = c * kSolveRows, c_hi = min(c_lo + kSolveRows, f);
     const int r = c_lo + tid;
     const bool rok = r < c_hi;
-    const int qlane = 2 * lane;
     double xr = (rok && r >= k) ? v[r] : 0.0;   // rows >= k: final (gathered from the ancestors)
-    double pr[kSW];
-    for (int b = nb - 1; b >= 0; b--) {
+    const int btop = min(nb, (c_hi + w - 1) / w) - 1;   // the first block (from the bottom) reaching this chunk
+    // rows taking part in block b's partial: below the block (the owner's own block rows: none)
+    auto rows_ok = [&](int b) {
+        const int j0 = b * w;
+        return rok && r >= j0 + (j0 >= c_lo ? min(w, k - j0) : 0);
+    };
+    double H0[32], H1[32];
+    if (btop >= 0) load_half(P, ld, r, btop * w, 0, min(w, k - btop * w), rows_ok(btop), H0);
+    for (int b = btop; b >= 0; b--) {
         const int j0 = b * w, we = min(w, k - j0);
-        if (j0 >= c_hi) continue;                // block below this chunk: it contributes nothing
         const bool owner = j0 >= c_lo;
+        load_half(P, ld, r, j0, 1, we, rows_ok(b), H1);   // second half in flight
         double mr[16];
         if (owner) inv_prefetch(Dinv + (int64_t)b * kSW * kSW, true, mr);
-        // partial L(rows, b)^T x(rows) over this chunk's rows below the block
-        load_row_block(P, ld, r, j0, we, rok && r >= j0 + (owner ? we : 0), pr);   // the owner's block rows: none
+        // partial L(rows, b)^T x(rows) over this chunk's rows below the block, per half
 #pragma unroll
-        for (int q = 0; q < kSW; q++) pr[q] *= xr;
-        warp_reduce_scatter64(pr);
-        red[warp][qlane] = pr[0];
-        red[warp][qlane + 1] = pr[1];
+        for (int q = 0; q < 32; q++) H0[q] *= xr;
+        warp_reduce_scatter32(H0);
+        red[warp][lane] = H0[0];
+        if (b > 0) {             // the next block's first half, while this half is reduced
+            const int j1 = j0 - w;
+            load_half(P, ld, r, j1, 0, min(w, k - j1), rows_ok(b - 1), H0);
+        }
+#pragma unroll
+        for (int q = 0; q < 32; q++) H1[q] *= xr;
+        warp_reduce_scatter32(H1);
+        red[warp][32 + lane] = H1[0];
         __syncthreads();
         double mine = 0.0;
         if (tid < we)
