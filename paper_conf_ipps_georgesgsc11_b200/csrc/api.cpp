@@ -640,7 +640,7 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
                     if (L.oz)   // int8 tensor cores, Ozaki scheme
                         launch_update_oz(d, c->d_probs, c->d_oz_probs, c->d_oz_split + 3 * L.oz_s, L.oz_ns,
                                          c->d_oz_tiles + L.oz_t, L.oz_nt, c->d_oz_scratch, c->d_oz_expo + L.oz_e,
-                                         L.oz_ne, P.oz_slices, st);
+                                         L.oz_ne, P.oz_slices, L.oz_wide, st);
                     else
                         launch_update(d, c->d_probs, c->d_tiles + L.off, L.count,
                                       L.count > 0 ? L.flops / (2.0 * kTileM * kTileN * L.count) : 0.0, st);

@@ -1233,15 +1233,15 @@ int kernels_init() {
 // Ozaki-scheme Schur update of one KC_UPDATE launch (S = slices, 3..8)
 void launch_update_oz(const DevPlan &d, const GemmProb *probs, const OzProb *oprobs, const int32_t *split,
                       int64_t nsplit, const OzTile *tiles, int64_t ntiles, int8_t *scratch, int32_t *expo,
-                      int64_t expo_words, int S, cudaStream_t st) {
+                      int64_t expo_words, int S, int wide, cudaStream_t st) {
     const UpdGather gv{d.child_ptr, d.child_list, d.sn_k, d.sn_f, d.U_off, d.relmap_ptr, d.relmap, d.ea_qs};
     switch (S) {
-        case 3: launch_oz<3>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv); break;
-        case 4: launch_oz<4>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv); break;
-        case 5: launch_oz<5>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv); break;
-        case 6: launch_oz<6>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv); break;
-        case 7: launch_oz<7>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv); break;
-        default: launch_oz<8>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv); break;
+        case 3: launch_oz<3>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv, wide); break;
+        case 4: launch_oz<4>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv, wide); break;
+        case 5: launch_oz<5>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv, wide); break;
+        case 6: launch_oz<6>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv, wide); break;
+        case 7: launch_oz<7>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv, wide); break;
+        default: launch_oz<8>(d.L, d.U, probs, oprobs, split, nsplit, tiles, ntiles, scratch, expo, expo_words, st, gv, wide); break;
     }
 }
 

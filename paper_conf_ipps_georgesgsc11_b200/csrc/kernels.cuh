@@ -61,7 +61,7 @@ void launch_update(const DevPlan &d, const GemmProb *probs, const TileTask *tile
 // Schur update of one launch on the int8 tensor cores (Ozaki scheme, S slices)
 void launch_update_oz(const DevPlan &d, const GemmProb *probs, const OzProb *oprobs, const int32_t *split,
                       int64_t nsplit, const OzTile *tiles, int64_t ntiles, int8_t *scratch, int32_t *expo,
-                      int64_t expo_words, int S, cudaStream_t st);
+                      int64_t expo_words, int S, int wide, cudaStream_t st);
 // fp64 iterative refinement (mixed-precision mode): B entry values, residual + norms, x += dx
 void launch_refine_bval(const DevPlan &d, const double *values, double *bval, int64_t nb, cudaStream_t st);
 void launch_refine_resid(const DevPlan &d, const int64_t *rs_ptr, const int32_t *rs_col, const int32_t *rs_ent,

@@ -181,6 +181,7 @@ struct Launch {
     // tasks (triples) [oz_s, oz_s + oz_ns), tiles [oz_t, oz_t + oz_nt); exponent
     // words [oz_e, oz_e + oz_ne) of the scratch
     int32_t oz = 0;
+    int32_t oz_wide = 0;   // Ozaki tiles of 128 x 128 (two-pass kernel) instead of 128 x 64
     double int8_ops = 0;   // int8 MMA operations of an Ozaki launch
     int64_t oz_p = 0, oz_np = 0, oz_s = 0, oz_ns = 0, oz_t = 0, oz_nt = 0, oz_e = 0, oz_ne = 0;
 };

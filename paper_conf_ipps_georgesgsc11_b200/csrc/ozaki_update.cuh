@@ -120,11 +120,12 @@ __device__ __forceinline__ uint64_t oz_desc(uint32_t saddr, uint32_t lbo, uint32
 constexpr uint32_t kOzIdesc = (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(kOzBN >> 3) << 17) |
                               ((uint32_t)(kOzBM >> 4) << 24);
 
-__device__ __forceinline__ void oz_mma(uint32_t dtmem, uint64_t adesc, uint64_t bdesc, uint32_t acc) {
+__device__ __forceinline__ void oz_mma(uint32_t dtmem, uint64_t adesc, uint64_t bdesc, uint32_t acc,
+                                       uint32_t idesc = kOzIdesc) {
     asm volatile(
         "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
         " tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n}\n" ::"r"(dtmem),
-        "l"(adesc), "l"(bdesc), "r"(kOzIdesc), "r"(acc)
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc)
         : "memory");
 }
 __device__ __forceinline__ void oz_commit(uint64_t *bar) {
@@ -320,16 +321,221 @@ __global__ void __launch_bounds__(kOzThreads, 1)
     }
 }
 
+
+// ------------------------------------------------------------------ 128 x 128 tiles, two passes
+// Measured (tools/ubench/ozaki_gemm.cu, 8192^2 x 4096 SYRK): S = 4 in one pass 2.30 ms
+// vs 3.16 ms with 128 x 64 tiles; S = 8 in two passes 5.56 vs 5.45 ms -- per output
+// element both move the same slice bytes from L2 (12 slice loads over 256 rows vs 8
+// over 192), which bounds them at ~5 TB/s of L2 -> shared-memory traffic.
+// k_oz_gemm2: the same product on 128 x 128 output tiles.  N = 128 halves the
+// shared-memory operand traffic per MMA (A 4 KB + B 4 KB per 64 cycles = 128 B/clk,
+// vs 192 B/clk for N = 64), but S accumulators of 128 columns do not fit TMEM, so
+// the diagonals are taken in two passes of at most four (pass 0: d = s + t <= 3,
+// slices 0..3, 64-byte k stages; pass 1: 4 <= d <= S - 1, all slices, 32-byte k
+// stages -- both 64 KB per stage).  Roles: warps 0-3 = epilogue (TMEM lane quarters),
+// warp 4 = producer (cp.async.bulk, runs ahead into pass 1 while pass 0 drains), warp
+// 5 = MMA issuer (waits for the epilogue to release TMEM before pass 1).  Pass 0's
+// epilogue writes C = (C or the gathered sum of the children's U^c) - P_0, pass 1's
+// C -= P_1 (each element by one thread: a fixed order).
+constexpr int kOz2BN = 128, kOz2Threads = 192, kOz2Stage = 64 * 1024, kOz2Stages = 3;
+constexpr uint32_t kOz2Idesc = (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(kOz2BN >> 3) << 17) |
+                               ((uint32_t)(kOzBM >> 4) << 24);
+constexpr size_t kOz2Smem = (size_t)kOz2Stages * kOz2Stage + 2048;
+
+__device__ __forceinline__ void oz2_bar_epi() { asm volatile("bar.sync 1, 128;\n" ::: "memory"); }
+
+template <int S>
+__global__ void __launch_bounds__(kOz2Threads, 1)
+    k_oz_gemm2(double *__restrict__ Larena, double *__restrict__ Uarena, const GemmProb *__restrict__ probs,
+               const OzProb *__restrict__ oprobs, const OzTile *__restrict__ tiles, const int8_t *__restrict__ slices,
+               const int32_t *__restrict__ expo, const UpdGather gv) {
+    constexpr int DA = S < 4 ? S : 4;                 // diagonals of pass 0
+    constexpr int NP = S > 4 ? 2 : 1;                 // passes
+    extern __shared__ __align__(1024) uint8_t osm[];
+    uint64_t *full = reinterpret_cast<uint64_t *>(osm + kOz2Stages * kOz2Stage);
+    uint64_t *empty = full + kOz2Stages;
+    uint64_t *tfull = empty + kOz2Stages;             // MMA -> epilogue, one phase per pass
+    uint64_t *tempty = tfull + 1;                     // epilogue -> MMA (TMEM released after pass 0)
+    uint32_t *tbase_sh = reinterpret_cast<uint32_t *>(tempty + 1);
+    int32_t *ej = reinterpret_cast<int32_t *>(tbase_sh + 1);   // E of the tile's 128 columns
+    int *rq = ej + kOz2BN, *cq = rq + kOzBM;          // gather maps
+    const OzTile t = tiles[blockIdx.x];
+    const OzProb o = oprobs[t.oprob];
+    const GemmProb g = probs[o.prob];
+    const int ti = t.tij >> 16, tj = t.tij & 0xffff;
+    const int i0 = ti * kOzBM, j0 = tj * kOz2BN;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int KC = o.Kpad / 16;
+
+    if (tid == 0) {
+        for (int st = 0; st < kOz2Stages; st++) {
+            mbar_init(full + st, 1);
+            mbar_init(empty + st, 1);
+        }
+        mbar_init(tfull, 1);
+        mbar_init(tempty, 4);
+        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+    }
+    if (warp == 2) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;\n" ::"r"(smem_u32(tbase_sh))
+                     : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n" ::: "memory");
+    }
+    if (tid < kOz2BN) ej[tid] = expo[o.ex_off + j0 + tid];
+    asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
+    const uint32_t tbase = *tbase_sh;
+    const int8_t *__restrict__ sl = slices + o.sl_off;
+    const int64_t kstride = (int64_t)o.Mpad * 16, sstride = (int64_t)KC * kstride;
+
+    if (warp == 4) {
+        // ---- producer: pass p stage = ns slices x nkc k-cores x (128 A rows + 128 B rows)
+        int gs = 0;
+        for (int p = 0; p < NP; p++) {
+            const int ns = p == 0 ? DA : S, nkc = ns <= 4 ? 4 : 2, KB = KC / nkc;
+            for (int kb = 0; kb < KB; kb++, gs++) {
+                const int st = gs % kOz2Stages;
+                if (gs >= kOz2Stages) mbar_wait(empty + st, ((gs / kOz2Stages) - 1) & 1);
+                if (lane == 0) mbar_arrive_tx(full + st, (unsigned)(2 * ns * nkc * kOzBM * 16));
+                __syncwarp();
+                uint8_t *As = osm + st * kOz2Stage, *Bs = As + ns * nkc * kOzBM * 16;
+                for (int c = lane; c < 2 * ns * nkc; c += 32) {
+                    const int isB = c >= ns * nkc, sc = isB ? c - ns * nkc : c, s = sc / nkc, kc = sc % nkc;
+                    const int8_t *src = sl + s * sstride + (int64_t)(kb * nkc + kc) * kstride +
+                                        (int64_t)(isB ? j0 : i0) * 16;
+                    bulk_g2s((isB ? Bs : As) + (s * nkc + kc) * (kOzBM * 16), src, kOzBM * 16, full + st);
+                }
+            }
+        }
+    } else if (warp == 5) {
+        // ---- MMA issuer
+        int gs = 0;
+        for (int p = 0; p < NP; p++) {
+            const int ns = p == 0 ? DA : S, nkc = ns <= 4 ? 4 : 2, KB = KC / nkc;
+            const int dlo = p == 0 ? 0 : DA, dhi = p == 0 ? DA : S;
+            if (p == 1) {   // TMEM is free once pass 0's epilogue has read it
+                mbar_wait(tempty, 0);
+                asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
+            }
+            for (int kb = 0; kb < KB; kb++, gs++) {
+                const int st = gs % kOz2Stages;
+                mbar_wait(full + st, (gs / kOz2Stages) & 1);
+                asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
+                if (lane == 0) {
+                    const uint32_t a0 = smem_u32(osm + st * kOz2Stage), b0 = a0 + ns * nkc * kOzBM * 16;
+                    for (int kk = 0; kk < nkc / 2; kk++)
+                        for (int s = 0; s < ns; s++) {
+                            const uint64_t ad = oz_desc(a0 + (s * nkc + 2 * kk) * (kOzBM * 16), kOzBM * 16, 128);
+                            for (int u = max(0, dlo - s); u < dhi - s && u < ns; u++) {
+                                const uint64_t bd = oz_desc(b0 + (u * nkc + 2 * kk) * (kOzBM * 16), kOzBM * 16, 128);
+                                oz_mma(tbase + (uint32_t)((s + u - dlo) * kOz2BN), ad, bd, (kb | kk | s) != 0, kOz2Idesc);
+                            }
+                        }
+                    oz_commit(empty + st);
+                }
+                __syncwarp();
+            }
+            if (lane == 0) oz_commit(tfull);
+            __syncwarp();
+        }
+    } else {
+        // ---- epilogue warps 0-3: thread = tile row (TMEM lane)
+        const int il = tid, i = i0 + il;
+        const int sh = (g.flags >> 1) & 1;
+        double *__restrict__ C = ((g.flags & 1) ? Uarena : Larena) + g.c_off;
+        const int64_t ldc = g.ldc;
+        const int Ei = expo[o.ex_off + i];
+        const bool row_ok = i < g.M && i >= sh;
+        const bool gather = (g.flags & 4) != 0;
+        if (gather) {   // C = 0 (+) U^c1 (+) U^c2 ..., in ascending child order (reading C6)
+            if (row_ok)
+                for (int c = 0; c < kOz2BN; c++) {
+                    const int j = j0 + c;
+                    if (j < g.N && i >= j && j >= sh) C[(i - sh) + (int64_t)(j - sh) * ldc] = 0.0;
+                }
+            const int q0 = gv.child_ptr[g.s], q1 = gv.child_ptr[g.s + 1], kp = gv.sn_k[g.s];
+            const int ntr1 = (g.M + kTileM - 1) / kTileM + 1;   // ea_qs tables are per 64-row tile
+            const int tr0 = i0 / kTileM, tr1 = min(tr0 + kOzBM / kTileM, ntr1 - 1);
+            const int tc0 = j0 / kTileN, tc1 = min(tc0 + kOz2BN / kTileN, ntr1 - 1);
+            for (int jc = 0; jc < q1 - q0; jc++) {
+                const int32_t *__restrict__ qs = gv.qs + g.qs_off + (int64_t)jc * ntr1;
+                const int ra = qs[tr0], rb = qs[tr1], ca = qs[tc0], cb = qs[tc1];
+                if (ra == rb || ca == cb) continue;   // uniform over the epilogue warps
+                const int ch = gv.child_list[q0 + jc];
+                const int mc = gv.sn_f[ch] - gv.sn_k[ch];
+                const int32_t *__restrict__ rel = gv.relmap + gv.relmap_ptr[ch];
+                const double *__restrict__ Uc = Uarena + gv.U_off[ch];
+                oz2_bar_epi();   // the previous child's maps are consumed
+                for (int x = tid; x < kOzBM + kOz2BN; x += 128) rq[x] = -1;
+                oz2_bar_epi();
+                for (int q = ra + tid; q < rb; q += 128) rq[__ldg(rel + q) - kp + sh - i0] = q;
+                for (int q = ca + tid; q < cb; q += 128) cq[__ldg(rel + q) - kp + sh - j0] = q;
+                oz2_bar_epi();
+                const int qi = rq[il];
+                if (qi >= 0 && row_ok)
+                    for (int c = 0; c < kOz2BN; c++) {
+                        const int qj = cq[c], j = j0 + c;
+                        if (qj >= 0 && qi >= qj && j < g.N && i >= j && j >= sh)
+                            C[(i - sh) + (int64_t)(j - sh) * ldc] += __ldg(Uc + qi + (int64_t)qj * mc);
+                    }
+            }
+        }
+        for (int p = 0; p < NP; p++) {
+            const int dlo = p == 0 ? 0 : DA, dhi = p == 0 ? DA : S;
+            mbar_wait(tfull, p & 1);
+            asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
+#pragma unroll 1
+            for (int c0 = 0; c0 < kOz2BN; c0 += 32) {
+                double v[32];
+#pragma unroll
+                for (int q = 0; q < 32; q++) v[q] = 0.0;
+#pragma unroll 1
+                for (int d = dhi - 1; d >= dlo; d--) {   // smallest weight first
+                    uint32_t r[32];
+                    OZ_LD32(tbase + ((uint32_t)(warp * 32) << 16) + (uint32_t)((d - dlo) * kOz2BN + c0), r);
+                    asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
+                    const double w = ldexp(1.0, -7 * (d + 2));
+#pragma unroll
+                    for (int q = 0; q < 32; q++) v[q] = fma((double)(int32_t)r[q], w, v[q]);
+                }
+                if (row_ok) {
+#pragma unroll
+                    for (int q = 0; q < 32; q++) {
+                        const int j = j0 + c0 + q;
+                        if (j < g.N && i >= j && j >= sh) {
+                            double *cp = C + (i - sh) + (int64_t)(j - sh) * ldc;
+                            *cp -= ldexp(v[q], Ei + ej[c0 + q]);
+                        }
+                    }
+                }
+            }
+            if (p + 1 < NP) {   // TMEM read: the MMA warp may overwrite it with pass 1
+                asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory");
+                __syncwarp();
+                if (lane == 0) mbar_arrive(tempty);
+            }
+        }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory");
+    __syncthreads();
+    if (warp == 2)
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;\n" ::"r"(tbase) : "memory");
+}
+
 // expo_words: the exponent words of this launch's problems (reset before the max).
 template <int S>
 inline cudaError_t oz_set_attr() {
-    return cudaFuncSetAttribute(k_oz_gemm<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)OzCfg<S>::SMEM);
+    cudaError_t e = cudaFuncSetAttribute(k_oz_gemm<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)OzCfg<S>::SMEM);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(k_oz_gemm2<S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kOz2Smem);
+    return e;
 }
 
 template <int S>
 inline void launch_oz(double *L, double *U, const GemmProb *probs, const OzProb *oprobs, const int32_t *split_tasks,
                       int64_t nsplit, const OzTile *tiles, int64_t ntiles, int8_t *slices, int32_t *expo,
-                      int64_t expo_words, cudaStream_t st, const UpdGather gv = UpdGather{}) {
+                      int64_t expo_words, cudaStream_t st, const UpdGather gv = UpdGather{}, int wide = 0) {
     if (nsplit > 0) {
         cudaMemsetAsync(expo, 0x80, (size_t)expo_words * sizeof(int32_t), st);   // 0x80808080 < any exponent
         k_oz_rowexp<S><<<(unsigned)nsplit, kOzBM, 0, st>>>(L, probs, oprobs, split_tasks, expo);
@@ -341,8 +547,11 @@ inline void launch_oz(double *L, double *U, const GemmProb *probs, const OzProb 
             oz_set_attr<S>();
             attr = true;
         }
-        k_oz_gemm<S><<<(unsigned)ntiles, kOzThreads, OzCfg<S>::SMEM, st>>>(L, U, probs, oprobs, tiles, slices, expo,
-                                                                             gv);
+        if (wide)   // 128 x 128 tiles, two passes
+            k_oz_gemm2<S><<<(unsigned)ntiles, kOz2Threads, kOz2Smem, st>>>(L, U, probs, oprobs, tiles, slices, expo, gv);
+        else
+            k_oz_gemm<S><<<(unsigned)ntiles, kOzThreads, OzCfg<S>::SMEM, st>>>(L, U, probs, oprobs, tiles, slices,
+                                                                                 expo, gv);
     }
 }
 

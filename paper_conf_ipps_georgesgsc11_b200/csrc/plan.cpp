@@ -430,7 +430,9 @@ static int plan_ozaki(Plan &P, int S) {
     auto up = [](int64_t x, int64_t a) { return (x + a - 1) / a * a; };
     std::map<int32_t, std::pair<int64_t, int64_t>> region;   // stream -> (slice bytes, exponent words)
     std::vector<std::pair<std::vector<Launch> *, size_t>> conv;
-    double min_k = kOzMinK;   // MF_OZ_MIN_K: tests drive small problems through the int8 path
+    // reduced slices need fewer pair MMAs per tile: they beat DMMA from K ~ 1024 (c5, S = 3 / 4:
+    // 153.6 / 160.9 ms at 1024 vs 167.7 / 172.7 ms at 2048 and 158.7 / 167.8 at 512)
+    double min_k = S >= 7 ? kOzMinK : 1024;   // MF_OZ_MIN_K: tests drive small problems through the int8 path
     if (const char *e = getenv("MF_OZ_MIN_K")) min_k = atof(e);
     for (std::vector<Launch> *prog : {&P.program, &P.program_top}) {
         for (size_t li = 0; li < prog->size(); li++) {
@@ -466,17 +468,34 @@ static int plan_ozaki(Plan &P, int S) {
                         P.oz_split.insert(P.oz_split.end(), {(int32_t)(L.oz_p + q), rb, sg});
             }
             L.oz_ns = (int64_t)P.oz_split.size() / 3 - L.oz_s;
+            // 128 x 128 tiles (two-pass kernel) when every problem of the launch is
+            // computed whole; a launch with a partial tile set (multi-GPU column
+            // ownership) keeps the DMMA tile columns with 128 x 64 tiles
+            std::map<int32_t, int64_t> have;
+            for (int64_t t = L.off; t < L.off + L.count; t++) have[P.tiles[t].prob]++;
+            bool whole = true;
+            for (int32_t p : probs) whole = whole && have[p] == count_tiles(P.probs[p].M, P.probs[p].N);
+            // (measured, tools/ubench/ozaki_gemm.cu: with S <= 4 the single-pass wide kernel is
+            // 1.4x the 128 x 64 one; with S = 8 both move the same slice bytes per output
+            // from L2 and run alike, so the narrow kernel stays)
+            // (and only without the fused extend-add gather: its epilogue gathers the
+            // children through global read-modify-writes, which ate the gain on c5)
+            bool gath = false;
+            for (int32_t p : probs) gath = gath || (P.probs[p].flags & kProbGather);
+            L.oz_wide = (whole && S <= 4 && !gath) ? 1 : 0;
+            const int32_t bn = whole ? 128 : kOzBN;
             L.oz_t = (int64_t)P.oz_tiles.size();
             std::set<std::pair<int32_t, int32_t>> seen;
             for (int64_t t = L.off; t < L.off + L.count; t++) {
                 const TileTask &tt = P.tiles[t];
-                const int32_t q = local[tt.prob], tij = (((tt.tij >> 16) * kTileM / kOzBM) << 16) | (tt.tij & 0xffff);
                 static_assert(kTileN == kOzBN, "Ozaki tiles keep the DMMA tile columns");
+                const int32_t q = local[tt.prob];
+                const int32_t tij = (((tt.tij >> 16) * kTileM / kOzBM) << 16) | ((tt.tij & 0xffff) * kTileN / bn);
                 if (seen.emplace(q, tij).second) P.oz_tiles.push_back(OzTile{(int32_t)(L.oz_p + q), tij});
             }
             L.oz_nt = (int64_t)P.oz_tiles.size() - L.oz_t;
             for (int64_t t = L.oz_t; t < L.oz_t + L.oz_nt; t++)
-                L.int8_ops += 2.0 * kOzBM * kOzBN * (double)P.oz_probs[P.oz_tiles[t].oprob].Kpad * (S * (S + 1) / 2);
+                L.int8_ops += 2.0 * kOzBM * bn * (double)P.oz_probs[P.oz_tiles[t].oprob].Kpad * (S * (S + 1) / 2);
             L.oz_ne = words;
             auto &rg = region[L.stream];
             rg.first = std::max(rg.first, bytes);

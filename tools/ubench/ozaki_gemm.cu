@@ -26,15 +26,17 @@ using Big = UpdCfg<64, 64, 16, 3, 2, 2, 4>;
     } while (0)
 
 template <int S>
-float run_oz(double *dL, double *dU, GemmProb *dprob, int M, int N, int K, int reps, const double *C0, size_t cbytes) {
+float run_oz(double *dL, double *dU, GemmProb *dprob, int M, int N, int K, int reps, const double *C0, size_t cbytes,
+             int wide = 0) {
+    const int BN = wide ? 128 : kOzBN;
     OzProb op{0, (M + kOzBM - 1) / kOzBM * kOzBM, (K + kOzBK - 1) / kOzBK * kOzBK, 0, 0, 0};
     std::vector<int32_t> tasks;
     for (int rb = 0; rb < op.Mpad / kOzBM; rb++)
         for (int sg = 0; sg < (op.Kpad + kOzSeg - 1) / kOzSeg; sg++) tasks.insert(tasks.end(), {0, rb, sg});
     std::vector<OzTile> tiles;
-    for (int tj = 0; tj < (N + kOzBN - 1) / kOzBN; tj++)
+    for (int tj = 0; tj < (N + BN - 1) / BN; tj++)
         for (int ti = 0; ti < op.Mpad / kOzBM; ti++)
-            if ((ti + 1) * kOzBM > tj * kOzBN) tiles.push_back({0, (ti << 16) | tj});
+            if ((ti + 1) * kOzBM > tj * BN) tiles.push_back({0, (ti << 16) | tj});
     OzProb *dop;
     int32_t *dt, *dex;
     OzTile *dtl;
@@ -57,7 +59,7 @@ float run_oz(double *dL, double *dU, GemmProb *dprob, int M, int N, int K, int r
         cudaEventRecord(e0);
         launch_oz<S>(dL, dU, dprob, dop, dt, (int64_t)tasks.size() / 3, nullptr, 0, dsl, dex, op.Mpad, 0);
         cudaEventRecord(e1);
-        launch_oz<S>(dL, dU, dprob, dop, nullptr, 0, dtl, (int64_t)tiles.size(), dsl, dex, 0, 0);
+        launch_oz<S>(dL, dU, dprob, dop, nullptr, 0, dtl, (int64_t)tiles.size(), dsl, dex, 0, 0, UpdGather{}, wide);
         cudaEventRecord(e2);
         CK(cudaEventSynchronize(e2));
         CK(cudaGetLastError());
@@ -66,7 +68,8 @@ float run_oz(double *dL, double *dU, GemmProb *dprob, int M, int N, int K, int r
         cudaEventElapsedTime(&t2, e0, e2);
         if (t2 < best) best = t2, bsplit = t1;
     }
-    printf("  ozaki S=%d: %zu tiles, split %.3f ms, total %.3f ms\n", S, tiles.size(), bsplit, best);
+    printf("  ozaki S=%d %s: %zu tiles, split %.3f ms, total %.3f ms\n", S, wide ? "128x128" : "128x64", tiles.size(),
+           bsplit, best);
     cudaFree(dop); cudaFree(dt); cudaFree(dtl); cudaFree(dsl); cudaFree(dex);
     return best;
 }
@@ -160,6 +163,12 @@ int main(int argc, char **argv) {
     float t8 = run_oz<8>(dL, dU, dprob, M, N, K, 4, dC0, cbytes);
     printf("  -> %.2f TF/s fp64-equivalent, %.2fx dmma\n", flops / t8 / 1e9, bd / t8);
     check("ozaki8");
+    float t8w = run_oz<8>(dL, dU, dprob, M, N, K, 4, dC0, cbytes, 1);
+    printf("  -> %.2f TF/s fp64-equivalent, %.2fx dmma\n", flops / t8w / 1e9, bd / t8w);
+    check("ozaki8w");
+    float t4w = run_oz<4>(dL, dU, dprob, M, N, K, 4, dC0, cbytes, 1);
+    printf("  -> %.2f TF/s fp64-equivalent, %.2fx dmma\n", flops / t4w / 1e9, bd / t4w);
+    check("ozaki4w");
     float t7 = run_oz<7>(dL, dU, dprob, M, N, K, 4, dC0, cbytes);
     printf("  -> %.2f TF/s fp64-equivalent, %.2fx dmma\n", flops / t7 / 1e9, bd / t7);
     check("ozaki7");
