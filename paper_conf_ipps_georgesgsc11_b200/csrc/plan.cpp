@@ -483,7 +483,7 @@ static int plan_ozaki(Plan &P, int S) {
             bool gath = false;
             for (int32_t p : probs) gath = gath || (P.probs[p].flags & kProbGather);
             L.oz_wide = (whole && S <= 4 && !gath) ? 1 : 0;
-            const int32_t bn = whole ? 128 : kOzBN;
+            const int32_t bn = L.oz_wide ? 128 : kOzBN;
             L.oz_t = (int64_t)P.oz_tiles.size();
             std::set<std::pair<int32_t, int32_t>> seen;
             for (int64_t t = L.off; t < L.off + L.count; t++) {
