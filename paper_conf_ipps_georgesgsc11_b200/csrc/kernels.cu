@@ -302,13 +302,19 @@ __device__ __forceinline__ int lower_bound_rel(const int32_t *__restrict__ rel, 
 }
 
 constexpr int kAsmMaxCh = 32;   // children handled through the shared column map (more: searched per column)
+static_assert(kAsmRowBlock % kAsmChunk == 0, "row blocks are whole chunks");
 __global__ void __launch_bounds__(kAsmThreads) k_assemble(DevPlan d, const int32_t *__restrict__ tasks,
                                                           const double *__restrict__ values) {
     constexpr int NW = kAsmThreads / 32;
     __shared__ double sbuf[NW][kAsmChunk];
     __shared__ int colmap[kAsmMaxCh][kAsmCols];   // child column landing in column c0 + x, or -1
     __shared__ int s_cp[NW][kAsmMaxCh];           // per warp and child: next child row to add
-    const int s = tasks[2 * blockIdx.x], c0 = tasks[2 * blockIdx.x + 1];
+    // task = (front, c0 | row block << 20): columns [c0, c0 + kAsmCols), rows of row block
+    // rb = [rb kAsmRowBlock, (rb + 1) kAsmRowBlock) -- tall fronts are split by rows so that
+    // their assembly spreads over the SMs (every element is still built by one warp:
+    // 0 + A + U^c1 + U^c2 ..., reading C6)
+    const int s = tasks[2 * blockIdx.x], c0 = tasks[2 * blockIdx.x + 1] & 0xfffff;
+    const int rb = tasks[2 * blockIdx.x + 1] >> 20;
     const int k = d.sn_k[s], f = d.sn_f[s], m = f - k, ld = d.sn_ld[s], first = d.sn_first[s];
     const int c1 = min(c0 + kAsmCols, d.fuse_ea ? k : f);   // fused extend-add: U^s is gathered by the syrk
     double *__restrict__ P = d.L + d.L_off[s];
@@ -341,11 +347,20 @@ __global__ void __launch_bounds__(kAsmThreads) k_assemble(DevPlan d, const int32
             col = Us + (int64_t)(c - k) * m - k;   // index by front row r >= c
             rlo = c;
         }
-        if (lane < nmap) cp[lane] = colmap[lane][c - c0];   // rel[qc] = c >= rlo: start at the diagonal
+        const int rbeg = max(rlo, rb * kAsmRowBlock), rend = min(f, (rb + 1) * kAsmRowBlock);
+        if (rbeg >= rend) continue;   // (uniform over the warp)
+        if (lane < nmap) {            // rel[qc] = c: the child's rows start at the diagonal
+            int qc = colmap[lane][c - c0];
+            if (qc >= 0 && rbeg > c) {   // ... or, in a lower row block, at its first row >= rbeg
+                const int ch = d.child_list[q0 + lane];
+                qc = lower_bound_rel(d.relmap + d.relmap_ptr[ch], qc, d.sn_f[ch] - d.sn_k[ch], rbeg);
+            }
+            cp[lane] = qc;
+        }
         __syncwarp();
         const int64_t e0 = c < k ? d.bcolptr[first + c] : 0, e1 = c < k ? d.bcolptr[first + c + 1] : 0;
-        for (int r0 = rlo; r0 < f; r0 += kAsmChunk) {
-            const int r1 = min(r0 + kAsmChunk, f);
+        for (int r0 = rbeg; r0 < rend; r0 += kAsmChunk) {
+            const int r1 = min(r0 + kAsmChunk, rend);
             for (int r = r0 + lane; r < r1; r += 32) buf[r - r0] = 0.0;
             __syncwarp();
             for (int64_t e = e0 + lane; e < e1; e += 32) {

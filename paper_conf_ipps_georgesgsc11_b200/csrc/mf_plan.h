@@ -265,6 +265,7 @@ struct Plan {
 
 constexpr int kTileM = 64, kTileN = 64;
 constexpr int kAsmCols = 16;
+constexpr int kAsmRowBlock = 2048;   // assembly tasks split tall fronts into row blocks of this many rows
 constexpr int kTrsmRows = 128;
 constexpr int kSmallClasses = 5;
 constexpr int kSolveRows = 256;   // dataflow solve: rows per chunk (a multiple of the 64-column block)

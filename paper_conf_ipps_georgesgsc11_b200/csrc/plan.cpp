@@ -961,9 +961,15 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
             for (int32_t s : large) {
                 // fused extend-add: only the panel columns (the syrk gathers U^s)
                 const int32_t cend = P.fuse_ea ? P.sn_k[s] : P.sn_f[s];
+                const int32_t nrb = (P.sn_f[s] + kAsmRowBlock - 1) / kAsmRowBlock;
+                if (nrb >= (1 << 11) || cend >= (1 << 20)) return MF_ERR_ARG;   // task encoding
                 for (int32_t c0 = 0; c0 < cend; c0 += kAsmCols) {
-                    P.asm_tasks.push_back(s);
-                    P.asm_tasks.push_back(c0);
+                    // panel columns span every row; U columns start at their diagonal
+                    const int32_t rb0 = c0 < P.sn_k[s] ? 0 : c0 / kAsmRowBlock;
+                    for (int32_t rb = rb0; rb < nrb; rb++) {
+                        P.asm_tasks.push_back(s);
+                        P.asm_tasks.push_back(c0 | (rb << 20));
+                    }
                 }
                 const double f = P.sn_f[s], k = P.sn_k[s], m = f - k;
                 if (P.fuse_ea)
