@@ -219,9 +219,11 @@ int mf_solve(mf_ctx *ctx, const double *b, double *x);
 
 /* nrhs right-hand sides: B and X are column-major n x nrhs with leading
  * dimensions ldb, ldx >= n (host or device, not aliased); X(:, r) = A^{-1} B(:, r),
- * bitwise the same as nrhs calls of mf_solve.  The right-hand sides are queued
- * back to back on the ctx stream (one CUDA-graph replay each, one final
- * synchronization).  MF_ERR_ARG for nrhs < 0 or ld < n. */
+ * bitwise the same as nrhs calls of mf_solve.  Single GPU: up to 8 solve
+ * pipelines (own vectors, flags, streams and CUDA graphs, allocated on first use)
+ * run right-hand sides concurrently, overlapping the latency-bound block chains of
+ * the large supernodes; one final synchronization.  With several ranks or with
+ * refinement: one mf_solve per column.  MF_ERR_ARG for nrhs < 0 or ld < n. */
 int mf_solve_nrhs(mf_ctx *ctx, int32_t nrhs, const double *B, int64_t ldb, double *X, int64_t ldx);
 
 int mf_get_info(const mf_ctx *ctx, mf_info *out);

@@ -24,8 +24,24 @@
 
 using namespace mf;
 
+// One extra solve pipeline (mf_solve_nrhs, single GPU): its own vectors, dataflow
+// flags / partial sums, solve epoch and ticket counters, a stream and a captured graph,
+// so several right-hand sides run concurrently -- the block chains of the large
+// supernodes are latency-bound, so overlapping them raises the throughput.
+struct SolveSlot {
+    mf::DevPlan d{};
+    double *y = nullptr, *bx = nullptr;
+    unsigned *tickets = nullptr;
+    cudaStream_t st = nullptr;
+    cudaEvent_t done = nullptr;
+    cudaGraph_t graph = nullptr;
+    cudaGraphExec_t exec = nullptr;
+};
+constexpr int kSolveSlots = 8;   // measured nrhs = 8: c5 2 / 4 / 8 slots 69.9 / 62.8 / 61.6 ms, c3 16.2 / 12.4 / 10.7 ms
+
 struct mf_ctx {
     Options opt;
+    std::vector<SolveSlot> slots;
     int device = 0;
     cudaStream_t stream = nullptr;
     bool own_stream = false;
@@ -137,10 +153,21 @@ void drop_graph(mf_ctx *c) {
     if (c->solve_graph) cudaGraphDestroy(c->solve_graph);
     c->solve_exec = nullptr;
     c->solve_graph = nullptr;
+    for (SolveSlot &q : c->slots) {
+        if (q.exec) cudaGraphExecDestroy(q.exec);
+        if (q.graph) cudaGraphDestroy(q.graph);
+        q.exec = nullptr;
+        q.graph = nullptr;
+    }
 }
 
 void free_device(mf_ctx *c) {
     drop_graph(c);
+    for (SolveSlot &q : c->slots) {   // buffers are in c->allocs
+        if (q.st) cudaStreamDestroy(q.st);
+        if (q.done) cudaEventDestroy(q.done);
+    }
+    c->slots.clear();
     for (void *p : c->allocs) {
         if (c->hfree) c->hfree(p, c->huser);
         else cudaFree(p);
@@ -841,29 +868,29 @@ int mf_factor(mf_ctx *c, const double *values) {
 }
 
 namespace {
-void run_solve_program(mf_ctx *c, const std::vector<SolveLaunch> &prog) {
+// One solve program on (d, y, tickets, st): the ctx's own pipeline or a SolveSlot's.
+void run_solve_program(mf_ctx *c, const std::vector<SolveLaunch> &prog, const DevPlan &d, double *y,
+                       unsigned *tickets, cudaStream_t st) {
     const Plan &P = c->P;
-    const DevPlan &d = c->d;
-    cudaStream_t st = c->stream;
     size_t base = P.program.size() + P.program_top.size();   // ticket slots of this solve program
     for (const std::vector<SolveLaunch> *q : {&P.fsolve, &P.bsolve, &P.fsolve_top, &P.bsolve_top}) {
         if (q == &prog) break;
         base += q->size();
     }
-    unsigned *tk0 = c->d_tickets + 2 * base;
+    unsigned *tk0 = tickets + 2 * base;
     for (size_t li = 0; li < prog.size(); li++) {
         const SolveLaunch &L = prog[li];
         switch (L.kind) {
-            case SK_SMALL_F: launch_fwd_solve(d, c->d_solve_list + L.off, (int)L.count, c->d_y, st); break;
-            case SK_INIT_F: launch_fsolve_init(d, c->d_solve_list + L.off, (int)L.count, c->d_y, st); break;
-            case SK_DF_F: launch_fsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, c->d_y, tk0 + 2 * li, st); break;
+            case SK_SMALL_F: launch_fwd_solve(d, c->d_solve_list + L.off, (int)L.count, y, st); break;
+            case SK_INIT_F: launch_fsolve_init(d, c->d_solve_list + L.off, (int)L.count, y, st); break;
+            case SK_DF_F: launch_fsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, y, tk0 + 2 * li, st); break;
             case SK_SMALL_B:
-                launch_bwd_solve(d, c->d_solve_list + L.off, (int)L.count, c->d_y, c->d_sn_rows, c->d_sn_rowptr, st);
+                launch_bwd_solve(d, c->d_solve_list + L.off, (int)L.count, y, c->d_sn_rows, c->d_sn_rowptr, st);
                 break;
             case SK_INIT_B:
-                launch_bsolve_init(d, c->d_solve_list + L.off, (int)L.count, c->d_y, c->d_sn_rows, c->d_sn_rowptr, st);
+                launch_bsolve_init(d, c->d_solve_list + L.off, (int)L.count, y, c->d_sn_rows, c->d_sn_rowptr, st);
                 break;
-            case SK_DF_B: launch_bsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, c->d_y, tk0 + 2 * li, st); break;
+            case SK_DF_B: launch_bsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, y, tk0 + 2 * li, st); break;
         }
     }
 }
@@ -895,8 +922,8 @@ int mf_solve(mf_ctx *c, const double *b, double *x) {
         if (!c->solve_exec) {
             CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
             launch_permute_in(d, c->d_bx, c->d_y, n, st);
-            run_solve_program(c, P.fsolve);
-            run_solve_program(c, P.bsolve);
+            run_solve_program(c, P.fsolve, d, c->d_y, c->d_tickets, st);
+            run_solve_program(c, P.bsolve, d, c->d_y, c->d_tickets, st);
             launch_permute_out(d, c->d_y, c->d_bx, n, st);
             cudaGraph_t g = nullptr;
             cudaError_t e2 = cudaStreamEndCapture(st, &g);
@@ -954,7 +981,7 @@ int mf_solve(mf_ctx *c, const double *b, double *x) {
     }
     launch_permute_in(d, bd, c->d_y, n, st);
     int r;
-    run_solve_program(c, P.fsolve);                  // forward, own subtrees
+    run_solve_program(c, P.fsolve, d, c->d_y, c->d_tickets, st);   // forward, own subtrees
     if (multi) {
         std::vector<mf_xfer> ops;                      // frontier roots' update vectors -> rank 0
         for (int32_t root : P.frontier_roots) {
@@ -965,15 +992,15 @@ int mf_solve(mf_ctx *c, const double *b, double *x) {
                                       c->d.fv + P.fv_off[root], (int64_t)P.sn_f[root] * (int64_t)sizeof(double)});
         }
         if ((r = exchange(c, ops))) return r;
-        run_solve_program(c, P.fsolve_top);          // rank 0: forward + backward on the top
-        run_solve_program(c, P.bsolve_top);
+        run_solve_program(c, P.fsolve_top, d, c->d_y, c->d_tickets, st);   // rank 0: forward + backward on the top
+        run_solve_program(c, P.bsolve_top, d, c->d_y, c->d_tickets, st);
         // rank 0's top solution -> every rank (y columns of the top supernodes)
         if (P.rank == 0) CK(cudaMemcpyAsync(c->d_ytmp, c->d_y, n * sizeof(double), cudaMemcpyDeviceToDevice, st));
         std::vector<mf_xfer> bc{mf_xfer{MF_XFER_BCAST, 0, c->d_ytmp, n * (int64_t)sizeof(double)}};
         if ((r = exchange(c, bc))) return r;
         if (P.rank != 0) launch_copy_cols(d, c->d_top_list, (int)P.top_list.size(), c->d_ytmp, c->d_y, st);
     }
-    run_solve_program(c, P.bsolve);                  // backward, own subtrees
+    run_solve_program(c, P.bsolve, d, c->d_y, c->d_tickets, st);   // backward, own subtrees
     if (multi) {   // every rank contributes its own columns; the sum is the full solution
         CK(cudaMemsetAsync(c->d_ytmp, 0, n * sizeof(double), st));
         launch_copy_cols(d, c->d_own_list, (int)P.own_list.size(), c->d_y, c->d_ytmp, st);
@@ -993,6 +1020,52 @@ int mf_solve(mf_ctx *c, const double *b, double *x) {
     return MF_OK;
 }
 
+namespace {
+// Extra solve pipelines for mf_solve_nrhs (allocated on first use; freed with the plan).
+int ensure_slots(mf_ctx *c, int ns) {
+    const Plan &P = c->P;
+    const int64_t n = c->S.n;
+    const size_t tk_words = 2 * (P.program.size() + P.program_top.size() + P.fsolve.size() + P.bsolve.size() +
+                                 P.fsolve_top.size() + P.bsolve_top.size() + 1);
+    while ((int)c->slots.size() < ns) {
+        SolveSlot q;
+        q.d = c->d;
+        void *p = nullptr;
+        int r;
+        if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(n, 1) * sizeof(double)))) return r;
+        q.y = (double *)p;
+        if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(n, 1) * sizeof(double)))) return r;
+        q.bx = (double *)p;
+        if ((r = dev_alloc(c, &p, (size_t)P.fv_words * sizeof(double)))) return r;
+        q.d.fv = (double *)p;
+        if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.df_nparts, 1) * sizeof(double)))) return r;
+        q.d.df_parts = (double *)p;
+        const size_t nfl = (size_t)std::max<int64_t>(P.df_nflags, 1) * sizeof(unsigned);
+        if ((r = dev_alloc(c, &p, nfl + 16))) return r;   // flags + the slot's solve epoch
+        CK(cudaMemsetAsync(p, 0, nfl + 16, c->stream));
+        q.d.df_flags = (unsigned *)p;
+        q.d.solve_epoch = (unsigned *)((char *)p + nfl);
+        if ((r = dev_alloc(c, &p, tk_words * sizeof(unsigned)))) return r;
+        CK(cudaMemsetAsync(p, 0, tk_words * sizeof(unsigned), c->stream));
+        q.tickets = (unsigned *)p;
+        CK(cudaStreamCreateWithFlags(&q.st, cudaStreamNonBlocking));
+        CK(cudaEventCreateWithFlags(&q.done, cudaEventDisableTiming));
+        // the same program as mf_solve's graph, on the slot's buffers and stream
+        CK(cudaStreamBeginCapture(q.st, cudaStreamCaptureModeThreadLocal));
+        launch_permute_in(q.d, q.bx, q.y, n, q.st);
+        run_solve_program(c, P.fsolve, q.d, q.y, q.tickets, q.st);
+        run_solve_program(c, P.bsolve, q.d, q.y, q.tickets, q.st);
+        launch_permute_out(q.d, q.y, q.bx, n, q.st);
+        cudaError_t e = cudaStreamEndCapture(q.st, &q.graph);
+        CK(e);
+        CK(cudaGraphInstantiate(&q.exec, q.graph, 0));
+        c->slots.push_back(q);
+    }
+    CK(cudaStreamSynchronize(c->stream));   // zeroed flags / tickets before first use
+    return MF_OK;
+}
+}  // namespace
+
 int mf_solve_nrhs(mf_ctx *c, int32_t nrhs, const double *B, int64_t ldb, double *X, int64_t ldx) {
     if (!c || nrhs < 0) return MF_ERR_ARG;
     if (c->state != 2 || c->host_only) return MF_ERR_STATE;
@@ -1000,8 +1073,8 @@ int mf_solve_nrhs(mf_ctx *c, int32_t nrhs, const double *B, int64_t ldb, double 
     if (nrhs == 0) return MF_OK;
     if (!B || !X || ldb < n || ldx < n) return MF_ERR_ARG;
     if ((const void *)B == (const void *)X) return MF_ERR_ARG;
-    if (c->P.nranks > 1 || !c->use_graph || c->opt.refine_iters > 0) {   // one column at a time through mf_solve
-        for (int32_t r = 0; r < nrhs; r++)
+    if (c->P.nranks > 1 || !c->use_graph || c->opt.refine_iters > 0 || nrhs == 1) {
+        for (int32_t r = 0; r < nrhs; r++)   // one column at a time through mf_solve
             if (int e = mf_solve(c, B + r * ldb, X + r * ldx)) return e;
         return MF_OK;
     }
@@ -1011,20 +1084,31 @@ int mf_solve_nrhs(mf_ctx *c, int32_t nrhs, const double *B, int64_t ldb, double 
     if (bdev || xdev) {
         if (int r = order_after_caller(c)) return r;
     }
-    if (!c->solve_exec || c->dinv_stale) {   // capture the solve graph / solve setup (same program as mf_solve)
-        if (int e = mf_solve(c, B, X)) return e;
-        if (nrhs == 1) return MF_OK;
-        B += ldb;
-        X += ldx;
-        nrhs -= 1;
+    if (c->dinv_stale) {   // solve setup (inverses of the diagonal blocks), once per factorization
+        launch_diag_inv(c->d, c->d_dinv_tasks, (int64_t)c->P.dinv_tasks.size() / 2, c->P.w, st);
+        c->dinv_stale = false;
     }
+    static const int max_slots = [] {   // MF_SOLVE_SLOTS: tuning override of kSolveSlots
+        const char *e = getenv("MF_SOLVE_SLOTS");
+        return e ? std::max(1, std::min(16, atoi(e))) : kSolveSlots;
+    }();
+    const int ns = std::min<int>(max_slots, nrhs);
+    if (int r = ensure_slots(c, ns)) return r;
     CK(cudaEventRecord(c->ev0, st));
+    for (int q = 0; q < ns; q++) CK(cudaStreamWaitEvent(c->slots[q].st, c->ev0, 0));
+    // right-hand side r on slot r mod ns: each slot's columns run in order on its stream,
+    // the slots concurrently (same kernels and order as mf_solve: bitwise the same x)
     for (int32_t r = 0; r < nrhs; r++) {
-        CK(cudaMemcpyAsync(c->d_bx, B + r * ldb, n * sizeof(double),
-                           bdev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, st));
-        CK(cudaGraphLaunch(c->solve_exec, st));
-        CK(cudaMemcpyAsync(X + r * ldx, c->d_bx, n * sizeof(double),
-                           xdev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, st));
+        SolveSlot &q = c->slots[r % ns];
+        CK(cudaMemcpyAsync(q.bx, B + r * ldb, n * sizeof(double),
+                           bdev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, q.st));
+        CK(cudaGraphLaunch(q.exec, q.st));
+        CK(cudaMemcpyAsync(X + r * ldx, q.bx, n * sizeof(double),
+                           xdev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, q.st));
+    }
+    for (int q = 0; q < ns; q++) {
+        CK(cudaEventRecord(c->slots[q].done, c->slots[q].st));
+        CK(cudaStreamWaitEvent(st, c->slots[q].done, 0));
     }
     CK(cudaGetLastError());
     CK(cudaEventRecord(c->ev1, st));
