@@ -18,6 +18,8 @@
 #include <map>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "kernels.cuh"
 #include "mf.h"
 #include "mf_plan.h"
@@ -103,6 +105,13 @@ struct mf_ctx {
 };
 
 namespace {
+
+// NVTX ranges around the host-side phases of every call (header-only NVTX v3: a
+// no-op unless a tool such as nsys / ncu injects itself), for timelines.
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
 
 int cuda_err(cudaError_t e) {
     if (e == cudaSuccess) return MF_OK;
@@ -383,6 +392,7 @@ void mf_destroy(mf_ctx *c) {
 
 int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowind, const int32_t *perm) {
     if (!c) return MF_ERR_ARG;
+    NvtxRange nvtx_("mf_analyze");
     auto t0 = std::chrono::steady_clock::now();
     if (!c->host_only) {
         CK(cudaSetDevice(c->device));
@@ -391,9 +401,16 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
         if (kernels_init()) return MF_ERR_CUDA;
     }
     c->state = 0;
-    int st = analyze_symbolic(n, colptr, rowind, perm, c->opt, c->S);
+    int st;
+    {
+        NvtxRange r("mf_analyze: symbolic");
+        st = analyze_symbolic(n, colptr, rowind, perm, c->opt, c->S);
+    }
     if (st) return st;
-    st = build_plan(c->S, c->opt, c->P);
+    {
+        NvtxRange r("mf_analyze: plan");
+        st = build_plan(c->S, c->opt, c->P);
+    }
     if (st) return st;
     if (c->host_only) {
         fill_info(c, n, 0);
@@ -735,6 +752,7 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
 // Hand a list of transfers to the caller's exchange callback (multi-GPU only);
 // the ctx stream is drained first, so the buffers are final.
 int exchange(mf_ctx *c, std::vector<mf_xfer> &ops) {
+    NvtxRange nvtx_("mf exchange");
     // every rank calls the callback at every exchange point, even with nothing to
     // move, so the caller's collectives stay aligned across ranks
     if (!c->xfn) return MF_ERR_STATE;
@@ -785,6 +803,7 @@ void accumulate_stats(mf_ctx *c, const std::vector<Launch> &prog, size_t ev_base
 
 int mf_factor(mf_ctx *c, const double *values) {
     if (!c || !values) return MF_ERR_ARG;
+    NvtxRange nvtx_("mf_factor");
     if (c->state < 1 || c->host_only) return MF_ERR_STATE;
     CK(cudaSetDevice(c->device));
     const Plan &P = c->P;
@@ -898,6 +917,7 @@ void run_solve_program(mf_ctx *c, const std::vector<SolveLaunch> &prog, const De
 
 int mf_solve(mf_ctx *c, const double *b, double *x) {
     if (!c || !b || !x || b == x) return MF_ERR_ARG;
+    NvtxRange nvtx_("mf_solve");
     if (c->state != 2 || c->host_only) return MF_ERR_STATE;
     CK(cudaSetDevice(c->device));
     const Plan &P = c->P;
@@ -1068,6 +1088,7 @@ int ensure_slots(mf_ctx *c, int ns) {
 
 int mf_solve_nrhs(mf_ctx *c, int32_t nrhs, const double *B, int64_t ldb, double *X, int64_t ldx) {
     if (!c || nrhs < 0) return MF_ERR_ARG;
+    NvtxRange nvtx_("mf_solve_nrhs");
     if (c->state != 2 || c->host_only) return MF_ERR_STATE;
     const int64_t n = c->S.n;
     if (nrhs == 0) return MF_OK;
