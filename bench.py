@@ -404,6 +404,28 @@ def main():
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
         t_e2e = float(t.item())
     t_solve = S.info()["t_solve"]
+    # ---- the solve on the device (NEXT-2): one right-hand side, and 8 through
+    # mf_solve_nrhs (concurrent solve pipelines), against reading the stored L twice
+    solve = None
+    if world == 1:
+        bd = torch.from_numpy(G.rhs(A.n, 0)).cuda()
+        xd = torch.empty_like(bd)
+        S.solve(bd, xd)
+        ts = []
+        for _ in range(3):
+            S.solve(bd, xd)
+            ts.append(S.info()["t_solve"] * 1e3)
+        B8 = torch.from_numpy(np.random.default_rng(1).uniform(-1, 1, (8, A.n))).cuda()
+        S.solve_nrhs(B8)
+        S.solve_nrhs(B8)
+        t8 = S.info()["t_solve"] * 1e3
+        hbm = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"] \
+            if os.path.exists(os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6650.0
+        bound = 2.0 * info["panel_words"] * 8 / (hbm * 1e9) * 1e3
+        solve = {"ms_1rhs": float(np.median(ts)), "ms_per_rhs_nrhs8": t8 / 8, "hbm_bound_ms": bound,
+                 "frac_1rhs": bound / float(np.median(ts)), "frac_nrhs8": bound / (t8 / 8),
+                 "what": "device b/x; bound = 2 x stored L bytes / measured HBM GB/s"}
+        del bd, xd, B8
 
     # ---- roofline of the dominant kernel (by event time inside the timed region)
     dom = max(stats, key=lambda s: s["ms"])
@@ -449,6 +471,7 @@ def main():
                 "seconds": t_e2e, "solve_seconds": t_solve,
                 "h2d_bytes_per_step": int(A.nnz * 8 + A.n * 8), "d2h_bytes_per_step": int(A.n * 8 + 4)},
         "gpu_launches": int(info["launches_factor"]) * args.steps,
+        "solve": solve,
         "roofline": roof,
         "kernels": [{k: (round(v, 4) if isinstance(v, float) else v) for k, v in s.items()} for s in stats],
         "profiled_ms_per_step": prof_ms,

@@ -846,8 +846,8 @@ int mf_factor(mf_ctx *c, const double *values) {
         for (int32_t root : P.frontier_roots) {
             const int32_t m = P.sn_f[root] - P.sn_k[root];
             if (m <= 0) continue;
-            ops.push_back(mf_xfer{MF_XFER_BCAST, P.owner[root], c->d.U + P.U_off[root],
-                                  (int64_t)m * m * (int64_t)sizeof(double)});
+            ops.push_back(mf_xfer{MF_XFER_BCAST, P.owner[root], c->d.U + P.U_off[root],   // packed lower U^c
+                                  (int64_t)m * (m + 1) / 2 * (int64_t)sizeof(double)});
         }
         if ((r = exchange(c, ops))) return r;
         // (2) every rank factors the top: replicated small fronts, cooperative large ones

@@ -108,7 +108,8 @@ struct UpdCfg {
     static_assert(BK % PSA16 == 0 && BK % PSB16 == 0, "staging map");
     static constexpr int STAGE_WORDS = BK * (SA + SB);
     static constexpr size_t SMEM =
-        (size_t)STAGES * STAGE_WORDS * sizeof(double) + 2 * STAGES * sizeof(uint64_t) + (BM + BN) * sizeof(int);
+        (size_t)STAGES * STAGE_WORDS * sizeof(double) + 2 * STAGES * sizeof(uint64_t) + (BM + BN) * sizeof(int) +
+        BN * sizeof(int64_t);
     static_assert(SA % 16 == 4 && SB % 16 == 4, "bank-conflict-free fragment loads");
     static_assert(TM % 8 == 0 && TN % 8 == 0 && BK % 4 == 0, "tile shape");
 };
@@ -204,6 +205,8 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
     // C(i - sh, j - sh) for the (shifted) tile coordinates (i, j)
     double *__restrict__ C = ((g.flags & 1) ? Uarena : Larena) + g.c_off;
     const int ldc = g.ldc;
+    const bool packed = (g.flags & 1) != 0;   // U^s: packed lower (mf_plan.h upk); L: column-major
+    auto cidx = [&](int i, int j) -> int64_t { return packed ? upk(i, j, ldc) : i + (int64_t)j * ldc; };
     double acc[MB][NB][2];
     if (!(g.flags & 4)) {
 #pragma unroll
@@ -215,7 +218,7 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
                 for (int e = 0; e < 2; e++) {
                     const int j = j0 + wn * TN + nb * 8 + 2 * tq + e;
                     acc[mb][nb][e] =
-                        (i < g.M && j < g.N && i >= sh && j >= sh) ? C[(i - sh) + (int64_t)(j - sh) * ldc] : 0.0;
+                        (i < g.M && j < g.N && i >= sh && j >= sh && i >= j) ? C[cidx(i - sh, j - sh)] : 0.0;
                 }
         }
     } else {
@@ -228,7 +231,8 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
         for (int mb = 0; mb < MB; mb++)
 #pragma unroll
             for (int nb = 0; nb < NB; nb++) acc[mb][nb][0] = acc[mb][nb][1] = 0.0;
-        int *rq = reinterpret_cast<int *>(empty + STAGES), *cq = rq + BM;
+        int64_t *cqb = reinterpret_cast<int64_t *>(empty + STAGES);   // packed column bases of cq
+        int *rq = reinterpret_cast<int *>(cqb + BN), *cq = rq + BM;
         const int q0 = gv.child_ptr[g.s], q1 = gv.child_ptr[g.s + 1], kp = gv.sn_k[g.s];
         const int ntr1 = (g.M + BM - 1) / BM + 1;
         for (int jc = 0; jc < q1 - q0; jc++) {
@@ -244,7 +248,11 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
             __syncthreads();
             // front row r >= kp sits at shifted U row r - kp + sh
             for (int q = ra + tid; q < rb; q += NT) rq[__ldg(rel + q) - kp + sh - i0] = q;
-            for (int q = ca + tid; q < cb; q += NT) cq[__ldg(rel + q) - kp + sh - j0] = q;
+            for (int q = ca + tid; q < cb; q += NT) {
+                const int x = __ldg(rel + q) - kp + sh - j0;
+                cq[x] = q;
+                cqb[x] = upk_col(q, mc) - q;   // child column q of the packed U^c, indexed by row
+            }
             __syncthreads();
 #pragma unroll
             for (int mb = 0; mb < MB; mb++) {
@@ -254,8 +262,8 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
                 for (int nb = 0; nb < NB; nb++)
 #pragma unroll
                     for (int e = 0; e < 2; e++) {
-                        const int qj = cq[wn * TN + nb * 8 + 2 * tq + e];
-                        if (qj >= 0 && qi >= qj) acc[mb][nb][e] += __ldg(Uc + qi + (int64_t)qj * mc);
+                        const int x = wn * TN + nb * 8 + 2 * tq + e, qj = cq[x];
+                        if (qj >= 0 && qi >= qj) acc[mb][nb][e] += __ldg(Uc + cqb[x] + qi);
                     }
             }
         }
@@ -311,7 +319,7 @@ __global__ void __launch_bounds__(Cfg::NT, Cfg::MINB)
 #pragma unroll
             for (int e = 0; e < 2; e++) {
                 const int j = j0 + wn * TN + nb * 8 + 2 * tq + e;
-                if (j < g.N && i >= j && j >= sh) C[(i - sh) + (int64_t)(j - sh) * ldc] = acc[mb][nb][e];
+                if (j < g.N && i >= j && j >= sh) C[cidx(i - sh, j - sh)] = acc[mb][nb][e];
             }
     }
 }

@@ -129,7 +129,7 @@ __global__ void __launch_bounds__(NT) k_small_front(DevPlan d, const int32_t *__
         const double *__restrict__ Uc = d.U + d.U_off[c];
         for (int qq = warp; qq < mc; qq += NW) {
             double *dst = F + rel[qq] * f;
-            const double *ucol = Uc + qq * mc;
+            const double *ucol = Uc + upk_col(qq, mc) - qq;   // packed column qq, indexed by row
             for (int p = qq + lane; p < mc; p += 32) dst[rel[p]] += ucol[p];
         }
         __syncthreads();
@@ -183,7 +183,7 @@ __global__ void __launch_bounds__(NT) k_small_front(DevPlan d, const int32_t *__
     if (m > 0) {
         double *__restrict__ Us = d.U + d.U_off[s];
         for (int c = warp; c < m; c += NW)
-            for (int i = c + lane; i < m; i += 32) Us[i + c * m] = F[(k + i) + (k + c) * f];
+            for (int i = c + lane; i < m; i += 32) Us[upk(i, c, m)] = F[(k + i) + (k + c) * f];
     }
 }
 
@@ -222,7 +222,7 @@ __global__ void __launch_bounds__(32 * kTinyWarps, TF <= 16 ? 8 : 4)
         const int myrel = lane < mc ? rel[lane] : 0;
         for (int qq = 0; qq < mc; qq++) {
             const int dc = __shfl_sync(0xffffffffu, myrel, qq);
-            if (lane >= qq && lane < mc) F[myrel + dc * kTinyLD] += Uc[lane + qq * mc];
+            if (lane >= qq && lane < mc) F[myrel + dc * kTinyLD] += Uc[upk(lane, qq, mc)];
         }
         __syncwarp();
     }
@@ -254,10 +254,10 @@ __global__ void __launch_bounds__(32 * kTinyWarps, TF <= 16 ? 8 : 4)
         for (int j = 0; j < TF; j++)
             if (j < k) P[lane + (int64_t)j * ld] = lane >= j ? a[j] : 0.0;
         if (m > 0) {
-            double *__restrict__ Us = d.U + d.U_off[s] - k - (int64_t)k * m;   // Us[(i-k) + (c-k) m]
+            double *__restrict__ Us = d.U + d.U_off[s];
 #pragma unroll
             for (int c = 0; c < TF; c++)
-                if (c >= k && c < f && lane >= c) Us[lane + (int64_t)c * m] = a[c];
+                if (c >= k && c < f && lane >= c) Us[upk(lane - k, c - k, m)] = a[c];
         }
     }
 }
@@ -344,7 +344,7 @@ __global__ void __launch_bounds__(kAsmThreads) k_assemble(DevPlan d, const int32
             col = P + (int64_t)c * ld;
             rlo = 0;
         } else {
-            col = Us + (int64_t)(c - k) * m - k;   // index by front row r >= c
+            col = Us + upk_col(c - k, m) - c;   // packed column c - k, indexed by front row r >= c
             rlo = c;
         }
         const int rbeg = max(rlo, rb * kAsmRowBlock), rend = min(f, (rb + 1) * kAsmRowBlock);
@@ -382,7 +382,7 @@ __global__ void __launch_bounds__(kAsmThreads) k_assemble(DevPlan d, const int32
                     if (qc >= mc || __ldg(rel + qc) != c) continue;
                     p = lower_bound_rel(rel, qc, mc, r0);
                 }
-                const double *__restrict__ ucol = d.U + d.U_off[ch] + (int64_t)qc * mc;
+                const double *__restrict__ ucol = d.U + d.U_off[ch] + upk_col(qc, mc) - qc;   // packed column qc
                 // consume child rows p, p+1, ... while rel < r1 (rel is increasing): 256 rows per
                 // step (8 loads of each kind in flight per lane), the stop found by warp ballots
                 while (p < mc) {

@@ -11,7 +11,20 @@
 #include <cstdint>
 #include <vector>
 
+#ifdef __CUDACC__
+#define MF_HD __host__ __device__ __forceinline__
+#else
+#define MF_HD inline
+#endif
+
 namespace mf {
+
+// Update matrices U^s (m x m, lower triangle) are stored PACKED, column-major lower:
+// column j (its diagonal first) starts at word j (2m - j + 1) / 2; element (i, j),
+// i >= j, is word upk_col(j, m) + i - j.  m (m + 1) / 2 words per front, half the
+// full square (workspace, and the bytes a multi-GPU exchange moves).
+MF_HD int64_t upk_col(int64_t j, int64_t m) { return j * (2 * m - j + 1) / 2; }
+MF_HD int64_t upk(int64_t i, int64_t j, int64_t m) { return upk_col(j, m) + (i - j); }
 
 struct Options {
     int amalgamate = 1;
@@ -91,8 +104,8 @@ int analyze_symbolic(int64_t n, const int64_t *colptr, const int32_t *rowind, co
 // A (lower-trapezoidal) Schur update problem:  C[i][j] -= sum_p A[i][p] * A[j][p]
 // for 0 <= j < N, j <= i < M (only entries with i >= j are written).
 // A: M x K, column-major, leading dim lda, inside the L arena.
-// C: column-major, leading dim ldc, inside the L arena (flags bit 0 = 0) or the U
-// arena (1).  flags bit 1: the problem is shifted one row / column up-left so that
+// C: column-major, leading dim ldc, inside the L arena (flags bit 0 = 0), or packed
+// lower of order ldc (upk) inside the U arena (1).  flags bit 1: the problem is shifted one row / column up-left so that
 // its first A row is even (16-byte staging); row / column 0 of the shifted space
 // are padding: C(i, j) of the kernel is C_orig(i - 1, j - 1).
 // flags bit 2 (the syrk on U^s with the extend-add fused into its prologue,

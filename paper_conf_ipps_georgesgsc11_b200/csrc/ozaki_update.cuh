@@ -296,18 +296,20 @@ __global__ void __launch_bounds__(kOzThreads, 1)
             if (qi >= 0)
                 for (int c = 0; c < kOzBN; c++) {
                     const int qj = cq[c];
-                    if (qj >= 0 && qi >= qj) Gs[c * kOzBM + il] += __ldg(Uc + qi + (int64_t)qj * mc);
+                    if (qj >= 0 && qi >= qj) Gs[c * kOzBM + il] += __ldg(Uc + upk(qi, qj, mc));
                 }
         }
     }
     __syncwarp();
     double *__restrict__ C = ((g.flags & 1) ? Uarena : Larena) + g.c_off;
     const int64_t ldc = g.ldc;
+    const bool packed = (g.flags & 1) != 0;   // U^s: packed lower (mf_plan.h upk); L: column-major
+    auto cidx = [&](int64_t i, int64_t j) -> int64_t { return packed ? upk(i, j, ldc) : i + j * ldc; };
     if (i < g.M && i >= sh) {
         for (int c = 0; c < kOzBN; c++) {
             const int j = j0 + c;
             if (j < g.N && i >= j && j >= sh) {
-                double *cp = C + (i - sh) + (int64_t)(j - sh) * ldc;
+                double *cp = C + cidx(i - sh, j - sh);
                 *cp = (gather ? Gs[c * kOzBM + il] : *cp) - Ps[c * kOzBM + il];
             }
         }
@@ -445,6 +447,8 @@ __global__ void __launch_bounds__(kOz2Threads, 1)
         const int sh = (g.flags >> 1) & 1;
         double *__restrict__ C = ((g.flags & 1) ? Uarena : Larena) + g.c_off;
         const int64_t ldc = g.ldc;
+        const bool packed = (g.flags & 1) != 0;   // U^s: packed lower (mf_plan.h upk); L: column-major
+        auto cidx = [&](int64_t i, int64_t j) -> int64_t { return packed ? upk(i, j, ldc) : i + j * ldc; };
         const int Ei = expo[o.ex_off + i];
         const bool row_ok = i < g.M && i >= sh;
         const bool gather = (g.flags & 4) != 0;
@@ -452,7 +456,7 @@ __global__ void __launch_bounds__(kOz2Threads, 1)
             if (row_ok)
                 for (int c = 0; c < kOz2BN; c++) {
                     const int j = j0 + c;
-                    if (j < g.N && i >= j && j >= sh) C[(i - sh) + (int64_t)(j - sh) * ldc] = 0.0;
+                    if (j < g.N && i >= j && j >= sh) C[cidx(i - sh, j - sh)] = 0.0;
                 }
             const int q0 = gv.child_ptr[g.s], q1 = gv.child_ptr[g.s + 1], kp = gv.sn_k[g.s];
             const int ntr1 = (g.M + kTileM - 1) / kTileM + 1;   // ea_qs tables are per 64-row tile
@@ -477,7 +481,7 @@ __global__ void __launch_bounds__(kOz2Threads, 1)
                     for (int c = 0; c < kOz2BN; c++) {
                         const int qj = cq[c], j = j0 + c;
                         if (qj >= 0 && qi >= qj && j < g.N && i >= j && j >= sh)
-                            C[(i - sh) + (int64_t)(j - sh) * ldc] += __ldg(Uc + qi + (int64_t)qj * mc);
+                            C[cidx(i - sh, j - sh)] += __ldg(Uc + upk(qi, qj, mc));
                     }
             }
         }
@@ -504,7 +508,7 @@ __global__ void __launch_bounds__(kOz2Threads, 1)
                     for (int q = 0; q < 32; q++) {
                         const int j = j0 + c0 + q;
                         if (j < g.N && i >= j && j >= sh) {
-                            double *cp = C + (i - sh) + (int64_t)(j - sh) * ldc;
+                            double *cp = C + cidx(i - sh, j - sh);
                             *cp -= ldexp(v[q], Ei + ej[c0 + q]);
                         }
                     }

@@ -212,7 +212,7 @@ static void map_subtrees(Plan &P, const std::vector<double> &front_load) {
         double bc = 0;   // broadcast of the frontier roots' update matrices
         for (int32_t r : fr) {
             const double m = P.sn_f[r] - P.sn_k[r];
-            bc += kXchgLatency / 8 + kXchgPerByte * 8.0 * m * m;
+            bc += kXchgLatency / 8 + kXchgPerByte * 8.0 * m * (m + 1) / 2;   // packed lower U^c
         }
         const double make = lpt(fr, assign, load) + topl + bc;
         // split_all: the first frontier with >= R subtrees wins, whatever the model says
@@ -307,8 +307,8 @@ static void assign_branches(Plan &P, const std::vector<double> &front_load, int 
 // whole arena minus the frontier roots' still-live slots.  Only offsets change.
 static void plan_u_reuse(Plan &P) {
     const int32_t ns = P.nsuper;
-    auto words = [&](int32_t s) -> int64_t {
-        const int64_t m = P.sn_f[s] - P.sn_k[s], w = m * m;
+    auto words = [&](int32_t s) -> int64_t {   // packed lower U^s (mf_plan.h upk)
+        const int64_t m = P.sn_f[s] - P.sn_k[s], w = m * (m + 1) / 2;
         return w + (w & 1);
     };
     std::vector<int64_t> off(ns, -1);
@@ -548,7 +548,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
         P.L_off[s] = loff;
         loff += (int64_t)P.sn_ld[s] * k;
         P.U_off[s] = uoff;
-        int64_t uw = (int64_t)m * m;
+        int64_t uw = (int64_t)m * (m + 1) / 2;   // packed lower (mf_plan.h upk)
         uoff += uw + (uw & 1);
         P.fv_off[s] = fvoff;
         fvoff += f + (f & 1);
@@ -1096,8 +1096,8 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
             for (int r = 0; r < R; r++) {   // original columns of rank r's shifted tile columns
                 const int32_t c0 = std::max(0, tb[r] * kTileN - sh), c1 = std::min(m, tb[r + 1] * kTileN - sh);
                 if (c1 <= c0) continue;
-                ux.push_back(XferSpec{MF_XFER_BCAST, r, 1, P.U_off[s] + (int64_t)c0 * m + c0,
-                                      (int64_t)(c1 - c0 - 1) * m + (m - c0)});
+                ux.push_back(XferSpec{MF_XFER_BCAST, r, 1, P.U_off[s] + upk_col(c0, m),   // packed columns [c0, c1)
+                                      upk_col(c1, m) - upk_col(c0, m)});
             }
         }
         Ls.count = (int64_t)P.tiles.size() - Ls.off;

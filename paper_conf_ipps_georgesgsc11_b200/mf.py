@@ -168,7 +168,7 @@ class Solver:
                  nranks: int = 1, rank: int = 0, exchange=None, split_all: bool = False,
                  nbranch: int | None = None, fuse_ea: bool | None = None, lookahead: bool | None = None,
                  variant_model="auto", torch_alloc: bool = False, ozaki_slices: int = 0,
-                 refine_iters: int | None = None):
+                 refine_iters: int | None = None, nrelax=None, zrelax=None):
         """variant_model: "auto" = the fitted kernel-variant selector packaged with the
         binding (selector.MODEL_PATH, Eqs. 3-5 fitted to B200 timings) when
         present, None = libmf's fixed front-order thresholds, or a theta array.
@@ -185,6 +185,12 @@ class Solver:
         o = Options()
         lib.mf_default_options(ctypes.byref(o))
         o.amalgamate = int(amalgamate)
+        if nrelax is not None:   # relaxed-amalgamation thresholds (default {4,16,48})
+            for i, v in enumerate(nrelax):
+                o.nrelax[i] = int(v)
+        if zrelax is not None:   # default {0.8, 0.1, 0.05}
+            for i, v in enumerate(zrelax):
+                o.zrelax[i] = float(v)
         if small_front_max is not None:
             o.small_front_max = small_front_max
         if panel_w is not None:
