@@ -455,8 +455,7 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     UP(&c->d_tiles, P.tiles);
     UP(&c->d_solve_list, P.solve_list);
     UP(&c->d_df_tasks, P.df_tasks);
-    int64_t *df_blk_off = nullptr, *df_part_off = nullptr, *dinv_off = nullptr;
-    UP(&df_blk_off, P.df_blk_off);
+    int64_t *df_part_off = nullptr, *dinv_off = nullptr;
     UP(&df_part_off, P.df_part_off);
     UP(&dinv_off, P.dinv_off);
     UP(&c->d_dinv_tasks, P.dinv_tasks);
@@ -526,7 +525,6 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     d.bvptr = bvptr;
     d.bvidx = bvidx;
     d.perm = perm_d;
-    d.df_blk_off = df_blk_off;
     d.df_part_off = df_part_off;
     d.dinv_off = dinv_off;
     d.ea_qs = ea_qs;
@@ -554,12 +552,8 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.dinv_words, 1) * sizeof(double))) != MF_OK) return r;
     d.dinv = (double *)p;
     c->dinv_stale = true;
-    if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.df_nflags, 1) * sizeof(unsigned))) != MF_OK) return r;
-    d.df_flags = (unsigned *)p;
-    CK(cudaMemsetAsync(d.df_flags, 0, (size_t)std::max<int64_t>(P.df_nflags, 1) * sizeof(unsigned), c->stream));
     d.failed = c->d_failed;
     d.epoch = reinterpret_cast<const unsigned *>(c->d_failed + 1);
-    d.solve_epoch = reinterpret_cast<unsigned *>(c->d_failed + 2);
     if ((r = dev_alloc(c, &p, std::max<int32_t>(P.nsuper, 1) * sizeof(unsigned))) != MF_OK) return r;
     d.leaf_flag = (unsigned *)p;
     CK(cudaMemsetAsync(d.leaf_flag, 0, std::max<int32_t>(P.nsuper, 1) * sizeof(unsigned), c->stream));
@@ -901,15 +895,15 @@ void run_solve_program(mf_ctx *c, const std::vector<SolveLaunch> &prog, const De
         const SolveLaunch &L = prog[li];
         switch (L.kind) {
             case SK_SMALL_F: launch_fwd_solve(d, c->d_solve_list + L.off, (int)L.count, y, st); break;
-            case SK_INIT_F: launch_fsolve_init(d, c->d_solve_list + L.off, (int)L.count, y, st); break;
-            case SK_DF_F: launch_fsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, y, tk0 + 2 * li, st); break;
+            case SK_INIT_F: launch_fsolve_init(d, c->d_df_tasks + 2 * L.off, L.count, y, st); break;
+            case SK_DF_F: launch_fsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, L.j0, y, tk0 + 2 * li, st); break;
             case SK_SMALL_B:
                 launch_bwd_solve(d, c->d_solve_list + L.off, (int)L.count, y, c->d_sn_rows, c->d_sn_rowptr, st);
                 break;
             case SK_INIT_B:
-                launch_bsolve_init(d, c->d_solve_list + L.off, (int)L.count, y, c->d_sn_rows, c->d_sn_rowptr, st);
+                launch_bsolve_init(d, c->d_df_tasks + 2 * L.off, L.count, y, c->d_sn_rows, c->d_sn_rowptr, st);
                 break;
-            case SK_DF_B: launch_bsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, y, tk0 + 2 * li, st); break;
+            case SK_DF_B: launch_bsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, L.j0, y, tk0 + 2 * li, st); break;
         }
     }
 }
@@ -1060,11 +1054,6 @@ int ensure_slots(mf_ctx *c, int ns) {
         q.d.fv = (double *)p;
         if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.df_nparts, 1) * sizeof(double)))) return r;
         q.d.df_parts = (double *)p;
-        const size_t nfl = (size_t)std::max<int64_t>(P.df_nflags, 1) * sizeof(unsigned);
-        if ((r = dev_alloc(c, &p, nfl + 16))) return r;   // flags + the slot's solve epoch
-        CK(cudaMemsetAsync(p, 0, nfl + 16, c->stream));
-        q.d.df_flags = (unsigned *)p;
-        q.d.solve_epoch = (unsigned *)((char *)p + nfl);
         if ((r = dev_alloc(c, &p, tk_words * sizeof(unsigned)))) return r;
         CK(cudaMemsetAsync(p, 0, tk_words * sizeof(unsigned), c->stream));
         q.tickets = (unsigned *)p;

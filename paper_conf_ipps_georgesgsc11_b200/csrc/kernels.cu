@@ -1278,11 +1278,7 @@ void launch_export_diag(const DevPlan &d, int nsuper, double *out, cudaStream_t 
 // per-front update vectors that the parent gathers through the same relative
 // maps as the extend-add (deterministic, no atomics).
 __global__ void k_permute_in(const int32_t *__restrict__ perm, const double *__restrict__ b, double *__restrict__ y,
-                             int64_t n, unsigned *solve_epoch) {
-    if (blockIdx.x == 0 && threadIdx.x == 0) {   // 20 bits (backward flags carry a 12-bit block counter); never 0
-        const unsigned e = (*solve_epoch + 1) & 0xfffffu;
-        *solve_epoch = e ? e : 1u;
-    }
+                             int64_t n) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
         y[i] = b[perm[i]];
 }
@@ -1292,7 +1288,7 @@ __global__ void k_permute_out(const int32_t *__restrict__ perm, const double *__
         x[perm[i]] = xf[i];
 }
 void launch_permute_in(const DevPlan &d, const double *b, double *y, int64_t n, cudaStream_t st) {
-    if (n > 0) k_permute_in<<<(unsigned)((n + 255) / 256 < 4096 ? (n + 255) / 256 : 4096), 256, 0, st>>>(d.perm, b, y, n, d.solve_epoch);
+    if (n > 0) k_permute_in<<<(unsigned)((n + 255) / 256 < 4096 ? (n + 255) / 256 : 4096), 256, 0, st>>>(d.perm, b, y, n);
 }
 void launch_permute_out(const DevPlan &d, const double *xf, double *x, int64_t n, cudaStream_t st) {
     if (n > 0) k_permute_out<<<(unsigned)((n + 255) / 256 < 4096 ? (n + 255) / 256 : 4096), 256, 0, st>>>(d.perm, xf, x, n);
@@ -1357,87 +1353,72 @@ __global__ void __launch_bounds__(kSolveThreads) k_bwd_solve(DevPlan d, const in
     }
 }
 
-// ---- large supernodes: blocked by w = 64 columns, many CTAs per supernode
-__global__ void __launch_bounds__(kSolveThreads) k_fsolve_init(DevPlan d, const int32_t *__restrict__ list,
-                                                               const double *__restrict__ y) {
-    const int s = list[blockIdx.x];
+// ---- dataflow solve hand-off: every published value is its own flag.  A slot that
+// is not yet written holds kSolvePending, a signaling-NaN bit pattern that no fp64
+// arithmetic produces (NaN results are quiet), so a consumer polls the value itself
+// (one L2 round trip; no flag word, no fence on the producer).  k_fsolve_init sets the
+// forward block entries of y pending, k_bsolve_init the backward x slots.
+constexpr unsigned long long kSolvePending = 0x7ff40000df5e0001ull;
+__device__ __forceinline__ double ld_relaxed_f64(const double *p) {
+    double v;
+    asm volatile("ld.relaxed.gpu.global.f64 %0, [%1];" : "=d"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ double wait_value(const double *p) {
+    double v;
+    while ((unsigned long long)__double_as_longlong(v = ld_relaxed_f64(p)) == kSolvePending) {
+    }
+    return v;
+}
+__device__ __forceinline__ double pending_value() { return __longlong_as_double((long long)kSolvePending); }
+
+#ifndef MF_DF_BUF
+#define MF_DF_BUF 2
+#endif
+constexpr int kSW = 64, kSLD = 65;   // solve block width and smem leading dimension
+constexpr int kDfThreads = 256;      // dataflow solve CTA: 64 rows x 4 groups of 16 columns
+constexpr int kDfRB = 64;            // rows per forward task / per backward slab
+constexpr int kDfBuf = MF_DF_BUF;    // register ring: blocks (forward) / slabs (backward) in flight
+constexpr int kInitRows = kSolveInitRows;   // rows of a front vector per init task
+
+// ---- large supernodes: v = [y(cols); 0] + the children's update vectors, one task
+// per (supernode, 2048-row part); a part finds each child's entries that land in it
+// by binary search (rel is increasing), children in a fixed order: deterministic.
+__global__ void __launch_bounds__(kSolveThreads) k_fsolve_init(DevPlan d, const int32_t *__restrict__ tasks,
+                                                               double *__restrict__ y) {
+    const int s = tasks[2 * blockIdx.x], part = tasks[2 * blockIdx.x + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], first = d.sn_first[s];
+    const int p0 = part * kInitRows, p1 = min(f, p0 + kInitRows);
     double *__restrict__ v = d.fv + d.fv_off[s];
-    for (int i = threadIdx.x; i < f; i += kSolveThreads) v[i] = i < k ? y[first + i] : 0.0;
-    __syncthreads();
+    for (int i = p0 + threadIdx.x; i < p1; i += kSolveThreads) {
+        v[i] = i < k ? y[first + i] : 0.0;
+        if (i < k) y[first + i] = pending_value();   // x of this column: published by k_fsolve_df
+    }
     for (int q = d.child_ptr[s]; q < d.child_ptr[s + 1]; q++) {
+        __syncthreads();
         const int c = d.child_list[q];
         const int kc = d.sn_k[c], mc = d.sn_f[c] - kc;
         const int32_t *__restrict__ rel = d.relmap + d.relmap_ptr[c];
         const double *__restrict__ vc = d.fv + d.fv_off[c] + kc;
-        for (int p = threadIdx.x; p < mc; p += kSolveThreads) v[rel[p]] += vc[p];
-        __syncthreads();
+        const int lo = lower_bound_rel(rel, 0, mc, p0), hi = lower_bound_rel(rel, lo, mc, p1);
+        for (int p = lo + threadIdx.x; p < hi; p += kSolveThreads) v[rel[p]] += vc[p];
     }
 }
 
-constexpr int kSW = 64, kSLD = 65;   // solve block width and smem leading dimension
-
-
-__global__ void __launch_bounds__(kSolveThreads) k_bsolve_init(DevPlan d, const int32_t *__restrict__ list,
+// v(k:f) = x(R(k:f)) (ancestors are final); the backward x slots of the pivot columns pending
+__global__ void __launch_bounds__(kSolveThreads) k_bsolve_init(DevPlan d, const int32_t *__restrict__ tasks,
                                                                const double *__restrict__ y,
                                                                const int32_t *__restrict__ sn_rows,
                                                                const int64_t *__restrict__ sn_rowptr) {
-    const int s = list[blockIdx.x];
+    const int s = tasks[2 * blockIdx.x], part = tasks[2 * blockIdx.x + 1];
     const int k = d.sn_k[s], f = d.sn_f[s];
+    const int p0 = part * kInitRows, p1 = min(f, p0 + kInitRows);
     double *__restrict__ v = d.fv + d.fv_off[s];
+    double *__restrict__ xp = d.df_parts + d.df_part_off[s];
     const int32_t *__restrict__ R = sn_rows + sn_rowptr[s];
-    for (int i = k + threadIdx.x; i < f; i += kSolveThreads) v[i] = y[R[i]];
-}
-
-// ---- dataflow solves: one launch per level for all its large supernodes.  CTA =
-// one 256-row chunk of one front, one row per thread (value in a register).
-// Forward: for each 64-column block b in order, the chunk that holds the block's
-// rows solves its triangle and publishes x_b (flag = solve epoch); every chunk
-// below applies v -= L(rows, b) x_b.  Backward: for each block b in reverse, every
-// chunk below the block publishes its partial L(rows, b)^T x(rows); the owner
-// sums them in a fixed chunk order (deterministic) and solves L_bb^T x_b = t.
-// CTAs are ordered so that a chunk only waits on lower CTA ids.
-__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned *p) {
-    unsigned v;
-    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ void st_release_u32(unsigned *p, unsigned v) {
-    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-
-// Row r's 64 entries of the column block [j0, j0 + we), zero past we (independent
-// loads: the whole slab is in flight at once).
-__device__ __forceinline__ void load_row_block(const double *__restrict__ P, int64_t ld, int r, int j0, int we,
-                                               bool ok, double (&Lr)[kSW]) {
-    const double *__restrict__ col = P + (int64_t)j0 * ld + r;
-#pragma unroll
-    for (int q = 0; q < kSW; q++) Lr[q] = (ok && q < we) ? col[(int64_t)q * ld] : 0.0;
-}
-
-// Half a row slab: row r's 32 entries of the columns [j0 + 32 h, j0 + 32 h + 32) of a
-// block (zero past we or when !ok).  The sweeps below keep two halves in registers:
-// while one is used, the next one is in flight (software pipelining across blocks).
-__device__ __forceinline__ void load_half(const double *__restrict__ P, int64_t ld, int r, int j0, int h, int we,
-                                          bool ok, double (&Lh)[32]) {
-    const double *__restrict__ col = P + (int64_t)(j0 + 32 * h) * ld + r;
-#pragma unroll
-    for (int q = 0; q < 32; q++) Lh[q] = (ok && 32 * h + q < we) ? col[(int64_t)q * ld] : 0.0;
-}
-// Butterfly reduce-scatter over the warp: 32 values per lane in, lane l ends with the
-// warp sum of value l in p[0] (31 shuffles).
-__device__ __forceinline__ void warp_reduce_scatter32(double (&p)[32]) {
-    const int lane = threadIdx.x & 31;
-#pragma unroll
-    for (int st = 0; st < 5; st++) {
-        const int half = 16 >> st, off = 16 >> st;
-        const bool up = (lane & off) != 0;
-#pragma unroll
-        for (int i = 0; i < half; i++) {
-            const double send = up ? p[i] : p[i + half];
-            const double keep = up ? p[i + half] : p[i];
-            p[i] = keep + __shfl_xor_sync(0xffffffffu, send, off);
-        }
+    for (int i = p0 + threadIdx.x; i < p1; i += kSolveThreads) {
+        if (i >= k) v[i] = y[R[i]];
+        else xp[i] = pending_value();
     }
 }
 
@@ -1480,234 +1461,260 @@ void launch_diag_inv(const DevPlan &d, const int32_t *tasks, int64_t count, int 
     if (count > 0) k_diag_inv<<<(unsigned)count, 64, 0, st>>>(d, tasks, w);
 }
 
-// 256 threads: out[i] = sum_q M[i + q 64] v[q] (trans = 0) or sum_q M[q + i 64] v[q]
-// (trans = 1) for the 64 x 64 column-major M; thread (i, g) sums q in [16 g, 16 g + 16)
-// from registers mr[16] (prefetched with oz_prefetch_inv), then the four quarters are
-// added in a fixed order (deterministic).
-__device__ __forceinline__ void inv_prefetch(const double *__restrict__ M, bool trans, double (&mr)[16]) {
-    const int i = threadIdx.x & 63, g = threadIdx.x >> 6;
+// ---- dataflow solves: one launch per level for all its large supernodes.  A CTA is
+// 64 rows x 4 column groups (thread (i, g) = row i, columns [16 g, 16 g + 16) of a
+// 64-column block); the L data streams through a ring of kDfBuf register blocks, issued
+// ahead of the values they multiply, so a task's only waits are for values.
+//
+// Forward (L y = b), row-oriented: task = 64 rows [r0, r0 + 64) of front s.  For
+// every column block b reaching the rows: wait for y_b (value by value), then each
+// thread adds its 16 products to a private partial sum.  The block the rows own
+// (j0 >= r0: the diagonal block) is solved in place: the partials are reduced into
+// t_b, x_b = inv(L_bb) t_b (all 256 threads, inverse staged in shared memory at task
+// start, off the chain) and published into y.  Rows >= k keep v for the parent.
+// The chain per block is one value hand-off + one 64 x 64 product + the inverse.
+__device__ __forceinline__ void fsolve_load(const double *__restrict__ P, int ld, int k, int w, int r, bool rok,
+                                            int b, double (&Lb)[16]) {
+    const int g = threadIdx.x >> 6, j0 = b * w, we = min(w, k - j0);
+    const bool ok = rok && r >= j0 + we;   // the diagonal block's own rows take no part
 #pragma unroll
     for (int u = 0; u < 16; u++) {
-        const int q = 16 * g + u;
-        mr[u] = __ldg(trans ? M + q + i * kSW : M + i + q * kSW);
+        const int c = 16 * g + u;
+        Lb[u] = (ok && c < we) ? P[(int64_t)(j0 + c) * ld + r] : 0.0;
     }
 }
-__device__ __forceinline__ double inv_apply(const double (&mr)[16], const double *__restrict__ v,
-                                            double (*red)[kSW]) {
-    const int i = threadIdx.x & 63, g = threadIdx.x >> 6;
-    double a = 0.0;
-#pragma unroll
-    for (int u = 0; u < 16; u++) a = fma(mr[u], v[16 * g + u], a);
-    red[g][i] = a;
-    __syncthreads();
-    return (red[0][i] + red[1][i]) + (red[2][i] + red[3][i]);   // valid for threads < 64
-}
-
-// Forward: CTA = 256-row chunk c of front s; for each 64-column block b whose rows
-// reach the chunk: every row's slab L(r, b) is in registers (two 32-column halves,
-// each loaded one half ahead of its use, so a lagging chunk streams its slabs
-// instead of paying a load latency per block); the chunk that holds block b's rows
-// (the owner) forms x_b = inv(L_bb) t_b with all 256 threads and publishes it (flag
-// = solve epoch); the others wait for it; then every row applies v_r -= L(r, b) x_b.
-// The owner's own block rows take no part in that product: their value becomes x.
-__device__ __forceinline__ void fsolve_df_task(const DevPlan &d, const int32_t *__restrict__ tasks, int w,
-                                               double *__restrict__ y, const int task) {
-    __shared__ double xs[kSW];
+template <int NBUF>
+__device__ __forceinline__ void fsolve_rows_task(const DevPlan &d, const int32_t *__restrict__ tasks, int w,
+                                                 double *__restrict__ y, const int task) {
+    __shared__ double Ms[kSW * kSLD];   // inv(L_bb) of the owned block: element (q, c) at q + c kSLD
+    __shared__ double ys[2][kSW];
     __shared__ double red[4][kSW];
-    const int s = tasks[2 * task], c = tasks[2 * task + 1];
+    __shared__ double vrow[kSW];
+    const int s = tasks[2 * task], rb = tasks[2 * task + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
     const double *__restrict__ P = d.L + d.L_off[s];
     const double *__restrict__ Dinv = d.dinv + d.dinv_off[s];
     double *__restrict__ v = d.fv + d.fv_off[s];
-    unsigned *__restrict__ bflag = d.df_flags + d.df_blk_off[s];
-    const unsigned epoch = *d.solve_epoch;
-    const int tid = threadIdx.x;
-    const int c_lo = c * kSolveRows, c_hi = min(c_lo + kSolveRows, f);
-    const int r = c_lo + tid;
-    const bool rok = r < c_hi;
-    double vr = rok ? v[r] : 0.0;
-    const int nb = min((k + w - 1) / w, (c_hi + w - 1) / w);   // blocks reaching this chunk
-    double H0[32], H1[32];
-    if (nb > 0) load_half(P, ld, r, 0, 0, min(w, k), rok, H0);
-    for (int b = 0; b < nb; b++) {
-        const int j0 = b * w, we = min(w, k - j0);
-        const bool okr = rok && r >= j0;
-        load_half(P, ld, r, j0, 1, we, okr, H1);   // second half in flight
-        if (j0 >= c_lo) {        // this chunk owns the block: x_b = inv(L_bb) t_b
-            double mr[16];
-            inv_prefetch(Dinv + (int64_t)b * kSW * kSW, false, mr);
-            const int i = r - j0;
-            const bool own = rok && i >= 0 && i < we;
-            if (own) {
-                xs[i] = vr;
+    const int tid = threadIdx.x, i = tid & 63, g = tid >> 6;
+    const int r0 = rb * kDfRB, r = r0 + i;
+    const bool rok = r < f;
+    const int nbr = (min(k, r0 + kDfRB) + w - 1) / w;   // column blocks reaching these rows
+    const int bown = r0 < k ? r0 / w : nbr;              // first owned block (w divides 64)
+    auto load_inv = [&](int b) {
+        const double *__restrict__ M = Dinv + (int64_t)b * kSW * kSW;
+        for (int q = tid; q < kSW * kSW; q += kDfThreads) Ms[(q & 63) + (q >> 6) * kSLD] = __ldg(M + q);
+    };
+    if (tid < kSW) vrow[tid] = rok ? v[r] : 0.0;
+    if (bown < nbr) load_inv(bown);
+    double Lb[NBUF][16];
 #pragma unroll
-                for (int q = 0; q < 32; q++) H0[q] = H1[q] = 0.0;
+    for (int q = 0; q < NBUF; q++)
+        if (q < nbr) fsolve_load(P, ld, k, w, r, rok, q, Lb[q]);
+    double acc = 0.0;
+    for (int b0 = 0; b0 < nbr; b0 += NBUF) {
+#pragma unroll
+        for (int q = 0; q < NBUF; q++) {
+            const int b = b0 + q;
+            if (b >= nbr) break;
+            const int j0 = b * w, we = min(w, k - j0);
+            double *yb = ys[b & 1];
+            const bool owned = j0 >= r0;
+            if (owned) {   // t_b = v - partials (rows of the block), x_b = inv(L_bb) t_b
+                red[g][i] = acc;
+                acc = 0.0;
+                __syncthreads();
+                if (tid < kSW) vrow[i] -= (red[0][i] + red[1][i]) + (red[2][i] + red[3][i]);
+                __syncthreads();
+                double a = 0.0;
+#pragma unroll
+                for (int u = 0; u < 16; u++) {
+                    const int c = 16 * g + u;
+                    a = fma(Ms[i + c * kSLD], c < we ? vrow[j0 - r0 + c] : 0.0, a);
+                }
+                red[g][i] = a;
+                __syncthreads();
+                if (tid < kSW) {
+                    const double x = (red[0][i] + red[1][i]) + (red[2][i] + red[3][i]);
+                    if (i < we) {
+                        __stcg(y + first + j0 + i, x);   // published: the value is its flag
+                        vrow[j0 - r0 + i] = x;
+                    }
+                    yb[i] = i < we ? x : 0.0;
+                }
+            } else if (tid < kSW) {   // a block above: its solution, value by value
+                yb[tid] = tid < we ? wait_value(y + first + j0 + tid) : 0.0;
             }
-            if (tid < kSW && tid >= we) xs[tid] = 0.0;
             __syncthreads();
-            const double xb = inv_apply(mr, xs, red);
-            if (tid < we) y[first + j0 + tid] = xb;
-            __syncthreads();     // every thread read xs / red
-            if (tid < kSW) xs[tid] = tid < we ? xb : 0.0;
-            __threadfence();
-            __syncthreads();
-            if (tid == 0) st_release_u32(bflag + b, epoch);
-            if (own) vr = xs[i];
-        } else {                 // a block above: wait for its solution
-            if (tid == 0)
-                while (ld_acquire_u32(bflag + b) != epoch) __nanosleep(32);
-            __syncthreads();
-            if (tid < kSW) xs[tid] = tid < we ? __ldcg(y + first + j0 + tid) : 0.0;
-            __syncthreads();
-        }
-        double a0 = 0.0, a1 = 0.0;
+            if (owned && b + 1 < nbr && (b + 1) * w < r0 + kDfRB) load_inv(b + 1);   // w < 64: the next owned block
 #pragma unroll
-        for (int q = 0; q < 32; q += 2) {
-            a0 += H0[q] * xs[q];
-            a1 += H0[q + 1] * xs[q + 1];
+            for (int u = 0; u < 16; u++) acc = fma(Lb[q][u], yb[16 * g + u], acc);
+            if (b + NBUF < nbr) fsolve_load(P, ld, k, w, r, rok, b + NBUF, Lb[q]);
         }
-        if (b + 1 < nb) {        // the next block's first half, while the second half is used
-            const int j1 = j0 + w;
-            load_half(P, ld, r, j1, 0, min(w, k - j1), rok && r >= j1, H0);
-        }
-#pragma unroll
-        for (int q = 0; q < 32; q += 2) {
-            a0 += H1[q] * xs[32 + q];
-            a1 += H1[q + 1] * xs[33 + q];
-        }
-        vr -= a0 + a1;           // rows not below the block have zero slabs
-        __syncthreads();
     }
-    if (rok && r >= k) v[r] = vr;   // the update vector the parent gathers
+    red[g][i] = acc;
+    __syncthreads();
+    if (tid < kSW && rok && r >= k) v[r] = vrow[i] - ((red[0][i] + red[1][i]) + (red[2][i] + red[3][i]));
 }
-__global__ void __launch_bounds__(kSolveThreads) k_fsolve_df(DevPlan d, const int32_t *__restrict__ tasks, int w,
-                                                             double *__restrict__ y, unsigned *tk) {
-    fsolve_df_task(d, tasks, w, y, take_ticket(tk));
+// NBUF = ring depth, MINB = CTAs / SM (tools/gpu/job_df_variants.sh: c5 solve 8.26 ms at <4, 1>,
+// 7.12 at <2, 2>); levels of small fronts take the shallow ring at 3 CTAs / SM
+template <int NBUF, int MINB>
+__global__ void __launch_bounds__(kDfThreads, MINB) k_fsolve_df(DevPlan d, const int32_t *__restrict__ tasks, int w,
+                                                                double *__restrict__ y, unsigned *tk) {
+    fsolve_rows_task<NBUF>(d, tasks, w, y, take_ticket(tk));
     drop_ticket(tk);
 }
 
-// Butterfly reduce-scatter over the warp: 64 values per lane in, lane l ends with
-// the warp sums of q = 2 l + {0, 1} in p[0], p[1] (62 shuffles).
-__device__ __forceinline__ void warp_reduce_scatter64(double (&p)[kSW]) {
+// Backward (L^T x = y), column-oriented: task = column block b of front s.  Its
+// dot products L(r, b)^T x_r run over the rows below the block in 64-row slabs:
+// first the rows >= k (final, from the ancestors), then the pivot rows from the top
+// block down (each thread waits for its own row's x, published by the task of that
+// block).  16 column partials per thread, reduced over the 64 rows at the end
+// (butterfly, fixed order); x_b = inv(L_bb)^T (y_b - dot) is published into y and
+// into the front's x slots.  The chain per block is one value hand-off + one slab +
+// the reduction and the inverse.
+__device__ __forceinline__ void bsolve_load(const double *__restrict__ P, int ld, int f, int j0, int we, int rlo,
+                                            int r, double (&Lb)[16]) {
+    const int g = threadIdx.x >> 6;
+    const bool ok = r >= rlo && r < f;
+#pragma unroll
+    for (int u = 0; u < 16; u++) {
+        const int c = 16 * g + u;
+        Lb[u] = (ok && c < we) ? P[(int64_t)(j0 + c) * ld + r] : 0.0;
+    }
+}
+// Butterfly reduce-scatter over the warp: 16 values per lane in; lane l ends with the
+// warp sum of value (l >> 1) & 15 in p[0] (16 shuffles).
+__device__ __forceinline__ void warp_reduce_scatter16(double (&p)[16]) {
     const int lane = threadIdx.x & 31;
 #pragma unroll
-    for (int st = 0; st < 5; st++) {
-        const int half = kSW >> (st + 1), off = 16 >> st;
+    for (int st = 0; st < 4; st++) {
+        const int half = 8 >> st, off = 16 >> st;
         const bool up = (lane & off) != 0;
 #pragma unroll
-        for (int i = 0; i < half; i++) {
-            const double send = up ? p[i] : p[i + half];
-            const double keep = up ? p[i + half] : p[i];
-            p[i] = keep + __shfl_xor_sync(0xffffffffu, send, off);
+        for (int j = 0; j < half; j++) {
+            const double send = up ? p[j] : p[j + half];
+            const double keep = up ? p[j + half] : p[j];
+            p[j] = keep + __shfl_xor_sync(0xffffffffu, send, off);
         }
     }
+    p[0] += __shfl_xor_sync(0xffffffffu, p[0], 1);
 }
-
-__device__ __forceinline__ void bsolve_df_task(const DevPlan &d, const int32_t *__restrict__ tasks, int w,
-                                               double *__restrict__ y, const int task) {
-    __shared__ double red[kSolveThreads / 32][kSW];
+template <int NBUF>
+__device__ __forceinline__ void bsolve_cols_task(const DevPlan &d, const int32_t *__restrict__ tasks, int w,
+                                                 double *__restrict__ y, const int task) {
+    __shared__ double Ms[kSW * kSLD];   // inv(L_bb)^T: element (q, c) = inv(c, q) at q + c kSLD
+    __shared__ double red[8][16];
     __shared__ double tv[kSW];
-    const int s = tasks[2 * task], c = tasks[2 * task + 1];
+    __shared__ double rx[4][kSW];
+    const int s = tasks[2 * task], b = tasks[2 * task + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
     const double *__restrict__ P = d.L + d.L_off[s];
-    const double *__restrict__ Dinv = d.dinv + d.dinv_off[s];
-    double *__restrict__ v = d.fv + d.fv_off[s];
-    const int nb = (k + w - 1) / w, nc = (f + kSolveRows - 1) / kSolveRows;
-    unsigned *__restrict__ cflag = d.df_flags + d.df_blk_off[s] + nb;
-    double *__restrict__ part = d.df_parts + d.df_part_off[s];
-    const unsigned epoch = *d.solve_epoch;
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int c_lo = c * kSolveRows, c_hi = min(c_lo + kSolveRows, f);
-    const int r = c_lo + tid;
-    const bool rok = r < c_hi;
-    double xr = (rok && r >= k) ? v[r] : 0.0;   // rows >= k: final (gathered from the ancestors)
-    const int btop = min(nb, (c_hi + w - 1) / w) - 1;   // the first block (from the bottom) reaching this chunk
-    // rows taking part in block b's partial: below the block (the owner's own block rows: none)
-    auto rows_ok = [&](int b) {
-        const int j0 = b * w;
-        return rok && r >= j0 + (j0 >= c_lo ? min(w, k - j0) : 0);
-    };
-    double H0[32], H1[32];
-    if (btop >= 0) load_half(P, ld, r, btop * w, 0, min(w, k - btop * w), rows_ok(btop), H0);
-    for (int b = btop; b >= 0; b--) {
-        const int j0 = b * w, we = min(w, k - j0);
-        const bool owner = j0 >= c_lo;
-        load_half(P, ld, r, j0, 1, we, rows_ok(b), H1);   // second half in flight
-        double mr[16];
-        if (owner) inv_prefetch(Dinv + (int64_t)b * kSW * kSW, true, mr);
-        // partial L(rows, b)^T x(rows) over this chunk's rows below the block, per half
+    const double *__restrict__ v = d.fv + d.fv_off[s];
+    double *__restrict__ xp = d.df_parts + d.df_part_off[s];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, i = tid & 63, g = tid >> 6;
+    const int j0 = b * w, we = min(w, k - j0), rlo = j0 + we;   // rows below the block
+    {
+        const double *__restrict__ M = d.dinv + d.dinv_off[s] + (int64_t)b * kSW * kSW;
+        for (int q = tid; q < kSW * kSW; q += kDfThreads) Ms[(q >> 6) + (q & 63) * kSLD] = __ldg(M + q);
+    }
+    const double yb = (tid < we) ? y[first + j0 + tid] : 0.0;   // forward result of the block (this task rewrites it)
+    // slabs: the tail slabs (rows >= k only) ascending, then the pivot slabs from the
+    // one holding row k - 1 down to the one holding row rlo (the first of them may also
+    // hold rows >= k).  The last block (rlo >= k) has tail slabs only, from rlo's.
+    const int ktop = (k - 1) / kDfRB, np = rlo < k ? ktop - rlo / kDfRB + 1 : 0;
+    const int kt0 = np > 0 ? ktop + 1 : rlo / kDfRB, nsl = (f + kDfRB - 1) / kDfRB;
+    const int nt = max(0, nsl - kt0);
+    const int ns = nt + np;
+    auto slab_row = [&](int q) { return (q < nt ? kt0 + q : ktop - (q - nt)) * kDfRB + i; };
+    double Lb[NBUF][16];
 #pragma unroll
-        for (int q = 0; q < 32; q++) H0[q] *= xr;
-        warp_reduce_scatter32(H0);
-        red[warp][lane] = H0[0];
-        if (b > 0) {             // the next block's first half, while this half is reduced
-            const int j1 = j0 - w;
-            load_half(P, ld, r, j1, 0, min(w, k - j1), rows_ok(b - 1), H0);
-        }
+    for (int q = 0; q < NBUF; q++)
+        if (q < ns) bsolve_load(P, ld, f, j0, we, rlo, slab_row(q), Lb[q]);
+    double acc[16];
 #pragma unroll
-        for (int q = 0; q < 32; q++) H1[q] *= xr;
-        warp_reduce_scatter32(H1);
-        red[warp][32 + lane] = H1[0];
-        __syncthreads();
-        double mine = 0.0;
-        if (tid < we)
+    for (int u = 0; u < 16; u++) acc[u] = 0.0;
+    for (int q0 = 0; q0 < ns; q0 += NBUF) {
 #pragma unroll
-            for (int q = 0; q < kSolveThreads / 32; q++) mine += red[q][tid];
-        // the partial of every chunk below, accumulated down the chunks: chunk cc publishes
-        // S_cc(b) = own_cc(b) + S_{cc+1}(b) (a fixed order: deterministic), so the owner
-        // reads one vector instead of summing all the chunks below on its critical path,
-        // and the chunks pass the sums along like a systolic array
-        double below = 0.0;
-        if (c + 1 < nc) {
-            if (tid == 0)
-                for (;;) {
-                    const unsigned fl = ld_acquire_u32(cflag + c + 1);
-                    if ((fl >> 12) == epoch && (fl & 0xfffu) >= (unsigned)(nb - b)) break;
-                    __nanosleep(32);
-                }
-            __syncthreads();
-            if (tid < we) below = __ldcg(part + ((int64_t)(c + 1) * nb + b) * w + tid);
+        for (int q = 0; q < NBUF; q++) {
+            const int sq = q0 + q;
+            if (sq >= ns) break;
+            const int r = slab_row(sq);
+            const double xr = (r >= rlo && r < f) ? (r >= k ? v[r] : wait_value(xp + r)) : 0.0;
+#pragma unroll
+            for (int u = 0; u < 16; u++) acc[u] = fma(Lb[q][u], xr, acc[u]);
+            if (sq + NBUF < ns) bsolve_load(P, ld, f, j0, we, rlo, slab_row(sq + NBUF), Lb[q]);
         }
-        if (!owner) {                             // publish own + everything below
-            if (tid < we) {
-                part[((int64_t)c * nb + b) * w + tid] = mine + below;
-                __threadfence();
-            }
-            __syncthreads();
-            if (tid == 0) st_release_u32(cflag + c, (epoch << 12) | (unsigned)(nb - b));
-            continue;
-        }
-        if (tid < kSW) tv[tid] = tid < we ? y[first + j0 + tid] - (mine + below) : 0.0;
-        __syncthreads();
-        const double xb = inv_apply(mr, tv, red);   // x_b = inv(L_bb)^T t
-        if (tid < we) y[first + j0 + tid] = xb;
-        __syncthreads();                            // tv / red read by every thread
-        if (tid < kSW) tv[tid] = tid < we ? xb : 0.0;
-        __syncthreads();
-        if (rok && r >= j0 && r < j0 + we) xr = tv[r - j0];
-        __syncthreads();
+    }
+    warp_reduce_scatter16(acc);   // lane l: value (l >> 1) & 15 over this warp's 32 rows
+    if ((lane & 1) == 0) red[warp][lane >> 1] = acc[0];
+    __syncthreads();
+    if (tid < kSW) {   // column c = 16 g' + u': the two warps of group g'
+        const int gc = tid >> 4, u = tid & 15;
+        tv[tid] = tid < we ? yb - (red[2 * gc][u] + red[2 * gc + 1][u]) : 0.0;
+    }
+    __syncthreads();
+    double a = 0.0;
+#pragma unroll
+    for (int u = 0; u < 16; u++) a = fma(Ms[i + (16 * g + u) * kSLD], tv[16 * g + u], a);
+    rx[g][i] = a;
+    __syncthreads();
+    if (tid < we) {
+        const double x = (rx[0][i] + rx[1][i]) + (rx[2][i] + rx[3][i]);
+        y[first + j0 + i] = x;
+        __stcg(xp + j0 + i, x);   // published: the value is its flag
     }
 }
-__global__ void __launch_bounds__(kSolveThreads) k_bsolve_df(DevPlan d, const int32_t *__restrict__ tasks, int w,
-                                                             double *__restrict__ y, unsigned *tk) {
-    bsolve_df_task(d, tasks, w, y, take_ticket(tk));
+template <int NBUF, int MINB>
+__global__ void __launch_bounds__(kDfThreads, MINB) k_bsolve_df(DevPlan d, const int32_t *__restrict__ tasks, int w,
+                                                                double *__restrict__ y, unsigned *tk) {
+    bsolve_cols_task<NBUF>(d, tasks, w, y, take_ticket(tk));
     drop_ticket(tk);
 }
 
-void launch_fsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, cudaStream_t st) {
-    if (count > 0) k_fsolve_init<<<count, kSolveThreads, 0, st>>>(d, list, y);
+void launch_fsolve_init(const DevPlan &d, const int32_t *tasks, int64_t count, double *y, cudaStream_t st) {
+    if (count > 0) k_fsolve_init<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, y);
 }
-void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, unsigned *tk,
-                      cudaStream_t st) {
-    if (count > 0) k_fsolve_df<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, w, y, tk);
+// MF_DF_VARIANT (tuning A/B): deep ring 0 = <2 blocks, 2 CTAs/SM>, 1 = <3, 2>, 2 = <4, 1>, 3 = <2, 3>
+static int df_variant() {
+    static const int v = [] {
+        const char *e = getenv("MF_DF_VARIANT");
+        return e ? atoi(e) : 0;
+    }();
+    return v;
 }
-void launch_bsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, const int32_t *sn_rows,
-                        const int64_t *sn_rowptr, cudaStream_t st) {
-    if (count > 0) k_bsolve_init<<<count, kSolveThreads, 0, st>>>(d, list, y, sn_rows, sn_rowptr);
+void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, int deep, double *y,
+                      unsigned *tk, cudaStream_t st) {
+    if (count <= 0) return;
+    const unsigned n = (unsigned)count;
+    if (!deep)
+        k_fsolve_df<1, 3><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+    else if (df_variant() == 1)
+        k_fsolve_df<3, 2><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+    else if (df_variant() == 2)
+        k_fsolve_df<4, 1><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+    else if (df_variant() == 3)
+        k_fsolve_df<2, 3><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+    else
+        k_fsolve_df<kDfBuf, 2><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
 }
-void launch_bsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, unsigned *tk,
-                      cudaStream_t st) {
-    if (count > 0) k_bsolve_df<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, w, y, tk);
+void launch_bsolve_init(const DevPlan &d, const int32_t *tasks, int64_t count, const double *y,
+                        const int32_t *sn_rows, const int64_t *sn_rowptr, cudaStream_t st) {
+    if (count > 0) k_bsolve_init<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, y, sn_rows, sn_rowptr);
+}
+void launch_bsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, int deep, double *y,
+                      unsigned *tk, cudaStream_t st) {
+    if (count <= 0) return;
+    const unsigned n = (unsigned)count;
+    if (!deep)
+        k_bsolve_df<1, 3><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+    else if (df_variant() == 1)
+        k_bsolve_df<3, 2><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+    else if (df_variant() == 2)
+        k_bsolve_df<4, 1><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+    else if (df_variant() == 3)
+        k_bsolve_df<2, 3><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+    else
+        k_bsolve_df<kDfBuf, 2><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
 }
 
 // dst[first_s + j] = src[first_s + j] for the columns of the listed supernodes

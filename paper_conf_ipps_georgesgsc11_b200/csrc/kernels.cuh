@@ -26,10 +26,8 @@ struct DevPlan {
     const unsigned *epoch;   // factorization counter (= failed + 1), bumped by the init kernel
     unsigned *leaf_flag;     // per supernode: fused-leaf "diagonal block done" flag
     unsigned *panel_flag;    // per supernode: kPanelFlags dataflow-panel tile flags
-    unsigned *solve_epoch;   // solve counter (= failed + 2), bumped by the first solve kernel
-    unsigned *df_flags;      // dataflow solve flags (forward per block, backward per chunk)
-    double *df_parts;        // dataflow backward partial sums per (chunk, block)
-    const int64_t *df_blk_off, *df_part_off;
+    double *df_parts;        // dataflow backward sweep: published x of the pivot columns (value = flag)
+    const int64_t *df_part_off;
     double *dinv;            // dataflow solve: inverses of the 64 x 64 diagonal blocks (solve setup)
     const int64_t *dinv_off; // per supernode: word offset of its blocks in dinv (-1: none)
     const int32_t *ea_qs;    // fused extend-add: tile-row start tables of the syrk problems
@@ -75,13 +73,15 @@ void launch_bwd_solve(const DevPlan &d, const int32_t *list, int count, double *
                       const int64_t *sn_rowptr, cudaStream_t st);
 // solve setup: inverses of the 64 x 64 diagonal blocks of the dataflow-solved supernodes
 void launch_diag_inv(const DevPlan &d, const int32_t *tasks, int64_t count, int w, cudaStream_t st);
-void launch_fsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, cudaStream_t st);
-void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, unsigned *tk,
-                      cudaStream_t st);
-void launch_bsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, double *y, unsigned *tk,
-                      cudaStream_t st);
-void launch_bsolve_init(const DevPlan &d, const int32_t *list, int count, const double *y, const int32_t *sn_rows,
-                        const int64_t *sn_rowptr, cudaStream_t st);
+// (supernode, 2048-row part) pairs: front vectors of the large supernodes, children gathered
+void launch_fsolve_init(const DevPlan &d, const int32_t *tasks, int64_t count, double *y, cudaStream_t st);
+// deep = 1: the levels with multi-block fronts (register ring of MF_DF_BUF blocks, 1 CTA / SM)
+void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, int deep, double *y,
+                      unsigned *tk, cudaStream_t st);
+void launch_bsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, int deep, double *y,
+                      unsigned *tk, cudaStream_t st);
+void launch_bsolve_init(const DevPlan &d, const int32_t *tasks, int64_t count, const double *y,
+                        const int32_t *sn_rows, const int64_t *sn_rowptr, cudaStream_t st);
 
 int small_front_smem_ok(int fmax);
 int kernels_init();

@@ -210,7 +210,7 @@ enum SolveKind : int32_t {
 };
 struct SolveLaunch {
     int32_t kind;
-    int32_t j0;
+    int32_t j0;   // factor launches: first column; SK_DF_*: 1 = deep register ring
     int64_t off, count;
 };
 
@@ -241,8 +241,8 @@ struct Plan {
     // solve
     std::vector<int32_t> solve_list;                 // supernode lists (small / large) per launch
     std::vector<int32_t> df_tasks;                   // dataflow solve: (front, chunk) pairs
-    std::vector<int64_t> df_blk_off, df_part_off;    // per supernode: block-flag and partial-sum bases
-    int64_t df_nflags = 0, df_nparts = 0;            // u32 flags / fp64 partial words
+    std::vector<int64_t> df_part_off;                // per supernode: base of its backward x slots (k words)
+    int64_t df_nparts = 0;                           // fp64 x-slot words
     // inverses of the 64 x 64 diagonal blocks of the dataflow-solved supernodes (solve setup,
     // computed once per factorization by the first solve): per supernode the word offset of
     // its ceil(k / 64) column-major 64 x 64 blocks; (supernode, block) task pairs
@@ -281,7 +281,9 @@ constexpr int kAsmCols = 16;
 constexpr int kAsmRowBlock = 2048;   // assembly tasks split tall fronts into row blocks of this many rows
 constexpr int kTrsmRows = 128;
 constexpr int kSmallClasses = 5;
-constexpr int kSolveRows = 256;   // dataflow solve: rows per chunk (a multiple of the 64-column block)
+constexpr int kSolveRowBlock = 64;    // dataflow forward solve: rows per task (a multiple of the block width w)
+constexpr int kSolveDeepK = 256;      // dataflow solve: levels with a front of k >= this take the deep ring
+constexpr int kSolveInitRows = 2048;  // solve init: front-vector rows per task (kernels.cu kInitRows)
 
 int build_plan(const Symbolic &S, const Options &opt, Plan &P);
 

@@ -94,45 +94,77 @@ static void build_solve_plan(const Symbolic &S, Plan &P, const std::vector<char>
         P.solve_list.insert(P.solve_list.end(), v.begin(), v.end());
         return off;
     };
-    // dataflow solve of the large supernodes: 256-row chunks; flags per 64-column
-    // block (forward) and per chunk (backward); partial sums per (chunk, block)
+    // dataflow solve of the large supernodes (kernels.cu): forward tasks = 64-row
+    // blocks, backward tasks = w-column blocks; x slots of the backward sweep (one per
+    // pivot column) and the inverses of the diagonal blocks
     auto ensure_df = [&](int32_t s) {
-        if (P.df_blk_off[s] >= 0) return;
-        const int64_t nb = (P.sn_k[s] + w - 1) / w, nc = (P.sn_f[s] + kSolveRows - 1) / kSolveRows;
-        P.df_blk_off[s] = P.df_nflags;
-        P.df_nflags += nb + nc;   // nb forward block flags, then nc backward chunk flags
+        if (P.df_part_off[s] >= 0) return;
+        const int64_t nb = (P.sn_k[s] + w - 1) / w;
         P.dinv_off[s] = P.dinv_words;
         P.dinv_words += nb * 64 * 64;   // one 64 x 64 slot per block (w <= 64; identity-extended)
         for (int32_t b = 0; b < nb; b++) P.dinv_tasks.insert(P.dinv_tasks.end(), {s, b});
         P.df_part_off[s] = P.df_nparts;
-        P.df_nparts += nc * nb * w;
+        P.df_nparts += P.sn_k[s];
+    };
+    // the deep register ring (1 CTA / SM) for levels whose largest front has several
+    // blocks; the shallow one (3 CTAs / SM) for levels of small fronts
+    auto deep_level = [&](const std::vector<int32_t> &v) {
+        int32_t kmax = 0;
+        for (int32_t s : v) kmax = std::max(kmax, P.sn_k[s]);
+        return (int32_t)(kmax >= kSolveDeepK);
+    };
+    auto push_task = [&](int32_t s, int32_t t) {
+        P.df_tasks.push_back(s);
+        P.df_tasks.push_back(t);
+    };
+    auto push_init = [&](const std::vector<int32_t> &v) {   // (supernode, 2048-row part)
+        const int64_t off = (int64_t)P.df_tasks.size() / 2;
+        for (int32_t s : v)
+            for (int32_t q = 0; q * kSolveInitRows < P.sn_f[s]; q++) push_task(s, q);
+        return off;
     };
     for (int32_t l = 0; l < P.nlevels; l++) {
         if (!small[l].empty()) fsolve.push_back({SK_SMALL_F, 0, push_list(small[l]), (int64_t)small[l].size()});
         if (large[l].empty()) continue;
-        fsolve.push_back({SK_INIT_F, 0, push_list(large[l]), (int64_t)large[l].size()});
-        const int64_t off = (int64_t)P.df_tasks.size() / 2;
-        for (int32_t s : large[l]) {   // chunks top-down: a chunk waits only on earlier blocks (lower CTA ids)
-            ensure_df(s);
-            for (int32_t c = 0; c * kSolveRows < P.sn_f[s]; c++) {
-                P.df_tasks.push_back(s);
-                P.df_tasks.push_back(c);
-            }
+        {
+            const int64_t off = push_init(large[l]);
+            fsolve.push_back({SK_INIT_F, 0, off, (int64_t)P.df_tasks.size() / 2 - off});
         }
-        fsolve.push_back({SK_DF_F, 0, off, (int64_t)P.df_tasks.size() / 2 - off});
+        // the pivot-row tasks of every front first, round robin (every chain starts at
+        // once), then the rows below k; a task waits only on lower tickets of its front
+        const int64_t off = (int64_t)P.df_tasks.size() / 2;
+        int32_t maxrb = 0;
+        for (int32_t s : large[l]) {
+            ensure_df(s);
+            maxrb = std::max(maxrb, (P.sn_k[s] + kSolveRowBlock - 1) / kSolveRowBlock);
+        }
+        for (int32_t rb = 0; rb < maxrb; rb++)
+            for (int32_t s : large[l])
+                if (rb * kSolveRowBlock < P.sn_k[s]) push_task(s, rb);
+        for (int32_t s : large[l])
+            for (int32_t rb = (P.sn_k[s] + kSolveRowBlock - 1) / kSolveRowBlock; rb * kSolveRowBlock < P.sn_f[s]; rb++)
+                push_task(s, rb);
+        fsolve.push_back({SK_DF_F, deep_level(large[l]), off, (int64_t)P.df_tasks.size() / 2 - off});
     }
     for (int32_t l = P.nlevels - 1; l >= 0; l--) {
         if (!large[l].empty()) {
-            bsolve.push_back({SK_INIT_B, 0, push_list(large[l]), (int64_t)large[l].size()});
-            const int64_t off = (int64_t)P.df_tasks.size() / 2;
-            for (int32_t s : large[l]) {   // chunks bottom-up: a chunk waits only on chunks below (lower CTA ids)
-                ensure_df(s);
-                for (int32_t c = (P.sn_f[s] + kSolveRows - 1) / kSolveRows - 1; c >= 0; c--) {
-                    P.df_tasks.push_back(s);
-                    P.df_tasks.push_back(c);
-                }
+            {
+                const int64_t off = push_init(large[l]);
+                bsolve.push_back({SK_INIT_B, 0, off, (int64_t)P.df_tasks.size() / 2 - off});
             }
-            bsolve.push_back({SK_DF_B, 0, off, (int64_t)P.df_tasks.size() / 2 - off});
+            // column blocks from the last one down, round robin over the fronts
+            const int64_t off = (int64_t)P.df_tasks.size() / 2;
+            int32_t maxnb = 0;
+            for (int32_t s : large[l]) {
+                ensure_df(s);
+                maxnb = std::max(maxnb, (P.sn_k[s] + w - 1) / w);
+            }
+            for (int32_t t = 0; t < maxnb; t++)
+                for (int32_t s : large[l]) {
+                    const int32_t nb = (P.sn_k[s] + w - 1) / w;
+                    if (t < nb) push_task(s, nb - 1 - t);
+                }
+            bsolve.push_back({SK_DF_B, deep_level(large[l]), off, (int64_t)P.df_tasks.size() / 2 - off});
         }
         if (!small[l].empty()) bsolve.push_back({SK_SMALL_B, 0, push_list(small[l]), (int64_t)small[l].size()});
     }
@@ -1111,7 +1143,6 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     }   // pass
     for (const GemmProb &g : P.probs)   // the DMMA kernel stages 16-byte row pairs
         if ((g.a_off & 1) || (g.lda & 1)) return MF_ERR_STATE;
-    P.df_blk_off.assign(ns, -1);
     P.df_part_off.assign(ns, -1);
     P.dinv_off.assign(ns, -1);
     build_solve_plan(S, P, inc_local, P.fsolve, P.bsolve);
