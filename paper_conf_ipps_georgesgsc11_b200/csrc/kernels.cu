@@ -1295,61 +1295,97 @@ void launch_permute_out(const DevPlan &d, const double *xf, double *x, int64_t n
 }
 
 constexpr int kSolveThreads = 256;
-__global__ void __launch_bounds__(kSolveThreads) k_fwd_solve(DevPlan d, const int32_t *__restrict__ list,
-                                                             double *__restrict__ y) {
-    const int s = list[blockIdx.x];
+// Small supernodes (f <= kSolveSmallMax): one WARP per front, the front vector in
+// shared memory, lane l holding rows l + 32 t; the L column of the next step is
+// loaded while the current one is applied (register double buffer).
+constexpr int kSmallSolveWarps = 8, kSmallSolveR = kSolveSmallMax / 32;
+__device__ __forceinline__ void small_col_load(const double *__restrict__ col, int lo, int f, double (&c)[kSmallSolveR]) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int t = 0; t < kSmallSolveR; t++) {
+        const int i = lane + 32 * t;
+        c[t] = (i >= lo && i < f) ? col[i] : 0.0;
+    }
+}
+__global__ void __launch_bounds__(32 * kSmallSolveWarps) k_fwd_solve(DevPlan d, const int32_t *__restrict__ list,
+                                                                     int count, double *__restrict__ y) {
+    __shared__ double vsm[kSmallSolveWarps][kSolveSmallMax];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int idx = blockIdx.x * kSmallSolveWarps + warp;
+    if (idx >= count) return;
+    const int s = list[idx];
     const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
-    double *__restrict__ v = d.fv + d.fv_off[s];
     const double *__restrict__ P = d.L + d.L_off[s];
-    const int tid = threadIdx.x;
-    for (int i = tid; i < f; i += kSolveThreads) v[i] = i < k ? y[first + i] : 0.0;
-    __syncthreads();
+    double *__restrict__ vs = vsm[warp];
+    double cur[kSmallSolveR], nxt[kSmallSolveR];
+    small_col_load(P, 1, f, cur);   // column 0 (rows below the pivot), in flight during the gather
+    for (int i = lane; i < f; i += 32) vs[i] = i < k ? y[first + i] : 0.0;
+    __syncwarp();
     for (int q = d.child_ptr[s]; q < d.child_ptr[s + 1]; q++) {
         const int c = d.child_list[q];
         const int kc = d.sn_k[c], mc = d.sn_f[c] - kc;
         const int32_t *__restrict__ rel = d.relmap + d.relmap_ptr[c];
         const double *__restrict__ vc = d.fv + d.fv_off[c] + kc;
-        for (int p = tid; p < mc; p += kSolveThreads) v[rel[p]] += vc[p];
-        __syncthreads();
+        for (int p = lane; p < mc; p += 32) vs[rel[p]] += vc[p];   // rel is injective: no conflicts
+        __syncwarp();
     }
     for (int j = 0; j < k; j++) {
-        const double xj = v[j] / P[j + (int64_t)j * ld];
-        if (tid == 0) y[first + j] = xj;
-        const double *__restrict__ col = P + (int64_t)j * ld;
-        for (int i = j + 1 + tid; i < f; i += kSolveThreads) v[i] -= col[i] * xj;
-        __syncthreads();
+        if (j + 1 < k) small_col_load(P + (int64_t)(j + 1) * ld, j + 2, f, nxt);
+        const double xj = vs[j] / P[j + (int64_t)j * ld];
+        __syncwarp();   // every lane read vs[j]
+        if (lane == 0) {
+            y[first + j] = xj;
+            vs[j] = xj;
+        }
+#pragma unroll
+        for (int t = 0; t < kSmallSolveR; t++) {
+            const int i = lane + 32 * t;
+            if (i > j && i < f) vs[i] = fma(-cur[t], xj, vs[i]);
+        }
+        __syncwarp();
+#pragma unroll
+        for (int t = 0; t < kSmallSolveR; t++) cur[t] = nxt[t];
     }
+    double *__restrict__ v = d.fv + d.fv_off[s];
+    for (int i = k + lane; i < f; i += 32) v[i] = vs[i];   // the update vector the parent gathers
 }
 
-__global__ void __launch_bounds__(kSolveThreads) k_bwd_solve(DevPlan d, const int32_t *__restrict__ list,
-                                                             double *__restrict__ y,
-                                                             const int32_t *__restrict__ sn_rows,
-                                                             const int64_t *__restrict__ sn_rowptr) {
-    const int s = list[blockIdx.x];
+__global__ void __launch_bounds__(32 * kSmallSolveWarps) k_bwd_solve(DevPlan d, const int32_t *__restrict__ list,
+                                                                     int count, double *__restrict__ y,
+                                                                     const int32_t *__restrict__ sn_rows,
+                                                                     const int64_t *__restrict__ sn_rowptr) {
+    __shared__ double vsm[kSmallSolveWarps][kSolveSmallMax];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int idx = blockIdx.x * kSmallSolveWarps + warp;
+    if (idx >= count) return;
+    const int s = list[idx];
     const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
-    double *__restrict__ v = d.fv + d.fv_off[s];
     const double *__restrict__ P = d.L + d.L_off[s];
     const int32_t *__restrict__ R = sn_rows + sn_rowptr[s];
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    __shared__ double red[kSolveThreads / 32];
-    for (int i = k + tid; i < f; i += kSolveThreads) v[i] = y[R[i]];   // ancestors are final
-    __syncthreads();
+    double *__restrict__ vs = vsm[warp];
+    double cur[kSmallSolveR], nxt[kSmallSolveR];
+    if (k > 0) small_col_load(P + (int64_t)(k - 1) * ld, k, f, cur);
+    for (int i = lane; i < f; i += 32) vs[i] = i < k ? y[first + i] : y[R[i]];   // ancestors are final
+    __syncwarp();
     for (int j = k - 1; j >= 0; j--) {
-        const double *__restrict__ col = P + (int64_t)j * ld;
+        if (j > 0) small_col_load(P + (int64_t)(j - 1) * ld, j, f, nxt);
         double part = 0.0;
-        for (int i = j + 1 + tid; i < f; i += kSolveThreads) part += col[i] * v[i];
+#pragma unroll
+        for (int t = 0; t < kSmallSolveR; t++) {
+            const int i = lane + 32 * t;
+            if (i > j && i < f) part = fma(cur[t], vs[i], part);
+        }
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) part += __shfl_xor_sync(0xffffffffu, part, o);
-        if (lane == 0) red[warp] = part;
-        __syncthreads();
-        if (tid == 0) {
-            double tot = 0.0;
-            for (int w = 0; w < kSolveThreads / 32; w++) tot += red[w];
-            const double xj = (y[first + j] - tot) / col[j];
-            v[j] = xj;
+        const double xj = (vs[j] - part) / P[j + (int64_t)j * ld];
+        __syncwarp();
+        if (lane == 0) {
+            vs[j] = xj;
             y[first + j] = xj;
         }
-        __syncthreads();
+        __syncwarp();
+#pragma unroll
+        for (int t = 0; t < kSmallSolveR; t++) cur[t] = nxt[t];
     }
 }
 
@@ -1730,11 +1766,14 @@ void launch_copy_cols(const DevPlan &d, const int32_t *list, int count, const do
 }
 
 void launch_fwd_solve(const DevPlan &d, const int32_t *list, int count, double *y, cudaStream_t st) {
-    if (count > 0) k_fwd_solve<<<count, kSolveThreads, 0, st>>>(d, list, y);
+    if (count > 0)
+        k_fwd_solve<<<(count + kSmallSolveWarps - 1) / kSmallSolveWarps, 32 * kSmallSolveWarps, 0, st>>>(d, list, count, y);
 }
 void launch_bwd_solve(const DevPlan &d, const int32_t *list, int count, double *y, const int32_t *sn_rows,
                       const int64_t *sn_rowptr, cudaStream_t st) {
-    if (count > 0) k_bwd_solve<<<count, kSolveThreads, 0, st>>>(d, list, y, sn_rows, sn_rowptr);
+    if (count > 0)
+        k_bwd_solve<<<(count + kSmallSolveWarps - 1) / kSmallSolveWarps, 32 * kSmallSolveWarps, 0, st>>>(
+            d, list, count, y, sn_rows, sn_rowptr);
 }
 
 }  // namespace mf

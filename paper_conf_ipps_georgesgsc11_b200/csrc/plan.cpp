@@ -84,7 +84,7 @@ static void build_solve_plan(const Symbolic &S, Plan &P, const std::vector<char>
         for (int32_t q = P.level_ptr[l]; q < P.level_ptr[l + 1]; q++) {
             const int32_t s = P.level_list[q];
             if (!include[s]) continue;
-            (P.sn_f[s] > P.small_max ? large[l] : small[l]).push_back(s);
+            (P.sn_f[s] > std::min(P.small_max, kSolveSmallMax) ? large[l] : small[l]).push_back(s);
         }
         std::stable_sort(large[l].begin(), large[l].end(),
                          [&](int32_t a, int32_t b) { return P.sn_k[a] > P.sn_k[b]; });
