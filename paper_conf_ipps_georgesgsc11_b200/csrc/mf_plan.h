@@ -282,7 +282,9 @@ constexpr int kAsmRowBlock = 2048;   // assembly tasks split tall fronts into ro
 constexpr int kTrsmRows = 128;
 constexpr int kSmallClasses = 5;
 constexpr int kSolveRowBlock = 64;    // dataflow forward solve: rows per task (a multiple of the block width w)
-constexpr int kSolveSmallMax = 256;   // solve: fronts of order <= min(this, small_max): one warp per front
+// solve: one warp per front for f <= 128, and for f <= kSolveSmallMax when k <= kSolveSmallK
+// (tools/gpu/job_solve_small.sh: c5 6.43 -> 5.73 ms, c2 1.74 -> 1.66, c3 unchanged)
+constexpr int kSolveSmallMax = 256, kSolveSmallK = 32;
 constexpr int kSolveDeepK = 256;      // dataflow solve: levels with a front of k >= this take the deep ring
 constexpr int kSolveInitRows = 2048;  // solve init: front-vector rows per task (kernels.cu kInitRows)
 

@@ -80,11 +80,20 @@ static void build_solve_plan(const Symbolic &S, Plan &P, const std::vector<char>
     (void)S;
     const int w = P.w;
     std::vector<std::vector<int32_t>> large(P.nlevels), small(P.nlevels);
+    static const int solve_small = [] {   // MF_SOLVE_SMALL: tuning override (<= kSolveSmallMax)
+        const char *e = getenv("MF_SOLVE_SMALL");
+        return e ? std::max(1, std::min(kSolveSmallMax, atoi(e))) : kSolveSmallMax;
+    }();
+    static const int solve_small_k = [] {   // MF_SOLVE_SMALL_K: above order 128, only fronts of k <= this
+        const char *e = getenv("MF_SOLVE_SMALL_K");
+        return e ? atoi(e) : kSolveSmallK;
+    }();
     for (int32_t l = 0; l < P.nlevels; l++) {
         for (int32_t q = P.level_ptr[l]; q < P.level_ptr[l + 1]; q++) {
             const int32_t s = P.level_list[q];
             if (!include[s]) continue;
-            (P.sn_f[s] > std::min(P.small_max, kSolveSmallMax) ? large[l] : small[l]).push_back(s);
+            const bool sm = P.sn_f[s] <= 128 || (P.sn_f[s] <= solve_small && P.sn_k[s] <= solve_small_k);
+            (sm ? small[l] : large[l]).push_back(s);
         }
         std::stable_sort(large[l].begin(), large[l].end(),
                          [&](int32_t a, int32_t b) { return P.sn_k[a] > P.sn_k[b]; });
