@@ -1417,6 +1417,23 @@ constexpr int kDfRB = 64;            // rows per forward task / per backward sla
 constexpr int kDfBuf = MF_DF_BUF;    // register ring: blocks (forward) / slabs (backward) in flight
 constexpr int kInitRows = kSolveInitRows;   // rows of a front vector per init task
 
+// First p in [0, n) with rel[p] >= key (rel increasing; n if none), by the whole CTA
+// of kSolveThreads in 256-way rounds (two dependent loads for n <= 65536 instead of
+// a log2(n) chain).  Uniform call.
+__device__ __forceinline__ int lower_bound_cta(const int32_t *__restrict__ rel, int n, int key) {
+    const int t = threadIdx.x;
+    int lo = 0, hi = n;   // the answer lies in [lo, hi]
+    while (hi - lo > kSolveThreads) {
+        const int len = hi - lo;
+        const int bt = lo + (int)((int64_t)t * len / kSolveThreads);
+        const int c = __syncthreads_count(t > 0 && __ldg(rel + bt - 1) < key);
+        hi = lo + (int)((int64_t)(c + 1) * len / kSolveThreads);
+        lo = lo + (int)((int64_t)c * len / kSolveThreads);
+    }
+    const int p = lo + t;
+    return lo + __syncthreads_count(p < hi && __ldg(rel + p) < key);
+}
+
 // ---- large supernodes: v = [y(cols); 0] + the children's update vectors, one task
 // per (supernode, 2048-row part); a part finds each child's entries that land in it
 // by binary search (rel is increasing), children in a fixed order: deterministic.
@@ -1436,7 +1453,8 @@ __global__ void __launch_bounds__(kSolveThreads) k_fsolve_init(DevPlan d, const 
         const int kc = d.sn_k[c], mc = d.sn_f[c] - kc;
         const int32_t *__restrict__ rel = d.relmap + d.relmap_ptr[c];
         const double *__restrict__ vc = d.fv + d.fv_off[c] + kc;
-        const int lo = lower_bound_rel(rel, 0, mc, p0), hi = lower_bound_rel(rel, lo, mc, p1);
+        const bool whole = p0 == 0 && p1 == f;   // one part: no search
+        const int lo = whole ? 0 : lower_bound_cta(rel, mc, p0), hi = whole ? mc : lower_bound_cta(rel, mc, p1);
         for (int p = lo + threadIdx.x; p < hi; p += kSolveThreads) v[rel[p]] += vc[p];
     }
 }
