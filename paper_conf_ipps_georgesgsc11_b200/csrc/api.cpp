@@ -455,8 +455,9 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     UP(&c->d_tiles, P.tiles);
     UP(&c->d_solve_list, P.solve_list);
     UP(&c->d_df_tasks, P.df_tasks);
-    int64_t *df_part_off = nullptr, *dinv_off = nullptr;
+    int64_t *df_part_off = nullptr, *df_seg_off = nullptr, *dinv_off = nullptr;
     UP(&df_part_off, P.df_part_off);
+    UP(&df_seg_off, P.df_seg_off);
     UP(&dinv_off, P.dinv_off);
     UP(&c->d_dinv_tasks, P.dinv_tasks);
     int32_t *ea_qs = nullptr;
@@ -526,6 +527,7 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     d.bvidx = bvidx;
     d.perm = perm_d;
     d.df_part_off = df_part_off;
+    d.df_seg_off = df_seg_off;
     d.dinv_off = dinv_off;
     d.ea_qs = ea_qs;
     d.fuse_ea = P.fuse_ea;
@@ -549,6 +551,9 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     }
     if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.df_nparts, 1) * sizeof(double))) != MF_OK) return r;
     d.df_parts = (double *)p;
+    if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.df_nseg_words, 1) * sizeof(double))) != MF_OK) return r;
+    d.df_seg = (double *)p;
+    launch_fill_pending(d.df_seg, P.df_nseg_words, c->stream);   // tail-segment partials: not yet written
     if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.dinv_words, 1) * sizeof(double))) != MF_OK) return r;
     d.dinv = (double *)p;
     c->dinv_stale = true;
@@ -1054,6 +1059,9 @@ int ensure_slots(mf_ctx *c, int ns) {
         q.d.fv = (double *)p;
         if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.df_nparts, 1) * sizeof(double)))) return r;
         q.d.df_parts = (double *)p;
+        if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.df_nseg_words, 1) * sizeof(double)))) return r;
+        q.d.df_seg = (double *)p;
+        launch_fill_pending(q.d.df_seg, P.df_nseg_words, c->stream);
         if ((r = dev_alloc(c, &p, tk_words * sizeof(unsigned)))) return r;
         CK(cudaMemsetAsync(p, 0, tk_words * sizeof(unsigned), c->stream));
         q.tickets = (unsigned *)p;

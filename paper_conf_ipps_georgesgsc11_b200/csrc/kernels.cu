@@ -1407,6 +1407,13 @@ __device__ __forceinline__ double wait_value(const double *p) {
     return v;
 }
 __device__ __forceinline__ double pending_value() { return __longlong_as_double((long long)kSolvePending); }
+__global__ void k_fill_pending(double *__restrict__ p, int64_t n) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        p[i] = pending_value();
+}
+void launch_fill_pending(double *p, int64_t n, cudaStream_t st) {
+    if (n > 0) k_fill_pending<<<(unsigned)std::min<int64_t>((n + 255) / 256, 2048), 256, 0, st>>>(p, n);
+}
 
 #ifndef MF_DF_BUF
 #define MF_DF_BUF 2
@@ -1416,6 +1423,7 @@ constexpr int kDfThreads = 256;      // dataflow solve CTA: 64 rows x 4 groups o
 constexpr int kDfRB = 64;            // rows per forward task / per backward slab
 constexpr int kDfBuf = MF_DF_BUF;    // register ring: blocks (forward) / slabs (backward) in flight
 constexpr int kInitRows = kSolveInitRows;   // rows of a front vector per init task
+constexpr int kBsSegSlabs = kSolveSegSlabs;  // backward: tail slabs per segment task
 
 // First p in [0, n) with rel[p] >= key (rel increasing; n if none), by the whole CTA
 // of kSolveThreads in 256-way rounds (two dependent loads for n <= 65536 instead of
@@ -1660,30 +1668,52 @@ __device__ __forceinline__ void bsolve_cols_task(const DevPlan &d, const int32_t
     __shared__ double red[8][16];
     __shared__ double tv[kSW];
     __shared__ double rx[4][kSW];
-    const int s = tasks[2 * task], b = tasks[2 * task + 1];
+    const int s = tasks[2 * task], b = tasks[2 * task + 1] & 0xffff, seg = tasks[2 * task + 1] >> 16;
     const int k = d.sn_k[s], f = d.sn_f[s], ld = d.sn_ld[s], first = d.sn_first[s];
     const double *__restrict__ P = d.L + d.L_off[s];
     const double *__restrict__ v = d.fv + d.fv_off[s];
     double *__restrict__ xp = d.df_parts + d.df_part_off[s];
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, i = tid & 63, g = tid >> 6;
     const int j0 = b * w, we = min(w, k - j0), rlo = j0 + we;   // rows below the block
-    {
+    // slabs of 64 rows: the pure tail ones (rows >= k, from slab T0 on), then the pivot
+    // ones from slab ktop (holding row k - 1; it may also hold rows >= k) down to the
+    // one holding row rlo.  A tall tail is cut into segments of kBsSegSlabs slabs, each
+    // a task of its own (seg >= 1, lower tickets, never waits) that publishes the 64
+    // column partials of its rows; the chain task (seg = 0) then streams no tail.
+    const int ktop = (k - 1) / kDfRB, T0 = ktop + 1, nsl = (f + kDfRB - 1) / kDfRB;
+    const int ntail = max(0, nsl - T0), nseg = ntail > kBsSegSlabs ? (ntail + kBsSegSlabs - 1) / kBsSegSlabs : 0;
+    double *__restrict__ segp = nseg ? d.df_seg + d.df_seg_off[s] + (int64_t)b * nseg * kSW : nullptr;
+    int t0, nt, np;
+    if (seg > 0) {
+        t0 = T0 + (seg - 1) * kBsSegSlabs;
+        nt = min(kBsSegSlabs, nsl - t0);
+        np = 0;
+    } else {
+        t0 = T0;
+        nt = nseg ? 0 : ntail;
+        np = max(0, ktop - rlo / kDfRB + 1);
+    }
+    double yb = 0.0;
+    if (seg == 0) {
         const double *__restrict__ M = d.dinv + d.dinv_off[s] + (int64_t)b * kSW * kSW;
         for (int q = tid; q < kSW * kSW; q += kDfThreads) Ms[(q >> 6) + (q & 63) * kSLD] = __ldg(M + q);
+        if (tid < we) yb = y[first + j0 + tid];   // forward result of the block (this task rewrites it)
     }
-    const double yb = (tid < we) ? y[first + j0 + tid] : 0.0;   // forward result of the block (this task rewrites it)
-    // slabs: the tail slabs (rows >= k only) ascending, then the pivot slabs from the
-    // one holding row k - 1 down to the one holding row rlo (the first of them may also
-    // hold rows >= k).  The last block (rlo >= k) has tail slabs only, from rlo's.
-    const int ktop = (k - 1) / kDfRB, np = rlo < k ? ktop - rlo / kDfRB + 1 : 0;
-    const int kt0 = np > 0 ? ktop + 1 : rlo / kDfRB, nsl = (f + kDfRB - 1) / kDfRB;
-    const int nt = max(0, nsl - kt0);
     const int ns = nt + np;
-    auto slab_row = [&](int q) { return (q < nt ? kt0 + q : ktop - (q - nt)) * kDfRB + i; };
+    auto slab_row = [&](int q) { return (q < nt ? t0 + q : ktop - (q - nt)) * kDfRB + i; };
     double Lb[NBUF][16];
 #pragma unroll
     for (int q = 0; q < NBUF; q++)
         if (q < ns) bsolve_load(P, ld, f, j0, we, rlo, slab_row(q), Lb[q]);
+    // the tail segments' partials (lower tickets: they are done or nearly so) -- read
+    // now, while the chain is still above this block, not on its critical path
+    double segsum = 0.0;
+    if (seg == 0 && tid < we)
+        for (int q = 0; q < nseg; q++) {
+            double *pq = segp + (int64_t)q * kSW + tid;
+            segsum += wait_value(pq);
+            __stcg(pq, pending_value());   // re-armed for the next solve (this task is its only reader)
+        }
     double acc[16];
 #pragma unroll
     for (int u = 0; u < 16; u++) acc[u] = 0.0;
@@ -1702,9 +1732,16 @@ __device__ __forceinline__ void bsolve_cols_task(const DevPlan &d, const int32_t
     warp_reduce_scatter16(acc);   // lane l: value (l >> 1) & 15 over this warp's 32 rows
     if ((lane & 1) == 0) red[warp][lane >> 1] = acc[0];
     __syncthreads();
-    if (tid < kSW) {   // column c = 16 g' + u': the two warps of group g'
+    if (seg > 0) {   // a tail segment: publish its column partials
+        if (tid < we) {
+            const int gc = tid >> 4, u = tid & 15;
+            __stcg(segp + (int64_t)(seg - 1) * kSW + tid, red[2 * gc][u] + red[2 * gc + 1][u]);
+        }
+        return;
+    }
+    if (tid < kSW) {   // column c = 16 g' + u': the two warps of group g', then the tail segments in order
         const int gc = tid >> 4, u = tid & 15;
-        tv[tid] = tid < we ? yb - (red[2 * gc][u] + red[2 * gc + 1][u]) : 0.0;
+        tv[tid] = tid < we ? yb - ((red[2 * gc][u] + red[2 * gc + 1][u]) + segsum) : 0.0;
     }
     __syncthreads();
     double a = 0.0;

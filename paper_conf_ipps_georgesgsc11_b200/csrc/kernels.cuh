@@ -28,6 +28,8 @@ struct DevPlan {
     unsigned *panel_flag;    // per supernode: kPanelFlags dataflow-panel tile flags
     double *df_parts;        // dataflow backward sweep: published x of the pivot columns (value = flag)
     const int64_t *df_part_off;
+    double *df_seg;          // dataflow backward sweep: column partials of the tail segments (value = flag)
+    const int64_t *df_seg_off;
     double *dinv;            // dataflow solve: inverses of the 64 x 64 diagonal blocks (solve setup)
     const int64_t *dinv_off; // per supernode: word offset of its blocks in dinv (-1: none)
     const int32_t *ea_qs;    // fused extend-add: tile-row start tables of the syrk problems
@@ -74,6 +76,7 @@ void launch_bwd_solve(const DevPlan &d, const int32_t *list, int count, double *
 // solve setup: inverses of the 64 x 64 diagonal blocks of the dataflow-solved supernodes
 void launch_diag_inv(const DevPlan &d, const int32_t *tasks, int64_t count, int w, cudaStream_t st);
 // (supernode, 2048-row part) pairs: front vectors of the large supernodes, children gathered
+void launch_fill_pending(double *p, int64_t n, cudaStream_t st);   // dataflow-solve slots: not yet written
 void launch_fsolve_init(const DevPlan &d, const int32_t *tasks, int64_t count, double *y, cudaStream_t st);
 // deep = 1: the levels with multi-block fronts (register ring of MF_DF_BUF blocks, 1 CTA / SM)
 void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, int deep, double *y,

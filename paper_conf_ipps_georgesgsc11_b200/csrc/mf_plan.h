@@ -243,6 +243,8 @@ struct Plan {
     std::vector<int32_t> df_tasks;                   // dataflow solve: (front, chunk) pairs
     std::vector<int64_t> df_part_off;                // per supernode: base of its backward x slots (k words)
     int64_t df_nparts = 0;                           // fp64 x-slot words
+    std::vector<int64_t> df_seg_off;                 // per supernode: backward tail-segment partials (-1: none)
+    int64_t df_nseg_words = 0;
     // inverses of the 64 x 64 diagonal blocks of the dataflow-solved supernodes (solve setup,
     // computed once per factorization by the first solve): per supernode the word offset of
     // its ceil(k / 64) column-major 64 x 64 blocks; (supernode, block) task pairs
@@ -286,7 +288,8 @@ constexpr int kSolveRowBlock = 64;    // dataflow forward solve: rows per task (
 // (tools/gpu/job_solve_small.sh: c5 6.43 -> 5.73 ms, c2 1.74 -> 1.66, c3 unchanged)
 constexpr int kSolveSmallMax = 256, kSolveSmallK = 32;
 constexpr int kSolveDeepK = 256;      // dataflow solve: levels with a front of k >= this take the deep ring
-constexpr int kSolveInitRows = 2048;  // solve init: front-vector rows per task (kernels.cu kInitRows)
+constexpr int kSolveInitRows = 2048;
+constexpr int kSolveSegSlabs = 16;    // dataflow backward solve: 64-row tail slabs per segment task  // solve init: front-vector rows per task (kernels.cu kInitRows)
 
 int build_plan(const Symbolic &S, const Options &opt, Plan &P);
 

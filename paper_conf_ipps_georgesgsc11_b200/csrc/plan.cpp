@@ -106,6 +106,11 @@ static void build_solve_plan(const Symbolic &S, Plan &P, const std::vector<char>
     // dataflow solve of the large supernodes (kernels.cu): forward tasks = 64-row
     // blocks, backward tasks = w-column blocks; x slots of the backward sweep (one per
     // pivot column) and the inverses of the diagonal blocks
+    auto bs_nseg = [&](int32_t s) {   // backward tail segments per column block (kernels.cu bsolve_cols_task)
+        const int32_t ktop = (P.sn_k[s] - 1) / kSolveRowBlock, nsl = (P.sn_f[s] + kSolveRowBlock - 1) / kSolveRowBlock;
+        const int32_t ntail = std::max(0, nsl - ktop - 1);
+        return ntail > kSolveSegSlabs ? (ntail + kSolveSegSlabs - 1) / kSolveSegSlabs : 0;
+    };
     auto ensure_df = [&](int32_t s) {
         if (P.df_part_off[s] >= 0) return;
         const int64_t nb = (P.sn_k[s] + w - 1) / w;
@@ -114,6 +119,10 @@ static void build_solve_plan(const Symbolic &S, Plan &P, const std::vector<char>
         for (int32_t b = 0; b < nb; b++) P.dinv_tasks.insert(P.dinv_tasks.end(), {s, b});
         P.df_part_off[s] = P.df_nparts;
         P.df_nparts += P.sn_k[s];
+        if (const int32_t ns = bs_nseg(s)) {
+            P.df_seg_off[s] = P.df_nseg_words;
+            P.df_nseg_words += nb * ns * 64;
+        }
     };
     // the deep register ring (1 CTA / SM) for levels whose largest front has several
     // blocks; the shallow one (3 CTAs / SM) for levels of small fronts
@@ -161,13 +170,20 @@ static void build_solve_plan(const Symbolic &S, Plan &P, const std::vector<char>
                 const int64_t off = push_init(large[l]);
                 bsolve.push_back({SK_INIT_B, 0, off, (int64_t)P.df_tasks.size() / 2 - off});
             }
-            // column blocks from the last one down, round robin over the fronts
+            // the tail segments first (they wait for nothing), then the column blocks from
+            // the last one down, round robin over the fronts
             const int64_t off = (int64_t)P.df_tasks.size() / 2;
             int32_t maxnb = 0;
             for (int32_t s : large[l]) {
                 ensure_df(s);
                 maxnb = std::max(maxnb, (P.sn_k[s] + w - 1) / w);
             }
+            for (int32_t t = 0; t < maxnb; t++)
+                for (int32_t s : large[l]) {
+                    const int32_t nb = (P.sn_k[s] + w - 1) / w, ns = bs_nseg(s);
+                    if (t < nb)
+                        for (int32_t q = 1; q <= ns; q++) push_task(s, (nb - 1 - t) | (q << 16));
+                }
             for (int32_t t = 0; t < maxnb; t++)
                 for (int32_t s : large[l]) {
                     const int32_t nb = (P.sn_k[s] + w - 1) / w;
@@ -1153,6 +1169,7 @@ int build_plan(const Symbolic &S, const Options &opt, Plan &P) {
     for (const GemmProb &g : P.probs)   // the DMMA kernel stages 16-byte row pairs
         if ((g.a_off & 1) || (g.lda & 1)) return MF_ERR_STATE;
     P.df_part_off.assign(ns, -1);
+    P.df_seg_off.assign(ns, -1);
     P.dinv_off.assign(ns, -1);
     build_solve_plan(S, P, inc_local, P.fsolve, P.bsolve);
     build_solve_plan(S, P, inc_top_solve, P.fsolve_top, P.bsolve_top);
