@@ -231,33 +231,37 @@ __global__ void __launch_bounds__(32 * kTinyWarps, TF <= 16 ? 8 : 4)
     for (int c = 0; c < TF; c++) a[c] = lane < TF ? F[lane + c * kTinyLD] : 0.0;
 #pragma unroll
     for (int j = 0; j < TF; j++) {
-        if (j < k) {
-            const double dj = __shfl_sync(0xffffffffu, a[j], j);
-            const double inv = rsqrt(dj);
-            if (lane == j) {
-                note_pivot(d, dj, first + j);
-                a[j] = dj * inv;
-            } else if (lane > j) {
-                a[j] *= inv;
-            }
+        if (j >= k) break;   // (uniform) the instruction stream stops at the front's k and f,
+        const double dj = __shfl_sync(0xffffffffu, a[j], j);   // not at the class bound TF
+        const double inv = rsqrt(dj);
+        if (lane == j) {
+            note_pivot(d, dj, first + j);
+            a[j] = dj * inv;
+        } else if (lane > j) {
+            a[j] *= inv;
+        }
 #pragma unroll
-            for (int c = j + 1; c < TF; c++) {
-                const double lc = __shfl_sync(0xffffffffu, a[j], c);
-                if (lane >= c && c < f) a[c] -= a[j] * lc;
-            }
+        for (int c = j + 1; c < TF; c++) {
+            if (c >= f) break;
+            const double lc = __shfl_sync(0xffffffffu, a[j], c);
+            if (lane >= c) a[c] -= a[j] * lc;
         }
     }
     if (lane < f) {
         double *__restrict__ P = d.L + d.L_off[s];
         const int ld = d.sn_ld[s];
 #pragma unroll
-        for (int j = 0; j < TF; j++)
-            if (j < k) P[lane + (int64_t)j * ld] = lane >= j ? a[j] : 0.0;
+        for (int j = 0; j < TF; j++) {
+            if (j >= k) break;
+            P[lane + (int64_t)j * ld] = lane >= j ? a[j] : 0.0;
+        }
         if (m > 0) {
             double *__restrict__ Us = d.U + d.U_off[s];
 #pragma unroll
-            for (int c = 0; c < TF; c++)
-                if (c >= k && c < f && lane >= c) Us[upk(lane - k, c - k, m)] = a[c];
+            for (int c = 0; c < TF; c++) {
+                if (c >= f) break;
+                if (c >= k && lane >= c) Us[upk(lane - k, c - k, m)] = a[c];
+            }
         }
     }
 }
