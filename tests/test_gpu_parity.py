@@ -122,6 +122,8 @@ def test_variant_paths_agree(mf, small_max, w):
     A, p = grid("27pt", (14, 13, 12))
     S, sym, panels = factor_both(mf, A, p, small_front_max=small_max, panel_w=w)
     check_panels(S, sym, panels)
+    b = spmv(A, G.rhs(A.n, 0))   # the solve's dataflow tasks with w-column blocks (w | 64)
+    assert backward_error(A, S.solve(b), b) <= TOL_BE
 
 
 @pytest.mark.parametrize("n", [1, 2, 63, 64, 65, 200, 1000, 2500])
@@ -429,3 +431,23 @@ def test_solve_nrhs(mf):
     Bt = torch.from_numpy(np.ascontiguousarray(B.T)).cuda()   # (nrhs, n) rows = columns of B
     Xt = S.solve_nrhs(Bt)
     np.testing.assert_array_equal(Xt.cpu().numpy().T, X)
+
+
+def test_solve_tall_tails(mf):
+    """Dataflow solve with fronts whose update part spans more than 16 slabs of 64
+    rows (the backward tail-segment tasks, kernels.cu bsolve_cols_task) and with a
+    several-chunk init: backward stable, and nrhs bitwise equal to single solves."""
+    A, p = grid("7pt", (40, 40, 40))
+    S = mf.Solver()
+    S.analyze(A.n, A.colptr, A.rowind, p)
+    S.factor(A.values)
+    sn = S.supernodes()
+    k = np.diff(sn["sn_first"])
+    f = np.diff(sn["sn_rowptr"])
+    assert (f - k > 16 * 64).any() and (f > 2048).any()
+    B = np.asfortranarray(np.stack([spmv(A, G.rhs(A.n, r)) for r in range(3)], axis=1))
+    X = S.solve_nrhs(B)
+    for r in range(3):
+        x = S.solve(np.ascontiguousarray(B[:, r]))
+        assert backward_error(A, x, B[:, r]) <= TOL_BE
+        np.testing.assert_array_equal(X[:, r], x)
