@@ -770,6 +770,22 @@ static_assert(64 * kPLD <= kPanelRingWords, "the L_bb tile aliases the staging r
 
 __device__ __forceinline__ int panel_tri(int c, int b) { return c * (c + 1) / 2 + b; }
 
+// Phase timeline of the dataflow panel (tools/ubench/panel_timeline.cu defines
+// MF_PANEL_TL; compiled out otherwise): %globaltimer at fixed event slots per task.
+#ifdef MF_PANEL_TL
+__device__ unsigned long long *g_panel_tl;
+#define PANEL_TL(task, ev)                                                                   \
+    do {                                                                                     \
+        if (threadIdx.x == 0 && g_panel_tl) {                                                \
+            unsigned long long t_;                                                           \
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));                           \
+            g_panel_tl[(int64_t)(task) * 64 + (ev)] = t_;                                    \
+        }                                                                                    \
+    } while (0)
+#else
+#define PANEL_TL(task, ev) do { } while (0)
+#endif
+
 // acc(64 x 64 tile; this warp's 32 x 32 fragment) -= A B^T with A = rows [ra0, ra0+64),
 // B = rows [rb0, rb0+64), columns [kc0, kc0 + K) of the panel Pn (column-major, ld);
 // rows >= arows / brows read as zero.  K is a multiple of 16.
@@ -925,7 +941,7 @@ __device__ __forceinline__ void upd_block8(double *A, int I, int J, int s0) {
 // updated with DMMA (K = 8).  Look-ahead: warp 0 updates the next block column
 // and its lane 0 factors the next pivot block while warps 1-3 update the rest.
 __device__ __forceinline__ void panel_potrf_dmma(const DevPlan &d, double *A, double *sinv, int R, int we,
-                                                 int first_col) {
+                                                 int first_col, int tl_task = 0) {
     constexpr int SB = 8;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int nrb = (R + 7) / 8, ncb = (we + 7) / 8;
@@ -956,6 +972,7 @@ __device__ __forceinline__ void panel_potrf_dmma(const DevPlan &d, double *A, do
                 if (q < nb) A[(s0 + q) * kPLD + r] = x[q];
         }
         __syncthreads();
+        PANEL_TL(tl_task, 44 + 2 * st);
         if (st + 1 < ncb) {
             const int J1 = st + 1;
             if (warp == 0) {
@@ -971,6 +988,7 @@ __device__ __forceinline__ void panel_potrf_dmma(const DevPlan &d, double *A, do
             }
         }
         __syncthreads();
+        PANEL_TL(tl_task, 45 + 2 * st);
     }
 }
 
@@ -1079,13 +1097,16 @@ __device__ __forceinline__ void panel_task(const DevPlan &d, const int32_t *__re
     for (int b = 0; b < nsteps; b++) {
         const int cb0 = j0 + 64 * b, wb = min(64, k - cb0);
         double acc[4][4][2];
+        PANEL_TL(task, 6 * b);
         panel_frag_load(acc, Pn, ld, r0, rows, cb0, wb);
         if (b > 0) {
             wait_flag(F + panel_tri(b, b - 1), tag);   // band tiles (b, 0..b-1) are final
             panel_tile_mma(acc, ring, Pn, ld, r0, rows, cb0, min(64, f - cb0), j0, 64 * b);
         }
         panel_frag_to_smem(acc, Xs);
+        PANEL_TL(task, 6 * b + 1);
         wait_flag(F + panel_tri(b, b), tag);           // L_bb is final
+        PANEL_TL(task, 6 * b + 2);
         {
             const double *__restrict__ D = Pn + (int64_t)cb0 * ld + cb0;
             for (int q = tid; q < 32 * 64; q += kPanelThreads) {
@@ -1108,6 +1129,7 @@ __device__ __forceinline__ void panel_task(const DevPlan &d, const int32_t *__re
             __syncthreads();
         }
         panel_trsm(Xs, ring, inv, wb);
+        PANEL_TL(task, 6 * b + 3);
         for (int q = tid; q < 64 * 64; q += kPanelThreads) {
             const int i = q & 63, j = q >> 6;
             if (i < rows && j < wb) Pn[(r0 + i) + (int64_t)(cb0 + j) * ld] = Xs[i + j * kPLD];
@@ -1127,8 +1149,10 @@ __device__ __forceinline__ void panel_task(const DevPlan &d, const int32_t *__re
 #pragma unroll
                 for (int t = 0; t < 9; t++) dmma(dacc[t][0], dacc[t][1], t <= warp ? a0 : a1, bj[t]);
             }
+            PANEL_TL(task, 6 * b + 4);
             panel_publish(F + panel_tri(c, b), tag);   // X(c,b) is stored: band tile final (+ CTA barrier:
                                                        // Xs / ring are rewritten by the next step)
+            PANEL_TL(task, 6 * b + 5);
         } else {
             __syncthreads();   // Xs / ring are rewritten by the next step
         }
@@ -1143,12 +1167,15 @@ __device__ __forceinline__ void panel_task(const DevPlan &d, const int32_t *__re
             for (int e = 0; e < 2; e++) Xs[I * 8 + gq + (J * 8 + 2 * tq + e) * kPLD] = dacc[t][e];
         }
         __syncthreads();
-        panel_potrf_dmma(d, Xs, inv, rows, we, d.sn_first[s] + r0);
+        PANEL_TL(task, 60);
+        panel_potrf_dmma(d, Xs, inv, rows, we, d.sn_first[s] + r0, task);
+        PANEL_TL(task, 61);
         for (int q = tid; q < 64 * 64; q += kPanelThreads) {
             const int i = q & 63, j = q >> 6;
             if (i < rows && j < we && i >= j) Pn[(r0 + i) + (int64_t)(r0 + j) * ld] = Xs[i + j * kPLD];
         }
         panel_publish(F + panel_tri(c, c), tag);
+        PANEL_TL(task, 62);
     }
 }
 
