@@ -545,9 +545,9 @@ int mf_analyze(mf_ctx *c, int64_t n, const int64_t *colptr, const int32_t *rowin
     {   // one counter pair per launch slot of every program (factor local / top, solves)
         const size_t slots = P.program.size() + P.program_top.size() + P.fsolve.size() + P.bsolve.size() +
                              P.fsolve_top.size() + P.bsolve_top.size() + 1;
-        if ((r = dev_alloc(c, &p, 2 * slots * sizeof(unsigned))) != MF_OK) return r;
+        if ((r = dev_alloc(c, &p, kTkWords * slots * sizeof(unsigned))) != MF_OK) return r;
         c->d_tickets = (unsigned *)p;
-        CK(cudaMemsetAsync(p, 0, 2 * slots * sizeof(unsigned), c->stream));
+        CK(cudaMemsetAsync(p, 0, kTkWords * slots * sizeof(unsigned), c->stream));
     }
     if ((r = dev_alloc(c, &p, (size_t)std::max<int64_t>(P.df_nparts, 1) * sizeof(double))) != MF_OK) return r;
     d.df_parts = (double *)p;
@@ -625,7 +625,7 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
     const Plan &P = c->P;
     const DevPlan &d = c->d;
     cudaStream_t st = c->stream;
-    unsigned *tk0 = c->d_tickets + 2 * (&prog == &P.program ? 0 : P.program.size());   // this program's slots
+    unsigned *tk0 = c->d_tickets + kTkWords * (&prog == &P.program ? 0 : P.program.size());   // this program's slots
     auto issue = [&](const double *v, bool with_events) -> int {
         if (with_init) launch_init_failed(c->d_failed, st);
         // subtree branches run on their own streams (forked after the init launch,
@@ -689,11 +689,11 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
                                       L.count > 0 ? L.flops / (2.0 * kTileM * kTileN * L.count) : 0.0, st);
                     break;
                 case KC_PANEL:
-                    launch_panel(d, c->d_panel + 2 * L.off, L.count, L.param, (int)L.count2, tk0 + 2 * li, st);
+                    launch_panel(d, c->d_panel + 2 * L.off, L.count, L.param, (int)L.count2, tk0 + kTkWords * li, st);
                     break;
                 case KC_LEAF:
                     launch_leaf(d, c->d_large + L.off, (int)L.count, c->d_trsm + 2 * L.off2, L.count2, L.param, P.w,
-                                tk0 + 2 * li, st);
+                                tk0 + kTkWords * li, st);
                     break;
                 default: return MF_ERR_STATE;   // exchange points are handled by run_with_exchanges
             }
@@ -895,20 +895,26 @@ void run_solve_program(mf_ctx *c, const std::vector<SolveLaunch> &prog, const De
         if (q == &prog) break;
         base += q->size();
     }
-    unsigned *tk0 = tickets + 2 * base;
+    unsigned *tk0 = tickets + kTkWords * base;
     for (size_t li = 0; li < prog.size(); li++) {
         const SolveLaunch &L = prog[li];
         switch (L.kind) {
             case SK_SMALL_F: launch_fwd_solve(d, c->d_solve_list + L.off, (int)L.count, y, st); break;
             case SK_INIT_F: launch_fsolve_init(d, c->d_df_tasks + 2 * L.off, L.count, y, st); break;
-            case SK_DF_F: launch_fsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, L.j0, y, tk0 + 2 * li, st); break;
-            case SK_SMALL_B:
-                launch_bwd_solve(d, c->d_solve_list + L.off, (int)L.count, y, c->d_sn_rows, c->d_sn_rowptr, st);
-                break;
             case SK_INIT_B:
                 launch_bsolve_init(d, c->d_df_tasks + 2 * L.off, L.count, y, c->d_sn_rows, c->d_sn_rowptr, st);
                 break;
-            case SK_DF_B: launch_bsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, P.w, L.j0, y, tk0 + 2 * li, st); break;
+            case SK_DF_F:
+                launch_fsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, c->d_df_tasks + 2 * L.off2, L.count2, P.w, L.j0,
+                                 y, tk0 + kTkWords * li, st);
+                break;
+            case SK_SMALL_B:
+                launch_bwd_solve(d, c->d_solve_list + L.off, (int)L.count, y, c->d_sn_rows, c->d_sn_rowptr, st);
+                break;
+            case SK_DF_B:
+                launch_bsolve_df(d, c->d_df_tasks + 2 * L.off, L.count, c->d_df_tasks + 2 * L.off2, L.count2, P.w, L.j0,
+                                 y, c->d_sn_rows, c->d_sn_rowptr, tk0 + kTkWords * li, st);
+                break;
         }
     }
 }
@@ -1044,7 +1050,7 @@ namespace {
 int ensure_slots(mf_ctx *c, int ns) {
     const Plan &P = c->P;
     const int64_t n = c->S.n;
-    const size_t tk_words = 2 * (P.program.size() + P.program_top.size() + P.fsolve.size() + P.bsolve.size() +
+    const size_t tk_words = kTkWords * (P.program.size() + P.program_top.size() + P.fsolve.size() + P.bsolve.size() +
                                  P.fsolve_top.size() + P.bsolve_top.size() + 1);
     while ((int)c->slots.size() < ns) {
         SolveSlot q;

@@ -690,6 +690,7 @@ __device__ __forceinline__ void drop_ticket(unsigned *tk) {
     if (threadIdx.x == 0 && atomicAdd(tk + 1, 1u) == gridDim.x - 1) {
         tk[0] = 0u;
         tk[1] = 0u;
+        tk[2] = 0u;   // the fused-init count of the solve launches (kTkWords)
         __threadfence();
     }
 }
@@ -1476,9 +1477,9 @@ __device__ __forceinline__ int lower_bound_cta(const int32_t *__restrict__ rel, 
 // ---- large supernodes: v = [y(cols); 0] + the children's update vectors, one task
 // per (supernode, 2048-row part); a part finds each child's entries that land in it
 // by binary search (rel is increasing), children in a fixed order: deterministic.
-__global__ void __launch_bounds__(kSolveThreads) k_fsolve_init(DevPlan d, const int32_t *__restrict__ tasks,
-                                                               double *__restrict__ y) {
-    const int s = tasks[2 * blockIdx.x], part = tasks[2 * blockIdx.x + 1];
+__device__ __forceinline__ void fsolve_init_task(const DevPlan &d, const int32_t *__restrict__ tasks,
+                                                 double *__restrict__ y, const int task) {
+    const int s = tasks[2 * task], part = tasks[2 * task + 1];
     const int k = d.sn_k[s], f = d.sn_f[s], first = d.sn_first[s];
     const int p0 = part * kInitRows, p1 = min(f, p0 + kInitRows);
     double *__restrict__ v = d.fv + d.fv_off[s];
@@ -1498,12 +1499,43 @@ __global__ void __launch_bounds__(kSolveThreads) k_fsolve_init(DevPlan d, const 
     }
 }
 
+__global__ void __launch_bounds__(kSolveThreads) k_fsolve_init(DevPlan d, const int32_t *__restrict__ tasks,
+                                                               double *__restrict__ y) {
+    fsolve_init_task(d, tasks, y, blockIdx.x);
+}
+void launch_fsolve_init(const DevPlan &d, const int32_t *tasks, int64_t count, double *y, cudaStream_t st) {
+    if (count > 0) k_fsolve_init<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, y);
+}
+
+// The init tasks of a level with few of them run in the level's dataflow launch
+// (SolveLaunch.off2; levels of many small fronts keep a launch of their own, whose
+// light CTAs cover them in fewer waves than the dataflow kernel's):
+// they take the lowest tickets, then count themselves done in tk[2]; every dataflow
+// task of the launch waits for that count (thread 0 polls) before it touches a front
+// vector, a y / x slot of the level or a partial -- its L loads are issued before.
+__device__ __forceinline__ void init_done(unsigned *cnt) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        atomicAdd(cnt, 1u);
+    }
+}
+__device__ __forceinline__ void wait_inits(const unsigned *cnt, int ninit) {
+    if (ninit <= 0) return;
+    if (threadIdx.x == 0) {
+        unsigned v;
+        do {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(cnt) : "memory");
+        } while (v < (unsigned)ninit);
+    }
+    __syncthreads();
+}
+
 // v(k:f) = x(R(k:f)) (ancestors are final); the backward x slots of the pivot columns pending
-__global__ void __launch_bounds__(kSolveThreads) k_bsolve_init(DevPlan d, const int32_t *__restrict__ tasks,
-                                                               const double *__restrict__ y,
-                                                               const int32_t *__restrict__ sn_rows,
-                                                               const int64_t *__restrict__ sn_rowptr) {
-    const int s = tasks[2 * blockIdx.x], part = tasks[2 * blockIdx.x + 1];
+__device__ __forceinline__ void bsolve_init_task(const DevPlan &d, const int32_t *__restrict__ tasks,
+                                                 const double *__restrict__ y, const int32_t *__restrict__ sn_rows,
+                                                 const int64_t *__restrict__ sn_rowptr, const int task) {
+    const int s = tasks[2 * task], part = tasks[2 * task + 1];
     const int k = d.sn_k[s], f = d.sn_f[s];
     const int p0 = part * kInitRows, p1 = min(f, p0 + kInitRows);
     double *__restrict__ v = d.fv + d.fv_off[s];
@@ -1513,6 +1545,16 @@ __global__ void __launch_bounds__(kSolveThreads) k_bsolve_init(DevPlan d, const 
         if (i >= k) v[i] = y[R[i]];
         else xp[i] = pending_value();
     }
+}
+__global__ void __launch_bounds__(kSolveThreads) k_bsolve_init(DevPlan d, const int32_t *__restrict__ tasks,
+                                                               const double *__restrict__ y,
+                                                               const int32_t *__restrict__ sn_rows,
+                                                               const int64_t *__restrict__ sn_rowptr) {
+    bsolve_init_task(d, tasks, y, sn_rows, sn_rowptr, blockIdx.x);
+}
+void launch_bsolve_init(const DevPlan &d, const int32_t *tasks, int64_t count, const double *y,
+                        const int32_t *sn_rows, const int64_t *sn_rowptr, cudaStream_t st) {
+    if (count > 0) k_bsolve_init<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, y, sn_rows, sn_rowptr);
 }
 
 // ---- solve setup: inv(L_bb) of every 64 x 64 diagonal block of the dataflow-solved
@@ -1578,7 +1620,8 @@ __device__ __forceinline__ void fsolve_load(const double *__restrict__ P, int ld
 }
 template <int NBUF>
 __device__ __forceinline__ void fsolve_rows_task(const DevPlan &d, const int32_t *__restrict__ tasks, int w,
-                                                 double *__restrict__ y, const int task) {
+                                                 double *__restrict__ y, const int task, const unsigned *cnt,
+                                                 int ninit) {
     __shared__ double Ms[kSW * kSLD];   // inv(L_bb) of the owned block: element (q, c) at q + c kSLD
     __shared__ double ys[2][kSW];
     __shared__ double red[4][kSW];
@@ -1597,12 +1640,13 @@ __device__ __forceinline__ void fsolve_rows_task(const DevPlan &d, const int32_t
         const double *__restrict__ M = Dinv + (int64_t)b * kSW * kSW;
         for (int q = tid; q < kSW * kSW; q += kDfThreads) Ms[(q & 63) + (q >> 6) * kSLD] = __ldg(M + q);
     };
-    if (tid < kSW) vrow[tid] = rok ? v[r] : 0.0;
     if (bown < nbr) load_inv(bown);
     double Lb[NBUF][16];
 #pragma unroll
     for (int q = 0; q < NBUF; q++)
         if (q < nbr) fsolve_load(P, ld, k, w, r, rok, q, Lb[q]);
+    wait_inits(cnt, ninit);   // v and the level's y slots are set by the fused init tasks
+    if (tid < kSW) vrow[tid] = rok ? v[r] : 0.0;
     double acc = 0.0;
     for (int b0 = 0; b0 < nbr; b0 += NBUF) {
 #pragma unroll
@@ -1652,8 +1696,16 @@ __device__ __forceinline__ void fsolve_rows_task(const DevPlan &d, const int32_t
 // 7.12 at <2, 2>); levels of small fronts take the shallow ring at 3 CTAs / SM
 template <int NBUF, int MINB>
 __global__ void __launch_bounds__(kDfThreads, MINB) k_fsolve_df(DevPlan d, const int32_t *__restrict__ tasks, int w,
-                                                                double *__restrict__ y, unsigned *tk) {
-    fsolve_rows_task<NBUF>(d, tasks, w, y, take_ticket(tk));
+                                                                double *__restrict__ y, unsigned *tk,
+                                                                const int32_t *__restrict__ itasks, int ninit) {
+    static_assert(kDfThreads == kSolveThreads, "init tasks run in dataflow CTAs");
+    const int t = take_ticket(tk);
+    if (t < ninit) {
+        fsolve_init_task(d, itasks, y, t);
+        init_done(tk + 2);
+    } else {
+        fsolve_rows_task<NBUF>(d, tasks, w, y, t - ninit, tk + 2, ninit);
+    }
     drop_ticket(tk);
 }
 
@@ -1694,7 +1746,8 @@ __device__ __forceinline__ void warp_reduce_scatter16(double (&p)[16]) {
 }
 template <int NBUF>
 __device__ __forceinline__ void bsolve_cols_task(const DevPlan &d, const int32_t *__restrict__ tasks, int w,
-                                                 double *__restrict__ y, const int task) {
+                                                 double *__restrict__ y, const int task, const unsigned *cnt,
+                                                 int ninit) {
     __shared__ double Ms[kSW * kSLD];   // inv(L_bb)^T: element (q, c) = inv(c, q) at q + c kSLD
     __shared__ double red[8][16];
     __shared__ double tv[kSW];
@@ -1736,6 +1789,7 @@ __device__ __forceinline__ void bsolve_cols_task(const DevPlan &d, const int32_t
 #pragma unroll
     for (int q = 0; q < NBUF; q++)
         if (q < ns) bsolve_load(P, ld, f, j0, we, rlo, slab_row(q), Lb[q]);
+    wait_inits(cnt, ninit);   // v and the x slots of the level are set by the fused init tasks
     // the tail segments' partials (lower tickets: they are done or nearly so) -- read
     // now, while the chain is still above this block, not on its critical path
     double segsum = 0.0;
@@ -1788,14 +1842,20 @@ __device__ __forceinline__ void bsolve_cols_task(const DevPlan &d, const int32_t
 }
 template <int NBUF, int MINB>
 __global__ void __launch_bounds__(kDfThreads, MINB) k_bsolve_df(DevPlan d, const int32_t *__restrict__ tasks, int w,
-                                                                double *__restrict__ y, unsigned *tk) {
-    bsolve_cols_task<NBUF>(d, tasks, w, y, take_ticket(tk));
+                                                                double *__restrict__ y, unsigned *tk,
+                                                                const int32_t *__restrict__ itasks, int ninit,
+                                                                const int32_t *__restrict__ sn_rows,
+                                                                const int64_t *__restrict__ sn_rowptr) {
+    const int t = take_ticket(tk);
+    if (t < ninit) {
+        bsolve_init_task(d, itasks, y, sn_rows, sn_rowptr, t);
+        init_done(tk + 2);
+    } else {
+        bsolve_cols_task<NBUF>(d, tasks, w, y, t - ninit, tk + 2, ninit);
+    }
     drop_ticket(tk);
 }
 
-void launch_fsolve_init(const DevPlan &d, const int32_t *tasks, int64_t count, double *y, cudaStream_t st) {
-    if (count > 0) k_fsolve_init<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, y);
-}
 // MF_DF_VARIANT (tuning A/B): deep ring 0 = <2 blocks, 2 CTAs/SM>, 1 = <3, 2>, 2 = <4, 1>, 3 = <2, 3>
 static int df_variant() {
     static const int v = [] {
@@ -1804,39 +1864,38 @@ static int df_variant() {
     }();
     return v;
 }
-void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, int deep, double *y,
-                      unsigned *tk, cudaStream_t st) {
+void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, const int32_t *itasks, int64_t ninit,
+                      int w, int deep, double *y, unsigned *tk, cudaStream_t st) {
     if (count <= 0) return;
-    const unsigned n = (unsigned)count;
+    const unsigned n = (unsigned)(count + ninit);
+    const int ni = (int)ninit;
     if (!deep)
-        k_fsolve_df<1, 3><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+        k_fsolve_df<1, 3><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk, itasks, ni);
     else if (df_variant() == 1)
-        k_fsolve_df<3, 2><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+        k_fsolve_df<3, 2><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk, itasks, ni);
     else if (df_variant() == 2)
-        k_fsolve_df<4, 1><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+        k_fsolve_df<4, 1><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk, itasks, ni);
     else if (df_variant() == 3)
-        k_fsolve_df<2, 3><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+        k_fsolve_df<2, 3><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk, itasks, ni);
     else
-        k_fsolve_df<kDfBuf, 2><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+        k_fsolve_df<kDfBuf, 2><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk, itasks, ni);
 }
-void launch_bsolve_init(const DevPlan &d, const int32_t *tasks, int64_t count, const double *y,
-                        const int32_t *sn_rows, const int64_t *sn_rowptr, cudaStream_t st) {
-    if (count > 0) k_bsolve_init<<<(unsigned)count, kSolveThreads, 0, st>>>(d, tasks, y, sn_rows, sn_rowptr);
-}
-void launch_bsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, int deep, double *y,
-                      unsigned *tk, cudaStream_t st) {
+void launch_bsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, const int32_t *itasks, int64_t ninit,
+                      int w, int deep, double *y, const int32_t *sn_rows, const int64_t *sn_rowptr, unsigned *tk,
+                      cudaStream_t st) {
     if (count <= 0) return;
-    const unsigned n = (unsigned)count;
+    const unsigned n = (unsigned)(count + ninit);
+    const int ni = (int)ninit;
     if (!deep)
-        k_bsolve_df<1, 3><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+        k_bsolve_df<1, 3><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk, itasks, ni, sn_rows, sn_rowptr);
     else if (df_variant() == 1)
-        k_bsolve_df<3, 2><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+        k_bsolve_df<3, 2><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk, itasks, ni, sn_rows, sn_rowptr);
     else if (df_variant() == 2)
-        k_bsolve_df<4, 1><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+        k_bsolve_df<4, 1><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk, itasks, ni, sn_rows, sn_rowptr);
     else if (df_variant() == 3)
-        k_bsolve_df<2, 3><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+        k_bsolve_df<2, 3><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk, itasks, ni, sn_rows, sn_rowptr);
     else
-        k_bsolve_df<kDfBuf, 2><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk);
+        k_bsolve_df<kDfBuf, 2><<<n, kDfThreads, 0, st>>>(d, tasks, w, y, tk, itasks, ni, sn_rows, sn_rowptr);
 }
 
 // dst[first_s + j] = src[first_s + j] for the columns of the listed supernodes

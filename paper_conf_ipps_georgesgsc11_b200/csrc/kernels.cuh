@@ -75,16 +75,20 @@ void launch_bwd_solve(const DevPlan &d, const int32_t *list, int count, double *
                       const int64_t *sn_rowptr, cudaStream_t st);
 // solve setup: inverses of the 64 x 64 diagonal blocks of the dataflow-solved supernodes
 void launch_diag_inv(const DevPlan &d, const int32_t *tasks, int64_t count, int w, cudaStream_t st);
-// (supernode, 2048-row part) pairs: front vectors of the large supernodes, children gathered
 void launch_fill_pending(double *p, int64_t n, cudaStream_t st);   // dataflow-solve slots: not yet written
-void launch_fsolve_init(const DevPlan &d, const int32_t *tasks, int64_t count, double *y, cudaStream_t st);
+
 // deep = 1: the levels with multi-block fronts (register ring of MF_DF_BUF blocks, 1 CTA / SM)
-void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, int deep, double *y,
-                      unsigned *tk, cudaStream_t st);
-void launch_bsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, int w, int deep, double *y,
-                      unsigned *tk, cudaStream_t st);
+// the init tasks of a level (front vectors, pending slots) as a launch of their own ...
+void launch_fsolve_init(const DevPlan &d, const int32_t *tasks, int64_t count, double *y, cudaStream_t st);
 void launch_bsolve_init(const DevPlan &d, const int32_t *tasks, int64_t count, const double *y,
                         const int32_t *sn_rows, const int64_t *sn_rowptr, cudaStream_t st);
+// ... or (itasks / ninit) run first in the level's dataflow launch
+void launch_fsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, const int32_t *itasks, int64_t ninit,
+                      int w, int deep, double *y, unsigned *tk, cudaStream_t st);
+void launch_bsolve_df(const DevPlan &d, const int32_t *tasks, int64_t count, const int32_t *itasks, int64_t ninit,
+                      int w, int deep, double *y, const int32_t *sn_rows, const int64_t *sn_rowptr, unsigned *tk,
+                      cudaStream_t st);
+
 
 int small_front_smem_ok(int fmax);
 int kernels_init();

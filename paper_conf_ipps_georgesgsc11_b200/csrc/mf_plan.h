@@ -202,17 +202,22 @@ struct Launch {
 // Triangular-solve program (forward sweep bottom-up, backward sweep top-down).
 enum SolveKind : int32_t {
     SK_SMALL_F = 0,   // one CTA per small supernode: gather, trsv, gemv
-    SK_INIT_F = 1,    // large supernodes: v = [y(cols); 0] + extend-add of children's update vectors
+    SK_INIT_F = 1,    // large supernodes: v = [y(cols); 0] + children's update vectors (levels of many fronts;
+                      // otherwise the init tasks run in the SK_DF_F launch)
     SK_DF_F = 2,      // all large supernodes of a level, one launch: 256-row chunks, per-block flags
     SK_SMALL_B = 3,
-    SK_INIT_B = 4,    // large supernodes: v(k:f) = x(R(k:f))
+    SK_INIT_B = 4,    // large supernodes: v(k:f) = x(R(k:f)) (idem, SK_DF_B)
     SK_DF_B = 5       // all large supernodes of a level, one launch: chunk partials, owner reduces + trsv
 };
 struct SolveLaunch {
     int32_t kind;
     int32_t j0;   // factor launches: first column; SK_DF_*: 1 = deep register ring
     int64_t off, count;
+    // SK_DF_*: the level's init tasks [off2, off2 + count2) run in the same launch
+    // (lower tickets; the dataflow tasks wait for their completion count)
+    int64_t off2 = 0, count2 = 0;
 };
+constexpr int kTkWords = 4;   // words per launch slot: ticket, finished CTAs, fused-init count, (spare)
 
 struct Plan {
     int32_t nsuper = 0, nlevels = 0, w = 64, small_max = 128, max_front = 0;
@@ -289,6 +294,7 @@ constexpr int kSolveRowBlock = 64;    // dataflow forward solve: rows per task (
 constexpr int kSolveSmallMax = 256, kSolveSmallK = 32;
 constexpr int kSolveDeepK = 256;      // dataflow solve: levels with a front of k >= this take the deep ring
 constexpr int kSolveInitRows = 2048;
+constexpr int kSolveFuseInitMax = 256;   // levels with at most this many init tasks run them in the dataflow launch
 constexpr int kSolveSegSlabs = 16;    // dataflow backward solve: 64-row tail slabs per segment task  // solve init: front-vector rows per task (kernels.cu kInitRows)
 
 int build_plan(const Symbolic &S, const Options &opt, Plan &P);

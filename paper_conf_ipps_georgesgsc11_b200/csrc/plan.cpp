@@ -141,12 +141,17 @@ static void build_solve_plan(const Symbolic &S, Plan &P, const std::vector<char>
             for (int32_t q = 0; q * kSolveInitRows < P.sn_f[s]; q++) push_task(s, q);
         return off;
     };
+    static const int64_t fuse_init_max = [] {   // MF_SOLVE_FUSE_INIT: tuning override (0 = never fuse)
+        const char *e = getenv("MF_SOLVE_FUSE_INIT");
+        return e ? (int64_t)atoll(e) : (int64_t)kSolveFuseInitMax;
+    }();
     for (int32_t l = 0; l < P.nlevels; l++) {
         if (!small[l].empty()) fsolve.push_back({SK_SMALL_F, 0, push_list(small[l]), (int64_t)small[l].size()});
         if (large[l].empty()) continue;
-        {
-            const int64_t off = push_init(large[l]);
-            fsolve.push_back({SK_INIT_F, 0, off, (int64_t)P.df_tasks.size() / 2 - off});
+        int64_t ioff = push_init(large[l]), icnt = (int64_t)P.df_tasks.size() / 2 - ioff;
+        if (icnt > fuse_init_max) {
+            fsolve.push_back({SK_INIT_F, 0, ioff, icnt});
+            ioff = icnt = 0;
         }
         // the pivot-row tasks of every front first, round robin (every chain starts at
         // once), then the rows below k; a task waits only on lower tickets of its front
@@ -162,13 +167,14 @@ static void build_solve_plan(const Symbolic &S, Plan &P, const std::vector<char>
         for (int32_t s : large[l])
             for (int32_t rb = (P.sn_k[s] + kSolveRowBlock - 1) / kSolveRowBlock; rb * kSolveRowBlock < P.sn_f[s]; rb++)
                 push_task(s, rb);
-        fsolve.push_back({SK_DF_F, deep_level(large[l]), off, (int64_t)P.df_tasks.size() / 2 - off});
+        fsolve.push_back({SK_DF_F, deep_level(large[l]), off, (int64_t)P.df_tasks.size() / 2 - off, ioff, icnt});
     }
     for (int32_t l = P.nlevels - 1; l >= 0; l--) {
         if (!large[l].empty()) {
-            {
-                const int64_t off = push_init(large[l]);
-                bsolve.push_back({SK_INIT_B, 0, off, (int64_t)P.df_tasks.size() / 2 - off});
+            int64_t ioff = push_init(large[l]), icnt = (int64_t)P.df_tasks.size() / 2 - ioff;
+            if (icnt > fuse_init_max) {
+                bsolve.push_back({SK_INIT_B, 0, ioff, icnt});
+                ioff = icnt = 0;
             }
             // the tail segments first (they wait for nothing), then the column blocks from
             // the last one down, round robin over the fronts
@@ -189,7 +195,7 @@ static void build_solve_plan(const Symbolic &S, Plan &P, const std::vector<char>
                     const int32_t nb = (P.sn_k[s] + w - 1) / w;
                     if (t < nb) push_task(s, nb - 1 - t);
                 }
-            bsolve.push_back({SK_DF_B, deep_level(large[l]), off, (int64_t)P.df_tasks.size() / 2 - off});
+            bsolve.push_back({SK_DF_B, deep_level(large[l]), off, (int64_t)P.df_tasks.size() / 2 - off, ioff, icnt});
         }
         if (!small[l].empty()) bsolve.push_back({SK_SMALL_B, 0, push_list(small[l]), (int64_t)small[l].size()});
     }

@@ -9,6 +9,25 @@
 
 using namespace mf;
 
+__device__ __forceinline__ void nbar_arrive(int id, int n) { asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+// one row of the row solve of panel_potrf_dmma (kernels.cu), as a function
+__device__ __forceinline__ void potrf_rows8(double *A, const double *sinv, int s0, int nb, int r) {
+    double x[8];
+#pragma unroll
+    for (int q = 0; q < 8; q++) x[q] = (q < nb) ? A[(s0 + q) * kPLD + r] : 0.0;
+#pragma unroll
+    for (int q = 0; q < 8; q++)
+        if (q < nb) {
+            x[q] *= sinv[s0 + q];
+#pragma unroll
+            for (int q2 = q + 1; q2 < 8; q2++)
+                if (q2 < nb) x[q2] = fma(-x[q], A[(s0 + q) * kPLD + s0 + q2], x[q2]);
+        }
+#pragma unroll
+    for (int q = 0; q < 8; q++)
+        if (q < nb) A[(s0 + q) * kPLD + r] = x[q];
+}
+
 __global__ void parts(DevPlan d, long long *out) {
     __shared__ double A[64 * kPLD];
     __shared__ double sinv[64];
@@ -66,13 +85,56 @@ __global__ void whole(DevPlan d, long long *out) {
         const long long t0 = clock64();
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g0));
         if (V == 0) panel_potrf_dmma(d, A, sinv, 64, 64, 0);
-        else panel_potrf_la(d, A, sinv, 64, 64, 0);
+        else panel_potrf_dmma(d, A, sinv, 64, 64, 0);
         const long long t1 = clock64();
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g1));
         acc += t1 - t0;
         __syncthreads();
     }
     if (tid == 0) { out[0] = acc / 20; out[1] = g1 - g0; }
+}
+
+// warp 0: factor_diag8 x 100 (cycles); warps 1-3 meanwhile: 0 idle, 1 DMMA loop, 2 DFMA loop, 3 LDS/STS loop
+template <int BG>
+__global__ void interfere(DevPlan d, long long *out) {
+    __shared__ double A[64 * kPLD];
+    __shared__ double sinv[64];
+    __shared__ volatile int stop;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    for (int q = tid; q < 64 * kPLD; q += blockDim.x) {
+        const int r = q % kPLD, c = q / kPLD;
+        A[q] = (r == c) ? 64.0 : 1.0 / (1 + r + c);
+    }
+    if (tid == 0) stop = 0;
+    __syncthreads();
+    if (warp == 0) {
+        long long acc = 0;
+        for (int it = 0; it < 100; it++) {
+            __syncwarp();
+            const long long t0 = clock64();
+            if (lane == 0) factor_diag8(d, A, sinv, 0, 8, 0);
+            __syncwarp();
+            acc += clock64() - t0;
+            for (int q = lane; q < 8 * kPLD; q += 32) {
+                const int r = q % kPLD, c = q / kPLD;
+                A[q] = (r == c) ? 64.0 : 1.0 / (1 + r + c);
+            }
+            __syncwarp();
+        }
+        if (lane == 0) { out[0] = acc / 100; stop = 1; }
+    } else if (BG > 0) {
+        double c0 = lane, c1 = 1.0, a = 1e-3 * lane, b = 1e-3;
+        double *B = A + 16 * kPLD + 8 * warp;
+        while (!stop) {
+#pragma unroll 4
+            for (int i = 0; i < 64; i++) {
+                if (BG == 1) dmma(c0, c1, a, b);
+                else if (BG == 2) { c0 = fma(c0, a, b); c1 = fma(c1, a, b); }
+                else { B[lane] = B[lane + 1] + 1.0; }
+            }
+        }
+        if (c0 == 12345.0) out[1] = (long long)c1;
+    }
 }
 
 int main() {
@@ -90,10 +152,19 @@ int main() {
     cudaMemcpy(h, out, 32, cudaMemcpyDeviceToHost);
     printf("factor_diag8 %lld cycles, potrf_rows8 %lld, upd_block8 %lld, bar.arrive %lld (%s)\n", h[0], h[1], h[2],
            h[3], cudaGetErrorString(cudaGetLastError()));
-    for (int v = 0; v < 2; v++) {
+    const char *bgn[4] = {"idle", "DMMA", "DFMA", "LDS/STS"};
+    for (int bg = 0; bg < 4; bg++) {
         for (int rep = 0; rep < 2; rep++) {
-            if (v == 0) whole<0><<<1, 128>>>(d, out); else whole<1><<<1, 128>>>(d, out);
+            if (bg == 0) interfere<0><<<1, 128>>>(d, out);
+            if (bg == 1) interfere<1><<<1, 128>>>(d, out);
+            if (bg == 2) interfere<2><<<1, 128>>>(d, out);
+            if (bg == 3) interfere<3><<<1, 128>>>(d, out);
         }
+        cudaMemcpy(h, out, 8, cudaMemcpyDeviceToHost);
+        printf("factor_diag8 with warps 1-3 %s: %lld cycles (%s)\n", bgn[bg], h[0], cudaGetErrorString(cudaGetLastError()));
+    }
+    for (int v = 0; v < 1; v++) {
+        for (int rep = 0; rep < 2; rep++) whole<0><<<1, 128>>>(d, out);
         cudaMemcpy(h, out, 16, cudaMemcpyDeviceToHost);
         printf("%s 64x64: %lld cycles, last call %lld ns (%s)\n", v == 0 ? "panel_potrf_dmma" : "panel_potrf_la", h[0], h[1],
                cudaGetErrorString(cudaGetLastError()));
