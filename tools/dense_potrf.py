@@ -26,7 +26,7 @@ for k in ks:
     rowind = np.concatenate([np.arange(j, k, dtype=np.int32) for j in range(k)])
     vals = rng.uniform(-1, 1, size=rowind.size)
     vals[colptr[:-1]] = 2.0 * k
-    S = mf.Solver()
+    S = mf.Solver(lookahead=bool(int(os.environ.get("MF_LA", "0"))))   # MF_LA=1: look-ahead schedule
     S.analyze(k, colptr, rowind, np.arange(k, dtype=np.int32))
     v = torch.from_numpy(vals).cuda()
     S.factor(v)
