@@ -1454,6 +1454,11 @@ constexpr int kSW = 64, kSLD = 65;   // solve block width and smem leading dimen
 constexpr int kDfThreads = 256;      // dataflow solve CTA: 64 rows x 4 groups of 16 columns
 constexpr int kDfRB = 64;            // rows per forward task / per backward slab
 constexpr int kDfBuf = MF_DF_BUF;    // register ring: blocks (forward) / slabs (backward) in flight
+#ifndef MF_YPRE
+#define MF_YPRE 8
+#endif
+constexpr int kYPre = MF_YPRE;       // forward: block solutions read per batch (a multiple of 4)
+static_assert(kYPre * 64 % 256 == 0, "kYPre blocks of 64 values over 256 threads");
 constexpr int kInitRows = kSolveInitRows;   // rows of a front vector per init task
 constexpr int kBsSegSlabs = kSolveSegSlabs;  // backward: tail slabs per segment task
 
@@ -1624,6 +1629,7 @@ __device__ __forceinline__ void fsolve_rows_task(const DevPlan &d, const int32_t
                                                  int ninit) {
     __shared__ double Ms[kSW * kSLD];   // inv(L_bb) of the owned block: element (q, c) at q + c kSLD
     __shared__ double ys[2][kSW];
+    __shared__ double yp[kYPre][kSW];   // solutions of the next kYPre blocks above, read in one batch
     __shared__ double red[4][kSW];
     __shared__ double vrow[kSW];
     const int s = tasks[2 * task], rb = tasks[2 * task + 1];
@@ -1656,6 +1662,20 @@ __device__ __forceinline__ void fsolve_rows_task(const DevPlan &d, const int32_t
             const int j0 = b * w, we = min(w, k - j0);
             double *yb = ys[b & 1];
             const bool owned = j0 >= r0;
+            if (b % kYPre == 0) {
+                // one batch of loads for the solutions of blocks b .. b + kYPre - 1 above the
+                // task's rows: a task walking blocks published long ago pays one L2 round
+                // trip per batch instead of one per block (the walk, not the hand-off, set
+                // the pace of the long chains); a slot still pending is polled at its block
+#pragma unroll
+                for (int t = 0; t < kYPre * kSW / kDfThreads; t++) {
+                    const int qq = (tid + t * kDfThreads) >> 6, e = tid & 63, bb = b + qq;
+                    double val = pending_value();
+                    if (bb < nbr && bb * w < r0 && e < min(w, k - bb * w)) val = ld_relaxed_f64(y + first + bb * w + e);
+                    yp[qq][e] = val;
+                }
+                __syncthreads();
+            }
             if (owned) {   // t_b = v - partials (rows of the block), x_b = inv(L_bb) t_b
                 red[g][i] = acc;
                 acc = 0.0;
@@ -1679,7 +1699,12 @@ __device__ __forceinline__ void fsolve_rows_task(const DevPlan &d, const int32_t
                     yb[i] = i < we ? x : 0.0;
                 }
             } else if (tid < kSW) {   // a block above: its solution, value by value
-                yb[tid] = tid < we ? wait_value(y + first + j0 + tid) : 0.0;
+                double val = 0.0;
+                if (tid < we) {
+                    val = yp[b % kYPre][tid];
+                    if ((unsigned long long)__double_as_longlong(val) == kSolvePending) val = wait_value(y + first + j0 + tid);
+                }
+                yb[tid] = val;
             }
             __syncthreads();
             if (owned && b + 1 < nbr && (b + 1) * w < r0 + kDfRB) load_inv(b + 1);   // w < 64: the next owned block
@@ -1802,13 +1827,24 @@ __device__ __forceinline__ void bsolve_cols_task(const DevPlan &d, const int32_t
     double acc[16];
 #pragma unroll
     for (int u = 0; u < 16; u++) acc[u] = 0.0;
-    for (int q0 = 0; q0 < ns; q0 += NBUF) {
+    // the x values of XP slabs (this thread's row in each) are loaded in one batch: a
+    // task walking rows whose x was published long ago pays one L2 round trip per
+    // batch instead of one per slab; a value still pending is polled at its slab
+    constexpr int XP = NBUF == 1 ? 1 : (4 % NBUF == 0 ? 4 : NBUF);   // (NBUF = 1 at 3 CTAs / SM: no room)
+    for (int q0 = 0; q0 < ns; q0 += XP) {
+        double xq[XP];
 #pragma unroll
-        for (int q = 0; q < NBUF; q++) {
-            const int sq = q0 + q;
+        for (int t = 0; t < XP; t++) {
+            const int sq = q0 + t, r = slab_row(sq);
+            xq[t] = (sq < ns && r >= rlo && r < f) ? (r >= k ? v[r] : ld_relaxed_f64(xp + r)) : 0.0;
+        }
+#pragma unroll
+        for (int t = 0; t < XP; t++) {
+            const int sq = q0 + t, q = t % NBUF;   // (q0 is a multiple of NBUF)
             if (sq >= ns) break;
             const int r = slab_row(sq);
-            const double xr = (r >= rlo && r < f) ? (r >= k ? v[r] : wait_value(xp + r)) : 0.0;
+            double xr = xq[t];
+            if ((unsigned long long)__double_as_longlong(xr) == kSolvePending) xr = wait_value(xp + r);
 #pragma unroll
             for (int u = 0; u < 16; u++) acc[u] = fma(Lb[q][u], xr, acc[u]);
             if (sq + NBUF < ns) bsolve_load(P, ld, f, j0, we, rlo, slab_row(sq + NBUF), Lb[q]);
