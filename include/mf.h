@@ -273,6 +273,8 @@ typedef struct {
     double bytes;
     double int8_ops;   /* Schur update on the int8 tensor cores (ozaki_slices): int8 MMA
                           operations executed (2 x MACs, padding included), else 0 */
+    int32_t stream;    /* single GPU: subtree branch (CUDA-graph branch) of the launch, -1 = main */
+    int32_t reserved;
 } mf_launch_info;
 
 /* out may be NULL to query *count only. */
@@ -290,7 +292,11 @@ int mf_set_exchange(mf_ctx *ctx, mf_exchange_fn fn, void *user);
  * of the top.  Any pointer may be NULL. */
 int mf_get_mapping(const mf_ctx *ctx, int32_t *owner, int8_t *top, double *rank_load, double *top_load);
 
-/* Enable (1) / disable (0) per-launch CUDA-event timing in mf_factor; resets the stats. */
+/* Per-launch CUDA-event timing in mf_factor; resets the stats.  enable = 1: the
+ * launches run eagerly on one stream, an event around each (serialised: per-kernel
+ * times); 2: timeline -- the factorization runs as its usual CUDA graph (subtree
+ * branches and streams concurrent), with timing events captured before and after
+ * every launch (mf_get_launch_timeline); 0: off. */
 int mf_set_profiling(mf_ctx *ctx, int enable);
 
 /* out[MF_KERNEL_CLASSES]: accumulated stats since the last mf_set_profiling; *count = classes written. */
@@ -299,6 +305,15 @@ int mf_get_kernel_stats(const mf_ctx *ctx, mf_kernel_stat *out, int32_t *count);
 /* Per-launch CUDA-event times (ms) of the last PROFILED factorization, in program
  * order (mf_get_program; the local program only).  out may be NULL to query *count. */
 int mf_get_launch_times(const mf_ctx *ctx, double *out_ms, int64_t max, int64_t *count);
+
+/* Timeline of the last factorization run with mf_set_profiling(ctx, 2): for every
+ * launch of the local program (program order, mf_get_program) the times (ms) at
+ * which its stream reached it and finished it, relative to the start of the
+ * factorization, as the concurrent graph ran -- the critical path of the
+ * schedule, not per-kernel costs.  start_ms / end_ms may be NULL (both NULL:
+ * *count only).  MF_ERR_STATE unless such a factorization ran.  Multi-GPU: the
+ * local program only. */
+int mf_get_launch_timeline(const mf_ctx *ctx, double *start_ms, double *end_ms, int64_t max, int64_t *count);
 
 /* Learned kernel-variant selector (Sec. VI, Eqs. 3-5).
  * The paper picks a CPU/GPU policy per factor-update call with a cost-sensitive

@@ -70,7 +70,10 @@ struct mf_ctx {
     bool dinv_stale = true;          // set by mf_factor; the next solve recomputes the block inverses
     cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev_in = nullptr;
     int64_t launches = 0;
-    bool profiling = false;
+    int profiling = 0;               // 1: eager per-launch events; 2: timeline (events captured in the graph)
+    cudaGraph_t graph_tl = nullptr;  // the timeline-mode graph of the local program (events after every launch)
+    cudaGraphExec_t graph_tl_exec = nullptr;
+    cudaEvent_t tl_base = nullptr;   // timeline zero: recorded after the init launch
     bool use_graph = true;
     cudaGraph_t graph = nullptr, graph_top = nullptr, solve_graph = nullptr;
     cudaGraphExec_t graph_exec = nullptr, graph_top_exec = nullptr, solve_exec = nullptr;
@@ -152,6 +155,9 @@ int dev_upload(mf_ctx *c, T **dst, const std::vector<T> &src) {
 void drop_graph(mf_ctx *c) {
     if (c->graph_exec) cudaGraphExecDestroy(c->graph_exec);
     if (c->graph) cudaGraphDestroy(c->graph);
+    if (c->graph_tl_exec) cudaGraphExecDestroy(c->graph_tl_exec);
+    if (c->graph_tl) cudaGraphDestroy(c->graph_tl);
+    if (c->tl_base) cudaEventDestroy(c->tl_base);
     if (c->graph_top_exec) cudaGraphExecDestroy(c->graph_top_exec);
     if (c->graph_top) cudaGraphDestroy(c->graph_top);
     c->graph_exec = nullptr;
@@ -626,8 +632,13 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
     const DevPlan &d = c->d;
     cudaStream_t st = c->stream;
     unsigned *tk0 = c->d_tickets + kTkWords * (&prog == &P.program ? 0 : P.program.size());   // this program's slots
-    auto issue = [&](const double *v, bool with_events) -> int {
+    // tl: timeline mode -- the graph keeps its branches and streams, with a timing
+    // event recorded before and after every launch on the launch's own stream
+    auto issue = [&](const double *v, bool with_events, bool tl = false) -> int {
         if (with_init) launch_init_failed(c->d_failed, st);
+        // (captured timing events must be external record nodes: a plain record in a
+        // capture only tracks a dependency and is never executed)
+        if (tl) CK(cudaEventRecordWithFlags(c->tl_base, st, cudaEventRecordExternal));
         // subtree branches run on their own streams (forked after the init launch,
         // joined before the first top launch); profiled runs stay on one stream
         const bool branches = !with_events && P.nbranch > 1 && (int)c->bstreams.size() >= P.nbranch;
@@ -674,6 +685,7 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
             }
             auto launch = [&](cudaStream_t st) -> int {
             if (with_events) CK(cudaEventRecord(c->prof_events[ev_base + 2 * li], st));
+            if (tl) CK(cudaEventRecordWithFlags(c->prof_events[ev_base + 2 * li], st, cudaEventRecordExternal));
             switch (L.kind) {
                 case KC_SMALL: launch_small_fronts(d, c->d_small + L.off, (int)L.count, L.param, v, st); break;
                 case KC_ASSEMBLE: launch_assemble(d, c->d_asm + 2 * L.off, L.count, v, st); break;
@@ -698,6 +710,7 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
                 default: return MF_ERR_STATE;   // exchange points are handled by run_with_exchanges
             }
             if (with_events) CK(cudaEventRecord(c->prof_events[ev_base + 2 * li + 1], st));
+            if (tl) CK(cudaEventRecordWithFlags(c->prof_events[ev_base + 2 * li + 1], st, cudaEventRecordExternal));
             return MF_OK;
             };
             if (int r = launch(ls)) return r;
@@ -711,8 +724,26 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
         }
         return MF_OK;
     };
-    if (c->profiling) return issue(vals, true);
+    if (c->profiling == 1) return issue(vals, true);
     if (!c->use_graph || !graph) return issue(vals, false);
+    if (c->profiling == 2) {   // timeline: its own graph of the local program, events captured into it
+        if (&prog != &P.program) return MF_ERR_STATE;
+        if (vals != c->d_values && c->S.nnz_in > 0 && with_init)
+            CK(cudaMemcpyAsync(c->d_values, vals, c->S.nnz_in * sizeof(double), cudaMemcpyDeviceToDevice, st));
+        if (!c->graph_tl_exec) {
+            if (!c->tl_base) CK(cudaEventCreate(&c->tl_base));
+            CK(cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
+            int r = issue(c->d_values, false, true);
+            cudaGraph_t g = nullptr;
+            cudaError_t e = cudaStreamEndCapture(st, &g);
+            if (r) return r;
+            CK(e);
+            c->graph_tl = g;
+            CK(cudaGraphInstantiateWithFlags(&c->graph_tl_exec, g, cudaGraphInstantiateFlagUseNodePriority));
+        }
+        CK(cudaGraphLaunch(c->graph_tl_exec, st));
+        return MF_OK;
+    }
     // the graph always reads the ctx's value buffer
     if (vals != c->d_values && c->S.nnz_in > 0 && with_init)
         CK(cudaMemcpyAsync(c->d_values, vals, c->S.nnz_in * sizeof(double), cudaMemcpyDeviceToDevice, st));
@@ -826,7 +857,7 @@ int mf_factor(mf_ctx *c, const double *values) {
         std::vector<mf_xfer> bc{mf_xfer{MF_XFER_BCAST, 0, c->d_values, c->S.nnz_in * (int64_t)sizeof(double)}};
         if (int r = exchange(c, bc)) return r;
     }
-    const bool prof = c->profiling;
+    const bool prof = c->profiling != 0;
     const size_t nev = 2 * (P.program.size() + P.program_top.size());
     if (prof && c->prof_events.size() < nev) {
         for (size_t i = c->prof_events.size(); i < nev; i++) {
@@ -1202,7 +1233,8 @@ static const char *kKernelNames[KC_COUNT] = {"small_front_fused", "assemble_exte
 
 int mf_set_profiling(mf_ctx *c, int enable) {
     if (!c) return MF_ERR_ARG;
-    c->profiling = enable != 0;
+    if (enable < 0 || enable > 2) return MF_ERR_ARG;
+    c->profiling = enable;
     for (int k = 0; k < KC_COUNT; k++) {
         c->kstats[k] = mf_kernel_stat{};
         snprintf(c->kstats[k].name, sizeof(c->kstats[k].name), "%s", kKernelNames[k]);
@@ -1230,8 +1262,8 @@ int mf_get_program(const mf_ctx *c, mf_launch_info *out, int64_t max, int64_t *c
     *count = (int64_t)prog.size();
     if (out)
         for (int64_t i = 0; i < std::min<int64_t>(max, (int64_t)prog.size()); i++)
-            out[i] = mf_launch_info{prog[i].kind, prog[i].level, prog[i].count, prog[i].flops, prog[i].bytes,
-                                    prog[i].int8_ops};
+            out[i] = mf_launch_info{prog[i].kind,     prog[i].level, prog[i].count, prog[i].flops, prog[i].bytes,
+                                    prog[i].int8_ops, prog[i].stream, 0};
     return MF_OK;
 }
 
@@ -1245,6 +1277,24 @@ int mf_get_launch_times(const mf_ctx *c, double *out, int64_t max, int64_t *coun
         float t = 0.f;
         cudaEventElapsedTime(&t, c->prof_events[2 * i], c->prof_events[2 * i + 1]);
         out[i] = t;
+    }
+    return MF_OK;
+}
+
+int mf_get_launch_timeline(const mf_ctx *c, double *start_ms, double *end_ms, int64_t max, int64_t *count) {
+    if (!c || !count) return MF_ERR_ARG;
+    const int64_t n = (int64_t)c->P.program.size();
+    *count = n;
+    if (!start_ms && !end_ms) return MF_OK;
+    if (c->host_only || c->profiling != 2 || c->prof_factors == 0 || !c->tl_base ||
+        (int64_t)c->prof_events.size() < 2 * n)
+        return MF_ERR_STATE;
+    for (int64_t i = 0; i < std::min(n, max); i++) {
+        float t0 = 0.f, t1 = 0.f;
+        cudaEventElapsedTime(&t0, c->tl_base, c->prof_events[2 * i]);
+        cudaEventElapsedTime(&t1, c->tl_base, c->prof_events[2 * i + 1]);
+        if (start_ms) start_ms[i] = t0;
+        if (end_ms) end_ms[i] = t1;
     }
     return MF_OK;
 }

@@ -27,7 +27,7 @@ EXPORTED_SYMBOLS = (
     "mf_get_perm", "mf_get_etree", "mf_get_supernodes", "mf_export_panel", "mf_export_diag", "mf_export_L",
     "mf_export_panels", "mf_solve_nrhs",
     "mf_get_program", "mf_set_profiling", "mf_get_kernel_stats", "mf_set_exchange", "mf_get_mapping", "mf_destroy", "mf_strerror",
-    "mf_get_launch_times", "mf_set_variant_model", "mf_get_variants",
+    "mf_get_launch_times", "mf_get_launch_timeline", "mf_set_variant_model", "mf_get_variants",
 )
 MF_VARIANTS = 7
 MF_VARIANT_FEATURES = 9
@@ -84,7 +84,8 @@ EXCHANGE_FN = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.POINTER(Xfe
 
 class LaunchInfo(ctypes.Structure):
     _fields_ = [("kind", ctypes.c_int32), ("level", ctypes.c_int32), ("count", ctypes.c_int64),
-                ("flops", ctypes.c_double), ("bytes", ctypes.c_double), ("int8_ops", ctypes.c_double)]
+                ("flops", ctypes.c_double), ("bytes", ctypes.c_double), ("int8_ops", ctypes.c_double),
+                ("stream", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 def lib_path() -> str:
@@ -120,6 +121,7 @@ def _load():
         "mf_destroy": ([vp], None),
         "mf_strerror": ([ctypes.c_int], ctypes.c_char_p),
         "mf_get_launch_times": ([vp, vp, i64, ctypes.POINTER(i64)], ctypes.c_int),
+        "mf_get_launch_timeline": ([vp, vp, vp, i64, ctypes.POINTER(i64)], ctypes.c_int),
         "mf_set_variant_model": ([vp, vp, i32, i32, i32], ctypes.c_int),
         "mf_get_variants": ([vp, vp], ctypes.c_int),
     }
@@ -358,8 +360,8 @@ class Solver:
         self._check(lib.mf_get_program(self._h, None, 0, ctypes.byref(cnt)), "mf_get_program")
         arr = (LaunchInfo * max(cnt.value, 1))()
         self._check(lib.mf_get_program(self._h, arr, cnt.value, ctypes.byref(cnt)), "mf_get_program")
-        return [dict(kind=a.kind, level=a.level, count=a.count, flops=a.flops, bytes=a.bytes, int8_ops=a.int8_ops)
-                for a in arr[:cnt.value]]
+        return [dict(kind=a.kind, level=a.level, count=a.count, flops=a.flops, bytes=a.bytes, int8_ops=a.int8_ops,
+                     stream=a.stream) for a in arr[:cnt.value]]
 
     def launch_times(self) -> np.ndarray:
         """CUDA-event ms of every launch of the last profiled factorization (program order)."""
@@ -369,6 +371,17 @@ class Solver:
         self._check(lib.mf_get_launch_times(self._h, out.ctypes.data, cnt.value, ctypes.byref(cnt)),
                     "mf_get_launch_times")
         return out[:cnt.value]
+
+    def launch_timeline(self) -> tuple[np.ndarray, np.ndarray]:
+        """(start_ms, end_ms) of every launch of the last factorization run with
+        set_profiling(2): the concurrent graph's timeline (program order)."""
+        cnt = ctypes.c_int64()
+        self._check(lib.mf_get_launch_timeline(self._h, None, None, 0, ctypes.byref(cnt)), "mf_get_launch_timeline")
+        t0 = np.zeros(max(cnt.value, 1), dtype=np.float64)
+        t1 = np.zeros(max(cnt.value, 1), dtype=np.float64)
+        self._check(lib.mf_get_launch_timeline(self._h, t0.ctypes.data, t1.ctypes.data, cnt.value,
+                                               ctypes.byref(cnt)), "mf_get_launch_timeline")
+        return t0[:cnt.value], t1[:cnt.value]
 
     def set_variant_model(self, theta=None, force: int = -1):
         """Kernel-variant selector (before analyze): theta (MF_VARIANT_FEATURES x MF_VARIANTS)
@@ -387,7 +400,8 @@ class Solver:
         self._check(lib.mf_get_variants(self._h, out.ctypes.data), "mf_get_variants")
         return out[:self._info["nsuper"]]
 
-    def set_profiling(self, enable: bool = True):
+    def set_profiling(self, enable: int = 1):
+        """1 (True): eager per-launch timing; 2: timeline of the concurrent graph; 0: off."""
         self._check(lib.mf_set_profiling(self._h, int(enable)), "mf_set_profiling")
 
     def kernel_stats(self) -> list[dict]:

@@ -331,6 +331,40 @@ def sum_panel_words(S, inf):
     return int((k * f).sum())
 
 
+@pytest.mark.parametrize("nb", [1, 4])
+def test_profiling_modes_same_factor(mf, nb):
+    """Eager per-launch timing (profiling 1) and the concurrent-graph timeline
+    (profiling 2: timing events captured into the graph) only observe: L is bitwise
+    equal to the plain graph's; every launch of the timeline ends after it starts,
+    the launches of one stream run in program order, and the per-launch times of
+    both modes are positive."""
+    A, p = grid("7pt", (24, 24, 24))
+    outs = []
+    for mode in (0, 1, 2):
+        S = mf.Solver(nbranch=nb)
+        S.analyze(A.n, A.colptr, A.rowind, p)
+        inf = S.info()
+        S.set_profiling(mode)
+        S.factor(A.values)
+        S.factor(A.values)
+        outs.append(S.export_panels(sum_panel_words(S, inf)))
+        if mode == 1:
+            assert (S.launch_times() > 0).all()
+        if mode == 2:
+            t0, t1 = S.launch_timeline()
+            prog = S.program()
+            assert len(t0) == len(prog) and (t1 >= t0).all() and (t0 >= 0).all()
+            for st in {L["stream"] for L in prog}:
+                idx = [i for i, L in enumerate(prog) if L["stream"] == st]
+                assert (np.diff(t1[idx]) >= 0).all()
+            assert all(k["launches"] > 0 for k in S.kernel_stats() if k["ms"] > 0)
+        else:
+            with pytest.raises(mf.MfError):
+                S.launch_timeline()
+    np.testing.assert_array_equal(outs[0], outs[1])
+    np.testing.assert_array_equal(outs[0], outs[2])
+
+
 def test_degenerate_inputs(mf):
     # n = 1
     A = dense_from_rows([[9.0]])
