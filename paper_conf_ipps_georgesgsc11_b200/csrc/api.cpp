@@ -724,10 +724,12 @@ int run_program(mf_ctx *c, const std::vector<Launch> &prog, size_t i0, size_t i1
         }
         return MF_OK;
     };
-    if (c->profiling == 1) return issue(vals, true);
+    // (timeline mode: the local program as a graph with captured events; anything else
+    // -- the multi-GPU top program's segments, or no graph -- eagerly with events)
+    if (c->profiling == 1 || (c->profiling == 2 && (!c->use_graph || !graph || &prog != &P.program)))
+        return issue(vals, true);
     if (!c->use_graph || !graph) return issue(vals, false);
     if (c->profiling == 2) {   // timeline: its own graph of the local program, events captured into it
-        if (&prog != &P.program) return MF_ERR_STATE;
         if (vals != c->d_values && c->S.nnz_in > 0 && with_init)
             CK(cudaMemcpyAsync(c->d_values, vals, c->S.nnz_in * sizeof(double), cudaMemcpyDeviceToDevice, st));
         if (!c->graph_tl_exec) {
@@ -1286,7 +1288,7 @@ int mf_get_launch_timeline(const mf_ctx *c, double *start_ms, double *end_ms, in
     const int64_t n = (int64_t)c->P.program.size();
     *count = n;
     if (!start_ms && !end_ms) return MF_OK;
-    if (c->host_only || c->profiling != 2 || c->prof_factors == 0 || !c->tl_base ||
+    if (c->host_only || c->profiling != 2 || c->prof_factors == 0 || !c->tl_base || !c->graph_tl_exec ||
         (int64_t)c->prof_events.size() < 2 * n)
         return MF_ERR_STATE;
     for (int64_t i = 0; i < std::min(n, max); i++) {

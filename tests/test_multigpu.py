@@ -117,12 +117,14 @@ def test_gloo_world2_mapping_and_exchange():
 
 
 # ---------------------------------------------------------------- GPU (loopback ranks)
-def run_loopback(A, perm, R, values=None, b=None, split_all=True, junk_others=True, **opts):
+def run_loopback(A, perm, R, values=None, b=None, split_all=True, junk_others=True, profiling=0, **opts):
     from paper_conf_ipps_georgesgsc11_b200.exchange import LoopbackHub
     hub = LoopbackHub(R)
     solvers = [mf.Solver(nranks=R, rank=r, exchange=hub.for_rank(r), split_all=split_all, **opts) for r in range(R)]
     for S in solvers:
         S.analyze(A.n, A.colptr, A.rowind, perm)
+        if profiling:
+            S.set_profiling(profiling)
     vals = A.values if values is None else values
     errs = [None] * R
     xs = [None] * R
@@ -206,6 +208,36 @@ def test_loopback_manufactured_bit_exact(R, dims, opts):
         k = int(sn["sn_first"][s + 1] - sn["sn_first"][s])
         for r in (range(R) if top[s] else [int(owner[s])]):
             np.testing.assert_array_equal(solvers[r].panel(s, f, k), ref.panel(s, f, k))
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("profiling", [1, 2])
+def test_loopback_profiling_modes(profiling):
+    """Per-launch timing on P ranks (the top program's segments between exchange
+    points always run eagerly with events) leaves the factor bitwise unchanged; in
+    timeline mode every rank's local program has a timeline."""
+    import oracle
+    from workloads import grids as G
+    A0, p = grid("27pt", (12, 12, 12))
+    s0 = oracle.symbolic(A0, p, keep_struct=True)
+    A, Lx = G.manufactured(A0.n, s0.Lp, s0.Li, s0.perm, seed=1234)
+    ref = mf.Solver()
+    ref.analyze(A.n, A.colptr, A.rowind, s0.perm)
+    ref.factor(A.values)
+    R = 2
+    solvers, _ = run_loopback(A, s0.perm, R, profiling=profiling, panel_w=16)
+    owner, top, _, _ = solvers[0].mapping()
+    sn = ref.supernodes()
+    for s in range(ref.info()["nsuper"]):
+        f = int(sn["sn_rowptr"][s + 1] - sn["sn_rowptr"][s])
+        k = int(sn["sn_first"][s + 1] - sn["sn_first"][s])
+        for r in (range(R) if top[s] else [int(owner[s])]):
+            np.testing.assert_array_equal(solvers[r].panel(s, f, k), ref.panel(s, f, k))
+    for S in solvers:
+        assert sum(k["launches"] for k in S.kernel_stats()) > 0
+        if profiling == 2:
+            t0, t1 = S.launch_timeline()
+            assert (t1 >= t0).all()
 
 
 @pytest.mark.gpu
