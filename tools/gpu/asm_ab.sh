@@ -1,0 +1,19 @@
+# large-front assembly with the A entries gathered once per column: bitwise hash of c2's L vs the previous kernel, tests, times
+python - > gpurun_out/asm_hash.txt 2>&1 <<'PY'
+import sys, hashlib
+sys.path.insert(0, ".")
+import numpy as np
+import paper_conf_ipps_georgesgsc11_b200 as mf
+from workloads import grids as G
+for cfg in ("c2", "c3"):
+    c = G.CONFIGS[cfg]
+    A, p = G.make_config(c["kind"], c["N"])
+    S = mf.Solver()
+    S.analyze(A.n, A.colptr, A.rowind, p)
+    S.factor(A.values)
+    Lp, Li, Lx = S.export_L()
+    print(cfg, hashlib.sha256(np.ascontiguousarray(Lx).tobytes()).hexdigest()[:16])
+PY
+cat gpurun_out/asm_hash.txt
+timeout 900 python -m pytest tests -m gpu -q -x -k "fused or manufactured or parity or variant or nanfill or assemble or dup" > gpurun_out/asmtest.log 2>&1; tail -1 gpurun_out/asmtest.log
+timeout 600 python tools/time_factor.py c2 c3 c5 > gpurun_out/asm_ab.txt 2>&1; cat gpurun_out/asm_ab.txt
