@@ -1,4 +1,4 @@
-# tiny-front assembly with batched loads: bitwise hash of c2's L vs the previous kernel, tests, times
+# factor A/B driver: bitwise hash of c2 / c3 L (export_L), targeted factor tests, c2 / c3 / c5 times
 python - > gpurun_out/tiny_hash.txt 2>&1 <<'PY'
 import sys, hashlib
 sys.path.insert(0, ".")
