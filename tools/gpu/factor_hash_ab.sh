@@ -1,5 +1,5 @@
 # factor A/B driver: bitwise hash of c2 / c3 L (export_L), targeted factor tests, c2 / c3 / c5 times
-python - > gpurun_out/asm_hash.txt 2>&1 <<'PY'
+python - > gpurun_out/factor_hash.txt 2>&1 <<'PY'
 import sys, hashlib
 sys.path.insert(0, ".")
 import numpy as np
@@ -14,6 +14,6 @@ for cfg in ("c2", "c3"):
     Lp, Li, Lx = S.export_L()
     print(cfg, hashlib.sha256(np.ascontiguousarray(Lx).tobytes()).hexdigest()[:16])
 PY
-cat gpurun_out/asm_hash.txt
-timeout 900 python -m pytest tests -m gpu -q -x -k "fused or manufactured or parity or variant or nanfill or assemble or dup" > gpurun_out/asmtest.log 2>&1; tail -1 gpurun_out/asmtest.log
-timeout 600 python tools/time_factor.py c2 c3 c5 > gpurun_out/asm_ab.txt 2>&1; cat gpurun_out/asm_ab.txt
+cat gpurun_out/factor_hash.txt
+timeout 900 python -m pytest tests -m gpu -q -x -k "fused or manufactured or parity or variant or nanfill or assemble or dup" > gpurun_out/factortest_hash.log 2>&1; tail -1 gpurun_out/factortest_hash.log
+timeout 600 python tools/time_factor.py c2 c3 c5 > gpurun_out/factor_hash_ab.txt 2>&1; cat gpurun_out/factor_hash_ab.txt

@@ -1,2 +1,4 @@
-# dataflow-panel phase timeline (tools/ubench/panel_timeline.cu): new vs old potrf, bitwise hash
-for b in panel_timeline panel_timeline_old; do for a in "6545 6545 8" "15000 15000 8" "2000 1000 8" "1000 700 8" "333 250 8"; do echo "== $b $a"; timeout 60 ./tools/ubench/$b $a | grep -v "^row" | grep -E "^f=|hash|max|potrf steps|^band (0|3|7)"; done; done > gpurun_out/panel_tl3.txt 2>&1
+# dataflow-panel phase timeline (tools/ubench/panel_timeline.cu, built with the PANEL_TL hook) + fp64 latency / potrf part ubenches
+for a in "6545 6545 8" "15000 15000 8" "2000 1000 8"; do ./tools/ubench/panel_timeline $a | grep -v "^row"; done > gpurun_out/panel_tl.txt 2>&1
+./tools/ubench/lat >> gpurun_out/panel_tl.txt 2>&1
+./tools/ubench/potrf_parts >> gpurun_out/panel_tl.txt 2>&1
